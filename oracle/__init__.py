@@ -1,0 +1,206 @@
+"""ORACLE — TEST INFRASTRUCTURE ONLY.
+
+ctypes front-end for `oracle/oracle.c`, the plain single-threaded CPU
+implementation of what the hot path computes.
+Only `tests/`, `__graft_entry__.smoke()` and `bench.py`'s cpu_baseline /
+`--impl reference` legs may import this package.  It shares no code with the
+CUDA path in `paper_conf_ipps_xiaohmxw17_b200/` and never imports it.
+
+Every function here is pinned in tests/test_oracle_*.py against something
+other than itself (library routines, closed forms, brute force, special
+cases).  Parity unpinned: none of these functions (the paper's printed timings
+are context only).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+import subprocess
+from dataclasses import dataclass
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SRC = os.path.join(_HERE, "oracle.c")
+_LIB = os.path.join(_HERE, "liboracle.so")
+
+OK, ERR_ARG, ERR_OOM, ERR_NOT_SPD, ERR_BREAKDOWN, ERR_NO_CONVERGENCE = 0, 1, 3, 4, 5, 6
+PC = {"none": 0, "bj": 1, "ssor_ai": 2, "ilu0": 3}
+
+
+def build(force: bool = False) -> str:
+    """Compile liboracle.so with gcc (no FMA contraction: values round as written)."""
+    if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math",
+                               "-fPIC", "-shared", "-Wall", "-Wno-unused-label", "-o", _LIB, _SRC, "-lm"])
+    return _LIB
+
+
+_lib = None
+
+
+def lib():
+    global _lib
+    if _lib is None:
+        L = C.CDLL(build())
+        P = C.c_void_p
+        L.orc_assemble.argtypes = [C.c_int32, P, C.c_int64, P, P, P, P, P, C.POINTER(C.c_void_p)]
+        L.orc_assemble.restype = C.c_int
+        L.orc_info.argtypes = [P, C.POINTER(C.c_int32), C.POINTER(C.c_int64)]
+        L.orc_export.argtypes = [P] * 8
+        L.orc_free.argtypes = [P]
+        L.orc_expand.argtypes = [P]
+        L.orc_full_nnz.argtypes = [P]
+        L.orc_full_nnz.restype = C.c_int64
+        L.orc_full_export.argtypes = [P, P, P, P]
+        L.orc_spmv.argtypes = [P, P, P]
+        L.orc_spmv_rows.argtypes = [P, P, C.c_int64, P, P]
+        L.orc_bj_inv.argtypes = [P, P, C.POINTER(C.c_int32)]
+        L.orc_ssor_ai_apply.argtypes = [P, P, C.c_double, P, P]
+        L.orc_ilu0_factor.argtypes = [P]
+        L.orc_ilu0_apply.argtypes = [P, P, P]
+        L.orc_pcg.argtypes = [P, P, P, P, C.c_double, C.c_int32, C.c_int32, C.c_double,
+                              C.POINTER(C.c_int32), C.POINTER(C.c_double), P]
+        L.orc_ldlt_solve.argtypes = [P, P, P]
+        _lib = L
+    return _lib
+
+
+def _p(a: np.ndarray):
+    return a.ctypes.data_as(C.c_void_p)
+
+
+class OracleError(RuntimeError):
+    def __init__(self, code, what):
+        super().__init__(f"oracle {what} failed with status {code}")
+        self.code = code
+
+
+@dataclass
+class Structure:
+    row_ptr: np.ndarray
+    col_idx: np.ndarray
+    low_ptr: np.ndarray
+    low_row: np.ndarray
+    low_to_up: np.ndarray
+    diag: np.ndarray      # [n,6,6]
+    upper: np.ndarray     # [nnzb,6,6]
+
+
+class OracleMatrix:
+    """O-1 assembled matrix (upper-symmetric BSR6) owned by the C oracle."""
+
+    def __init__(self, n, kdiag, bi, bj, pen, e, g):
+        L = lib()
+        self._keep = [np.ascontiguousarray(kdiag, np.float64), np.ascontiguousarray(bi, np.int32),
+                      np.ascontiguousarray(bj, np.int32), np.ascontiguousarray(pen, np.float64),
+                      np.ascontiguousarray(e, np.float64), np.ascontiguousarray(g, np.float64)]
+        kd, bi_, bj_, pen_, e_, g_ = self._keep
+        h = C.c_void_p()
+        st = L.orc_assemble(int(n), _p(kd), int(bi_.shape[0]), _p(bi_), _p(bj_), _p(pen_), _p(e_), _p(g_),
+                            C.byref(h))
+        self._keep = None
+        if st != OK:
+            raise OracleError(st, "assemble")
+        self.h = h
+        nn, nz = C.c_int32(), C.c_int64()
+        L.orc_info(h, C.byref(nn), C.byref(nz))
+        self.n, self.nnzb = int(nn.value), int(nz.value)
+
+    @classmethod
+    def from_problem(cls, P):
+        return cls(P.n, P.kdiag, P.bi, P.bj, P.pen, P.e, P.g)
+
+    def __del__(self):
+        h = getattr(self, "h", None)
+        if h is not None and _lib is not None:
+            _lib.orc_free(h)
+            self.h = None
+
+    def export(self) -> Structure:
+        n, z = self.n, self.nnzb
+        s = Structure(np.empty(n + 1, np.int32), np.empty(z, np.int32), np.empty(n + 1, np.int32),
+                      np.empty(z, np.int32), np.empty(z, np.int32), np.empty((n, 6, 6)), np.empty((z, 6, 6)))
+        lib().orc_export(self.h, _p(s.row_ptr), _p(s.col_idx), _p(s.low_ptr), _p(s.low_row),
+                         _p(s.low_to_up), _p(s.diag), _p(s.upper))
+        return s
+
+    def full_csr(self):
+        """O-2 full scalar CSR as (indptr int64, indices int32, data float64)."""
+        L = lib()
+        nnz = L.orc_full_nnz(self.h)
+        if nnz < 0:
+            raise OracleError(ERR_OOM, "expand")
+        ip = np.empty(6 * self.n + 1, np.int64); ix = np.empty(nnz, np.int32); dv = np.empty(nnz)
+        L.orc_full_export(self.h, _p(ip), _p(ix), _p(dv))
+        return ip, ix, dv
+
+    def spmv(self, x):
+        x = np.ascontiguousarray(x, np.float64)
+        y = np.empty(6 * self.n)
+        st = lib().orc_spmv(self.h, _p(x), _p(y))
+        if st != OK:
+            raise OracleError(st, "spmv")
+        return y
+
+    def spmv_rows(self, rows, x):
+        rows = np.ascontiguousarray(rows, np.int64)
+        x = np.ascontiguousarray(x, np.float64)
+        y = np.empty(rows.shape[0])
+        lib().orc_spmv_rows(self.h, _p(rows), int(rows.shape[0]), _p(x), _p(y))
+        return y
+
+    def bj_inv(self):
+        dinv = np.empty((self.n, 6, 6))
+        bad = C.c_int32()
+        st = lib().orc_bj_inv(self.h, _p(dinv), C.byref(bad))
+        if st != OK:
+            raise OracleError(st, f"bj_inv (block {bad.value})")
+        return dinv
+
+    def ssor_ai_apply(self, r, omega=1.0):
+        dinv = self.bj_inv()
+        r = np.ascontiguousarray(r, np.float64)
+        z = np.empty_like(r)
+        st = lib().orc_ssor_ai_apply(self.h, _p(dinv), float(omega), _p(r), _p(z))
+        if st != OK:
+            raise OracleError(st, "ssor_ai_apply")
+        return z
+
+    def ilu0_apply(self, r):
+        st = lib().orc_ilu0_factor(self.h)
+        if st != OK:
+            raise OracleError(st, "ilu0_factor")
+        r = np.ascontiguousarray(r, np.float64)
+        z = np.empty_like(r)
+        lib().orc_ilu0_apply(self.h, _p(r), _p(z))
+        return z
+
+    def pcg(self, F, d0=None, tol=1e-10, maxit=10000, precond="bj", omega=1.0, trace=False):
+        """O-5 textbook PCG.  Returns (d, iters, rel_res, status[, trace[k, 6n]])."""
+        N = 6 * self.n
+        F = np.ascontiguousarray(F, np.float64)
+        d0 = np.zeros(N) if d0 is None else np.ascontiguousarray(d0, np.float64)
+        d = np.empty(N)
+        it, rr = C.c_int32(), C.c_double()
+        tr = np.zeros((maxit + 1, N)) if trace else None
+        st = lib().orc_pcg(self.h, _p(F), _p(d0), _p(d), float(tol), int(maxit), PC[precond], float(omega),
+                           C.byref(it), C.byref(rr), _p(tr) if trace else None)
+        if st not in (OK, ERR_NO_CONVERGENCE, ERR_BREAKDOWN):
+            raise OracleError(st, "pcg")
+        out = (d, int(it.value), float(rr.value), int(st))
+        if trace:
+            out = out + (tr[: int(it.value) + 1],)
+        return out
+
+    def ldlt_solve(self, b):
+        b = np.ascontiguousarray(b, np.float64)
+        x = np.empty_like(b)
+        st = lib().orc_ldlt_solve(self.h, _p(b), _p(x))
+        if st != OK:
+            raise OracleError(st, "ldlt_solve")
+        return x
+
+
+def assemble(P) -> OracleMatrix:
+    return OracleMatrix.from_problem(P)
