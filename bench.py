@@ -1,0 +1,358 @@
+#!/usr/bin/env python
+"""Benchmark of the DDA equation-solving hot path on B200 (BASELINE.json metric).
+
+One STEP = one pass of the whole hot path on device-resident synthetic input:
+  dda_build_matrix   (A1: springs -> upper-symmetric BSR6 + transpose map)
+  dda_bj_setup       (A3: 6x6 Cholesky inverses)
+  dda_pcg_solve      (A4-A6: block-Jacobi PCG to 1e-10, cold start d0 = 0;
+                      one persistent kernel: symmetric SpMV + fused vector ops)
+on the configs[4] workload at N=1: a ~1M-block jittered-brick slope (6M DOF),
+which fits one B200 (the matrix is 1.29 GB).  `value` = device ms per step
+(CUDA events on the launching stream, max over ranks); lower is better.
+
+Extra keys: `roofline` for the dominant kernel (the persistent PCG kernel,
+algorithmic bytes per launch / its CUDA-event duration vs the measured HBM
+copy peak), `spmv` (the standalone symmetric SpMV GB/s and % of HBM peak —
+the first half of the metric), `e2e` (dda_solve_host with pinned host
+buffers, copies inside the timed region), `cpu_baseline` (the oracle, one
+core, on a bounded sample), `clocks` (NVML, sampled during the timed region).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl reference] [--blocks N]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np
+
+METRIC = "BSR6 sym SpMV GB/s & % HBM peak; PCG solve ms to 1e-10 at 1/2/4/8 B200"
+UNIT = "ms"
+DEFAULT_BLOCKS = 1_000_000
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def bytes_per_row_spmv(u: float) -> float:
+    """Algorithmic bytes of one symmetric SpMV per block row:
+    D 288 + u*(V 288 + col 4 + low_row 4 + low_to_up 4) + row_ptr/low_ptr 8 + x 48 + y 48."""
+    return 392.0 + 300.0 * u
+
+
+def pcg_launch_bytes(n: int, u: float, iters: int) -> float:
+    """Algorithmic bytes of one k_pcg launch with block-Jacobi, d0 = 0:
+    init 432 B/row (F, Dinv read; d, r, z, p written), per iteration SpMV + 528 (phase B:
+    p, d, r, q, Dinv read; d, r, z written) + 144 (phase C: z, p read, p written), final
+    true-residual SpMV + 96 (F, q read)."""
+    S = bytes_per_row_spmv(u)
+    return n * (432.0 + iters * (S + 528.0 + 144.0) + S + 96.0)
+
+
+class ClockSampler:
+    """NVML sampler of SM clock and throttle reasons during the timed region."""
+
+    def __init__(self, index: int, period: float = 0.05):
+        self.index, self.period = index, period
+        self.samples, self.reasons = [], set()
+        self.max_mhz = None
+        self._stop = threading.Event()
+        self._t = None
+        self.ok = False
+
+    def __enter__(self):
+        try:
+            import pynvml as N
+            N.nvmlInit()
+            h = N.nvmlDeviceGetHandleByIndex(self.index)
+            self.max_mhz = N.nvmlDeviceGetMaxClockInfo(h, N.NVML_CLOCK_SM)
+            names = {
+                "gpu_idle": getattr(N, "nvmlClocksEventReasonGpuIdle", 0x1),
+                "applications_clocks_setting": 0x2,
+                "sw_power_cap": 0x4,
+                "hw_slowdown": 0x8,
+                "sync_boost": 0x10,
+                "sw_thermal_slowdown": 0x20,
+                "hw_thermal_slowdown": 0x40,
+                "hw_power_brake_slowdown": 0x80,
+                "display_clock_setting": 0x100,
+            }
+
+            def run():
+                while not self._stop.is_set():
+                    try:
+                        self.samples.append(N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_SM))
+                        fn = getattr(N, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
+                            N.nvmlDeviceGetCurrentClocksThrottleReasons
+                        mask = fn(h)
+                        for k, bit in names.items():
+                            if mask & bit and k != "gpu_idle":
+                                self.reasons.add(k)
+                    except Exception:
+                        pass
+                    time.sleep(self.period)
+
+            self._t = threading.Thread(target=run, daemon=True)
+            self._t.start()
+            self.ok = True
+        except Exception as e:  # no NVML: report it rather than guess
+            self.err = repr(e)
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": ["nvml_unavailable"]}
+        return {"sm_mhz": float(statistics.median(self.samples)), "sm_max_mhz": self.max_mhz,
+                "reasons": sorted(self.reasons), "samples": len(self.samples)}
+
+
+def dist_env():
+    return int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("RANK", "0")), int(os.environ.get("LOCAL_RANK", "0"))
+
+
+# ----------------------------------------------------------------------------- CPU oracle legs
+
+def oracle_step_sample(n_sample: int, seed: int = 1005):
+    """Oracle (one thread, as it stands) on a bounded sample of the workload: the full
+    step (assembly O-1 + expansion O-2, block inverses, PCG to 1e-10) on a slope of
+    ~n_sample blocks from the same recipe.  Returns (seconds, n, iters)."""
+    import oracle
+    from synth import make_slope, preset
+    P = make_slope(preset(n_sample, seed=seed))
+    t0 = time.perf_counter()
+    M = oracle.assemble(P)
+    M.full_csr()
+    d, it, rr, st = M.pcg(P.F, tol=1e-10, maxit=10000, precond="bj")
+    t1 = time.perf_counter()
+    return t1 - t0, P.n, it
+
+
+def run_reference(args):
+    """--impl reference: the oracle timed as it stands on the host cores (rank 0 only)."""
+    world, rank, _ = dist_env()
+    if rank != 0:
+        return
+    n_full = args.blocks
+    n_s = args.ref_sample_blocks
+    import oracle
+    oracle.build()
+    for _ in range(args.warmup):
+        oracle_step_sample(n_s)
+    times, its, ns = [], [], []
+    for _ in range(args.steps):
+        s, n_act, it = oracle_step_sample(n_s)
+        times.append(s); its.append(it); ns.append(n_act)
+    n_act = ns[0]
+    scale = n_full / n_act
+    ms = 1000.0 * statistics.median(times) * scale
+    sample = (f"oracle full step (assembly+expansion, BJ inverses, PCG to 1e-10) on a {n_act}-block slope "
+              f"from the same recipe ({its[0]} iters), 1 thread, scaled x{scale:.2f} by block count to "
+              f"the {n_full}-block workload")
+    line = {"impl": "reference", "metric": METRIC, "value": ms, "unit": UNIT, "higher_is_better": False,
+            "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": workload_name(n_full)},
+            "cpu_baseline": {"value": ms, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "e2e": {"value": ms, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def workload_name(n):
+    return (f"slope-{n // 1000}k: jittered-brick slope (configs[4] at N=1), ~{n} blocks = {6 * n} DOF, "
+            f"~5 contacts/block; assemble + BJ setup + BJ-PCG to 1e-10 (cold start)")
+
+
+# ----------------------------------------------------------------------------- our arm
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--blocks", type=int, default=DEFAULT_BLOCKS)
+    ap.add_argument("--precond", default="bj")
+    ap.add_argument("--spmv-reps", type=int, default=20)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--cpu-sample-blocks", type=int, default=65_536)
+    ap.add_argument("--ref-sample-blocks", type=int, default=16_384)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        print("warning: --warmup < 3 violates the timing rules; using 3", file=sys.stderr)
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+        return
+
+    import torch
+    world, rank, local = dist_env()
+    if world != args.gpus:
+        if world == 1 and args.gpus > 1:
+            raise SystemExit("launch N>1 with torchrun (one process per GPU)")
+    torch.cuda.set_device(local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    import __graft_entry__
+    __graft_entry__.build() if rank == 0 else None
+    if world > 1:
+        torch.distributed.barrier()
+    import paper_conf_ipps_xiaohmxw17_b200 as dda
+    from synth import make_slope, preset
+
+    if world > 1:
+        raise SystemExit("row-partitioned multi-GPU solve: not in this build yet (DESIGN.md §7)")
+
+    P = make_slope(preset(args.blocks, seed=1005))
+    t = dda.problem_to_device(P)
+    stream = torch.cuda.current_stream()
+    hbm_peak, peak_src = measured_peaks()
+
+    def step(ev=None):
+        if ev: ev[0].record(stream)
+        K = dda.build_matrix(t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+        if ev: ev[1].record(stream)
+        K.bj_setup()
+        if ev: ev[2].record(stream)
+        d, it, rr, st = K.pcg_solve(t["F"], tol=1e-10, maxit=10000, precond=args.precond)
+        if ev: ev[3].record(stream)
+        return K, d, it, rr, st
+
+    for _ in range(args.warmup):
+        K, d, it, rr, st = step()
+        K.free()
+    torch.cuda.synchronize()
+
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(4)] for _ in range(args.steps)]
+    start, stop = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    results = []
+    l0 = dda.launch_count()
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        start.record(stream)
+        for k in range(args.steps):
+            K, d, it, rr, st = step(evs[k])
+            results.append((K.n, K.nnzb, it, rr, st))
+            K.free()
+        stop.record(stream)
+        torch.cuda.synchronize()
+    launches = dda.launch_count() - l0
+    total_ms = start.elapsed_time(stop)
+    ms_step = total_ms / args.steps
+    if world > 1:
+        tt = torch.tensor([ms_step], device="cuda")
+        torch.distributed.all_reduce(tt, op=torch.distributed.ReduceOp.MAX)
+        ms_step = float(tt.item())
+    ph_build = statistics.median(e[0].elapsed_time(e[1]) for e in evs)
+    ph_bj = statistics.median(e[1].elapsed_time(e[2]) for e in evs)
+    ph_pcg = [e[2].elapsed_time(e[3]) for e in evs]
+    n, nnzb, iters, rel_res, status = results[-1]
+    assert all(r[4] == dda.OK for r in results), results
+    assert rel_res <= 1e-10 * 1.01, rel_res
+    u = nnzb / n
+    pcg_ms = statistics.mean(ph_pcg)
+    pcg_bytes = pcg_launch_bytes(n, u, iters)
+    ach = pcg_bytes / (pcg_ms * 1e-3) / 1e9
+
+    # ---- standalone symmetric SpMV (metric's first half), back to back (hot, as PCG sees it)
+    K = dda.build_matrix(t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+    x = torch.rand(6 * n, dtype=torch.float64, device="cuda") * 2 - 1
+    y = torch.empty_like(x)
+    for _ in range(3):
+        K.spmv(x, y)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(args.spmv_reps):
+        K.spmv(x, y)
+    e1.record(stream)
+    torch.cuda.synchronize()
+    spmv_ms = e0.elapsed_time(e1) / args.spmv_reps
+    spmv_bytes = n * bytes_per_row_spmv(u)
+    spmv_gbs = spmv_bytes / (spmv_ms * 1e-3) / 1e9
+    K.free()
+    del x, y
+
+    # ---- e2e: dda_solve_host, pinned host buffers, H2D + D2H inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        pin = lambda a: torch.from_numpy(a).pin_memory()
+        hk, hbi, hbj, hpen, he, hg, hF = (pin(P.kdiag), pin(P.bi), pin(P.bj), pin(P.pen), pin(P.e), pin(P.g), pin(P.F))
+        hd = torch.empty(6 * n, dtype=torch.float64).pin_memory()
+        dda.solve_host(hk, hbi, hbj, hpen, he, hg, hF, out=hd.numpy())   # warm
+        torch.cuda.synchronize()
+        e2e_ms = []
+        for _ in range(max(1, min(args.steps, 3))):
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            _, it2, rr2, st2 = dda.solve_host(hk, hbi, hbj, hpen, he, hg, hF, out=hd.numpy())
+            a1.record(stream)
+            torch.cuda.synchronize()
+            e2e_ms.append(a0.elapsed_time(a1))
+        h2d = sum(a.numel() * a.element_size() for a in (hk, hbi, hbj, hpen, he, hg, hF))
+        e2e = {"value": statistics.median(e2e_ms), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": int(hd.numel() * 8), "api": "dda_solve_host (C ABI, pinned host buffers)"}
+
+    # ---- CPU oracle baseline (rank 0, N=1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        s, n_s, it_s = oracle_step_sample(args.cpu_sample_blocks)
+        scale = n / n_s
+        cpu = {"value": 1000.0 * s * scale, "unit": UNIT, "cores": 1, "kind": "oracle",
+               "sample": (f"oracle full step (assembly+expansion, BJ inverses, PCG to 1e-10: {it_s} iters) on a "
+                          f"{n_s}-block slope of the same recipe, 1 thread, {s:.1f} s, scaled x{scale:.2f} by "
+                          f"block count"), "host_cores": os.cpu_count()}
+
+    line = {
+        "metric": METRIC, "value": ms_step, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": False, "scaling": "strong",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": workload_name(args.blocks), "n_blocks": n, "dof": 6 * n, "springs": P.m,
+                   "contacts": P.n_contacts, "nnzb_upper": nnzb, "u": round(u, 3), "precond": args.precond,
+                   "tol": 1e-10, "start": "cold (d0 = 0)",
+                   "l2": f"inputs larger than L2 (matrix {(n * 288 + nnzb * 300) / 1e9:.2f} GB vs 126 MB L2); no flush",
+                   "parallelism": f"dp{world}" if world > 1 else "single GPU",
+                   "step": "dda_build_matrix + dda_bj_setup + dda_pcg_solve"},
+        "phases_ms": {"assemble": ph_build, "bj_setup": ph_bj, "pcg": pcg_ms, "pcg_iters": iters,
+                      "pcg_us_per_iter": 1000.0 * pcg_ms / max(iters, 1), "true_rel_res": rel_res},
+        "roofline": {"kernel": "k_pcg (persistent PCG: SpMV + fused vector phases)", "bound": "hbm",
+                     "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
+                     "traffic": None, "peak_source": peak_src,
+                     "algorithmic_bytes_per_launch": pcg_bytes},
+        "spmv": {"kernel": "k_spmv<FULL>", "ms": spmv_ms, "gbs": spmv_gbs, "frac_hbm": spmv_gbs / hbm_peak,
+                 "gflops": n * (72 + 144 * u) / (spmv_ms * 1e-3) / 1e9, "bytes": spmv_bytes,
+                 "timing": "back to back (hot), inputs > L2"},
+        "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": int(launches),
+        "clocks": clk.summary(),
+    }
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

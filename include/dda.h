@@ -1,0 +1,190 @@
+/*
+ * dda.h — C ABI of the B200-native DDA equation-solving hot path.
+ *
+ * The path is the open-close inner-loop solve K·d = F of 2-D Discontinuous
+ * Deformation Analysis (§IV): K is the global
+ * stiffness matrix, "naturally blocky and symmetric", each entry a 6x6
+ * sub-matrix, all diagonal sub-matrices nonzero, a_ij != 0 only if blocks i and
+ * j are in contact, and "only the upper entry of A is computed and stored"
+ * (P:102).  K is solved by preconditioned conjugate gradients with
+ * block-Jacobi, SSOR approximate inverse or ILU(0).
+ *
+ * Conventions (every entry point):
+ *  - Block ids are 0-based int32; the DOFs of block b are (u0, v0, r0, ex, ey,
+ *    gxy) at global indices 6b..6b+5 (reading Z11).  Values are IEEE fp64.
+ *  - "device" pointers are CUDA device (or managed) memory owned by the caller
+ *    and valid for the duration of the call; "host" pointers are host memory
+ *    (pinned memory gives the fastest copies).  No pointer is retained.
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *    stream).  Work is stream-ordered; calls documented as "synchronising"
+ *    wait for the stream before returning.
+ *  - Every status is returned, never thrown; there is no global error state.
+ *    dda_status_string() names a status.
+ *  - A dda_matrix_t is an opaque handle owning device arrays; it is bound to the
+ *    device that was current when it was built and must be released with
+ *    dda_matrix_free().  Handles are not thread-safe: do not use one handle
+ *    from two host threads at once.
+ */
+#ifndef DDA_H
+#define DDA_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct dda_matrix *dda_matrix_t;
+
+typedef enum {
+    DDA_OK = 0,
+    DDA_ERR_ARG = 1,             /* invalid argument (sizes, null pointers, ids, tol, maxit, penalties) */
+    DDA_ERR_CUDA = 2,            /* a CUDA runtime call failed (message via dda_last_cuda_error) */
+    DDA_ERR_OOM = 3,             /* device allocation failed */
+    DDA_ERR_NOT_SPD = 4,         /* a (pivot) diagonal block is not symmetric positive definite */
+    DDA_ERR_BREAKDOWN = 5,       /* PCG breakdown: p^T K p <= 0, r^T z <= 0 or not finite (Z19) */
+    DDA_ERR_NO_CONVERGENCE = 6,  /* maxit reached before ||r|| <= tol ||F|| */
+    DDA_ERR_NCCL = 7             /* reserved for the distributed solver */
+} dda_status_t;
+
+typedef enum {
+    DDA_PC_NONE = 0,     /* plain CG */
+    DDA_PC_BJ = 1,       /* block Jacobi: z_i = D_i^{-1} r_i (Table I) */
+    DDA_PC_SSOR_AI = 2,  /* SSOR approximate inverse (ref [36]; reading Z14) */
+    DDA_PC_ILU0 = 3      /* block ILU(0) = IC(0) for symmetric K (reading Z15) */
+} dda_precond_t;
+
+/*
+ * A1 — Assembly (§III.C; Fig. 4 steps: per-contact sub-matrix →
+ * sort by block number → boundary flags → scan → segment sums).
+ *
+ * Builds K from per-block diagonal terms and m contact springs.  Spring s =
+ * (bi[s], bj[s], pen[s], e[s][6], g[s][6]) couples vertex block i = bi[s] and
+ * edge block j = bj[s] and contributes
+ *      a_ii += p e e^T,   a_jj += p g g^T,   a_ij += p e g^T  (a_ji = a_ij^T).
+ * The stored off-diagonal block is (min(i,j), max(i,j)); it receives p e g^T
+ * if i < j and its transpose if i > j (reading Z7).  Every entry is the sum,
+ * in increasing spring index, of the products (p*e[r])*g[c] rounded as
+ * written (no FMA contraction), so values are bit-identical to the
+ * definition (reading Z8); the diagonal starts from kdiag's upper triangle
+ * (the lower triangle of kdiag is ignored, reading Z9).  A spring with p = 0
+ * still creates its block (reading Z10).  m = 0 is valid (K block diagonal).
+ *
+ *  n_blocks     number of blocks n > 0 (6n unknowns)
+ *  kdiag        device, [n][6][6] row-major: elastic + inertia + fixed-point
+ *               terms of each block; upper triangle read
+ *  n_springs    m >= 0
+ *  bi, bj       device, [m] int32 block ids in [0, n), bi[s] != bj[s]
+ *  pen          device, [m] penalties, finite and >= 0
+ *  e, g         device, [m][6] spring vectors of block bi / bj
+ *  stream       cudaStream_t
+ *  out          receives the new handle (NULL on failure)
+ * Errors: DDA_ERR_ARG for n <= 0, m < 0, a NULL pointer with m > 0, an id out
+ * of range, bi == bj, or a negative / non-finite penalty (the id and penalty
+ * checks run on the device and are reported after the call synchronises the
+ * stream once to size the output).  DDA_ERR_OOM / DDA_ERR_CUDA otherwise.
+ * Synchronising.
+ */
+dda_status_t dda_build_matrix(int32_t n_blocks, const double *kdiag, int64_t n_springs,
+                              const int32_t *bi, const int32_t *bj, const double *pen,
+                              const double *e, const double *g, void *stream, dda_matrix_t *out);
+
+/*
+ * A1 (inner-loop variant, NEXT-1) — value-only re-assembly.  Same springs
+ * (same count, same (bi, bj) sequence) with new penalties / vectors / diagonal
+ * terms: reuses the cached sort permutation and structure (contacts are fixed
+ * within a time step; only states and penalties change in the open-close loop,
+ * P:27).  The caller guarantees bi/bj are unchanged (not checked
+ * beyond the count).  Invalidates preconditioner state.  Stream-ordered.
+ */
+dda_status_t dda_update_values(dda_matrix_t K, const double *kdiag, int64_t n_springs,
+                               const double *pen, const double *e, const double *g, void *stream);
+
+/* Sizes of a built matrix: n and the number of stored upper off-diagonal blocks. */
+dda_status_t dda_matrix_info(dda_matrix_t K, int32_t *n_blocks, int64_t *nnzb_upper);
+
+/*
+ * A2 — Canonical export.  Host buffers, each may be NULL:
+ *  row_ptr   [n+1]   upper CSR offsets; the paper's row-up-i[i] = row_ptr[i+1]
+ *  col_idx   [nnzb]  strictly increasing within a row, every entry > its row
+ *  low_ptr   [n+1]   CSR offsets of the virtual lower part; row-low-i[i] = low_ptr[i+1]
+ *  low_row   [nnzb]  for lower position t in row i: the k < i with (k,i) stored, ascending
+ *  low_to_up [nnzb]  row-low-p: position of block (k,i) in the upper storage
+ *  diag      [n][36] row-major D_i
+ *  upper     [nnzb][36] row-major V_ij, in row_ptr order
+ * Internal device layouts are private.  Synchronising.
+ */
+dda_status_t dda_matrix_export(dda_matrix_t K, int32_t *row_ptr, int32_t *col_idx, int32_t *low_ptr,
+                               int32_t *low_row, int32_t *low_to_up, double *diag, double *upper);
+
+/*
+ * A4 — Symmetric block SpMV  y = K x  (§IV.B), from the upper
+ * storage only: y_i = D_i x_i + sum_{j>i} V_ij x_j + sum_{k<i} V_ki^T x_k.
+ * Atomic-free and deterministic (bitwise run-to-run).
+ *  x, y   device, [6n]; must not alias.   Stream-ordered.
+ */
+dda_status_t dda_spmv(dda_matrix_t K, const double *x, double *y, void *stream);
+
+/*
+ * A3 — Block-Jacobi setup (Table I "construction" P:174): D_i^{-1} for
+ * every diagonal block by 6x6 Cholesky.  Called implicitly by dda_pcg_solve;
+ * exposed for testing.  If dinv (device, [n][36] row-major) is non-NULL the
+ * inverses are also written there.  DDA_ERR_NOT_SPD if some D_i is not SPD;
+ * *bad_block (host, may be NULL) receives its index (-1 otherwise).
+ * Synchronising.
+ */
+dda_status_t dda_bj_setup(dda_matrix_t K, double *dinv, int32_t *bad_block, void *stream);
+
+/*
+ * A7/A8 — Preconditioner application z = M^{-1} r (device [6n] each) for
+ * testing the preconditioners in isolation.  Sets the preconditioner up first
+ * if needed.  omega is used by DDA_PC_SSOR_AI only.  Synchronising.
+ */
+dda_status_t dda_precond_apply(dda_matrix_t K, dda_precond_t pc, double omega, const double *r, double *z,
+                               void *stream);
+
+/*
+ * A5/A6 — PCG solve of K d = F, warm-started from d0
+ * ("the equation solution of the previous step is the initial value").
+ *  F       device [6n]
+ *  d0      device [6n] initial guess, or NULL for zero; may alias d
+ *  d       device [6n] solution
+ *  tol     > 0: stop when ||r_k||_2 <= tol ||F||_2 on the recursive residual (reading Z1)
+ *  maxit   >= 0 (the paper's DDA policy is 200)
+ *  pc      preconditioner;  omega: SSOR-AI relaxation (1.0 default, ignored otherwise)
+ *  iters   host out: iterations performed
+ *  rel_res host out: TRUE relative residual ||F - K d||_2 / ||F||_2 (one extra SpMV)
+ * The whole iteration runs on the device (one persistent cooperative kernel);
+ * the host reads the result once at the end.  Returns DDA_OK,
+ * DDA_ERR_NO_CONVERGENCE (d, iters, rel_res still filled), DDA_ERR_BREAKDOWN
+ * (d = last iterate), DDA_ERR_NOT_SPD (preconditioner setup).  F = 0 gives
+ * d = 0, iters = 0, rel_res = 0, DDA_OK (reading Z2).  Synchronising.
+ */
+dda_status_t dda_pcg_solve(dda_matrix_t K, const double *F, const double *d0, double *d, double tol,
+                           int32_t maxit, dda_precond_t pc, double omega, int32_t *iters, double *rel_res,
+                           void *stream);
+
+/*
+ * End-to-end entry with HOST buffers (the benchmark's e2e leg): copies the
+ * inputs host→device, assembles, sets up the preconditioner, solves, copies d
+ * device→host and frees everything.  Arguments as dda_build_matrix and
+ * dda_pcg_solve, all host pointers; d0 may be NULL.  Synchronising.
+ */
+dda_status_t dda_solve_host(int32_t n_blocks, const double *kdiag, int64_t n_springs, const int32_t *bi,
+                            const int32_t *bj, const double *pen, const double *e, const double *g,
+                            const double *F, const double *d0, double *d, double tol, int32_t maxit,
+                            dda_precond_t pc, double omega, int32_t *iters, double *rel_res, void *stream);
+
+/* Number of kernel launches the library has issued in this process (for the
+ * benchmark's gpu_launches count). */
+int64_t dda_launch_count(void);
+
+void dda_matrix_free(dda_matrix_t K);
+const char *dda_status_string(dda_status_t s);
+/* Text of the last CUDA error seen by this thread ("" if none). */
+const char *dda_last_cuda_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DDA_H */

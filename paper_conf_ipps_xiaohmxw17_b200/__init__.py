@@ -1,0 +1,252 @@
+"""B200-native DDA equation-solving hot path: thin Python binding of libdda.so.
+
+Argument marshalling only — every step of the path (assembly, SpMV,
+block-Jacobi setup, PCG, SSOR-AI) runs in the CUDA kernels behind the C ABI
+declared in include/dda.h.  PyTorch supplies device memory and streams.
+There is no CPU fallback: if the shared library is missing or no CUDA device
+is present the calls raise.
+
+Names follow the ABI: build_matrix, spmv, bj_setup, precond_apply, pcg_solve,
+update_values, solve_host (§III.C P:100-110 and §IV).
+"""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libdda.so")
+
+OK, ERR_ARG, ERR_CUDA, ERR_OOM, ERR_NOT_SPD, ERR_BREAKDOWN, ERR_NO_CONVERGENCE, ERR_NCCL = range(8)
+PRECOND = {"none": 0, "bj": 1, "ssor_ai": 2, "ilu0": 3}
+
+# symbols declared in include/dda.h (checked by tests/test_abi.py)
+ABI_SYMBOLS = ("dda_build_matrix", "dda_update_values", "dda_matrix_info", "dda_matrix_export", "dda_spmv",
+               "dda_bj_setup", "dda_precond_apply", "dda_pcg_solve", "dda_solve_host", "dda_launch_count",
+               "dda_matrix_free", "dda_status_string", "dda_last_cuda_error")
+
+_lib = None
+
+
+class DDAError(RuntimeError):
+    def __init__(self, status: int, what: str):
+        name = lib().dda_status_string(status).decode() if _lib is not None else str(status)
+        detail = lib().dda_last_cuda_error().decode() if (_lib is not None and status == ERR_CUDA) else ""
+        super().__init__(f"{what}: {name}{' (' + detail + ')' if detail else ''}")
+        self.status = status
+
+
+def lib() -> C.CDLL:
+    """Load libdda.so (build it first with __graft_entry__.build() or _build.py)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: run `python __graft_entry__.py build` (no CPU fallback)")
+        L = C.CDLL(LIB_PATH)
+        P, I32, I64, D = C.c_void_p, C.c_int32, C.c_int64, C.c_double
+        st = C.c_int
+        L.dda_build_matrix.argtypes = [I32, P, I64, P, P, P, P, P, P, C.POINTER(P)]
+        L.dda_build_matrix.restype = st
+        L.dda_update_values.argtypes = [P, P, I64, P, P, P, P]
+        L.dda_update_values.restype = st
+        L.dda_matrix_info.argtypes = [P, C.POINTER(I32), C.POINTER(I64)]
+        L.dda_matrix_info.restype = st
+        L.dda_matrix_export.argtypes = [P] * 8
+        L.dda_matrix_export.restype = st
+        L.dda_spmv.argtypes = [P, P, P, P]
+        L.dda_spmv.restype = st
+        L.dda_bj_setup.argtypes = [P, P, C.POINTER(I32), P]
+        L.dda_bj_setup.restype = st
+        L.dda_precond_apply.argtypes = [P, st, D, P, P, P]
+        L.dda_precond_apply.restype = st
+        L.dda_pcg_solve.argtypes = [P, P, P, P, D, I32, st, D, C.POINTER(I32), C.POINTER(D), P]
+        L.dda_pcg_solve.restype = st
+        L.dda_solve_host.argtypes = [I32, P, I64, P, P, P, P, P, P, P, P, D, I32, st, D,
+                                     C.POINTER(I32), C.POINTER(D), P]
+        L.dda_solve_host.restype = st
+        L.dda_launch_count.argtypes = []
+        L.dda_launch_count.restype = I64
+        L.dda_matrix_free.argtypes = [P]
+        L.dda_matrix_free.restype = None
+        L.dda_status_string.argtypes = [st]
+        L.dda_status_string.restype = C.c_char_p
+        L.dda_last_cuda_error.argtypes = []
+        L.dda_last_cuda_error.restype = C.c_char_p
+        _lib = L
+    return _lib
+
+
+def _torch():
+    import torch
+    return torch
+
+
+def _stream(stream=None) -> int:
+    torch = _torch()
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return int(s.cuda_stream)
+
+
+def _dev(t, dtype, shape=None, name="tensor"):
+    torch = _torch()
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise TypeError(f"{name} must be a CUDA tensor")
+    if t.dtype != dtype:
+        raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    if shape is not None and tuple(t.shape) != tuple(shape):
+        raise ValueError(f"{name} has shape {tuple(t.shape)}, expected {tuple(shape)}")
+    return C.c_void_p(t.data_ptr())
+
+
+def _check(st: int, what: str):
+    if st != OK:
+        raise DDAError(st, what)
+
+
+def launch_count() -> int:
+    return int(lib().dda_launch_count())
+
+
+class Matrix:
+    """Upper-symmetric BSR6 stiffness matrix K owned by the library (A1)."""
+
+    def __init__(self, handle: C.c_void_p):
+        self._h = handle
+        n, z = C.c_int32(), C.c_int64()
+        _check(lib().dda_matrix_info(handle, C.byref(n), C.byref(z)), "dda_matrix_info")
+        self.n, self.nnzb = int(n.value), int(z.value)
+
+    @property
+    def handle(self):
+        if self._h is None:
+            raise ValueError("matrix has been freed")
+        return self._h
+
+    def free(self):
+        if self._h is not None and _lib is not None:
+            _lib.dda_matrix_free(self._h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+    def export(self) -> dict:
+        n, z = self.n, self.nnzb
+        out = {"row_ptr": np.empty(n + 1, np.int32), "col_idx": np.empty(z, np.int32),
+               "low_ptr": np.empty(n + 1, np.int32), "low_row": np.empty(z, np.int32),
+               "low_to_up": np.empty(z, np.int32), "diag": np.empty((n, 6, 6)), "upper": np.empty((z, 6, 6))}
+        p = {k: v.ctypes.data_as(C.c_void_p) for k, v in out.items()}
+        _check(lib().dda_matrix_export(self.handle, p["row_ptr"], p["col_idx"], p["low_ptr"], p["low_row"],
+                                       p["low_to_up"], p["diag"], p["upper"]), "dda_matrix_export")
+        return out
+
+    def spmv(self, x, y=None, stream=None):
+        torch = _torch()
+        N = 6 * self.n
+        xp = _dev(x, torch.float64, (N,), "x")
+        if y is None:
+            y = torch.empty_like(x)
+        yp = _dev(y, torch.float64, (N,), "y")
+        _check(lib().dda_spmv(self.handle, xp, yp, C.c_void_p(_stream(stream))), "dda_spmv")
+        return y
+
+    def bj_setup(self, full: bool = False, stream=None):
+        torch = _torch()
+        out = torch.empty((self.n, 6, 6), dtype=torch.float64, device="cuda") if full else None
+        bad = C.c_int32()
+        st = lib().dda_bj_setup(self.handle, C.c_void_p(out.data_ptr()) if full else None, C.byref(bad),
+                                C.c_void_p(_stream(stream)))
+        if st != OK:
+            raise DDAError(st, f"dda_bj_setup (block {bad.value})")
+        return out
+
+    def precond_apply(self, r, precond="bj", omega=1.0, stream=None):
+        torch = _torch()
+        N = 6 * self.n
+        z = torch.empty_like(r)
+        _check(lib().dda_precond_apply(self.handle, PRECOND[precond], float(omega),
+                                       _dev(r, torch.float64, (N,), "r"), _dev(z, torch.float64, (N,), "z"),
+                                       C.c_void_p(_stream(stream))), "dda_precond_apply")
+        return z
+
+    def pcg_solve(self, F, d0=None, d=None, tol=1e-10, maxit=10000, precond="bj", omega=1.0, stream=None,
+                  raise_on_fail=False):
+        """Returns (d, iters, rel_res, status); status OK / NO_CONVERGENCE / BREAKDOWN."""
+        torch = _torch()
+        N = 6 * self.n
+        Fp = _dev(F, torch.float64, (N,), "F")
+        d0p = _dev(d0, torch.float64, (N,), "d0") if d0 is not None else None
+        if d is None:
+            d = torch.empty_like(F)
+        dp = _dev(d, torch.float64, (N,), "d")
+        it, rr = C.c_int32(), C.c_double()
+        st = lib().dda_pcg_solve(self.handle, Fp, d0p, dp, float(tol), int(maxit), PRECOND[precond], float(omega),
+                                 C.byref(it), C.byref(rr), C.c_void_p(_stream(stream)))
+        if st not in (OK, ERR_NO_CONVERGENCE, ERR_BREAKDOWN) or (raise_on_fail and st != OK):
+            raise DDAError(st, "dda_pcg_solve")
+        return d, int(it.value), float(rr.value), int(st)
+
+    def update_values(self, kdiag, pen, e, g, stream=None):
+        torch = _torch()
+        m = int(pen.shape[0])
+        _check(lib().dda_update_values(self.handle, _dev(kdiag, torch.float64, (self.n, 6, 6), "kdiag"), m,
+                                       _dev(pen, torch.float64, (m,), "pen"), _dev(e, torch.float64, (m, 6), "e"),
+                                       _dev(g, torch.float64, (m, 6), "g"), C.c_void_p(_stream(stream))),
+               "dda_update_values")
+
+
+def build_matrix(kdiag, bi, bj, pen, e, g, stream=None) -> Matrix:
+    """A1: assemble K from diagonal terms [n,6,6] and springs (bi, bj, pen, e[m,6], g[m,6])."""
+    torch = _torch()
+    n = int(kdiag.shape[0])
+    m = int(bi.shape[0])
+    h = C.c_void_p()
+    st = lib().dda_build_matrix(n, _dev(kdiag, torch.float64, (n, 6, 6), "kdiag"), m,
+                                _dev(bi, torch.int32, (m,), "bi"), _dev(bj, torch.int32, (m,), "bj"),
+                                _dev(pen, torch.float64, (m,), "pen"), _dev(e, torch.float64, (m, 6), "e"),
+                                _dev(g, torch.float64, (m, 6), "g"), C.c_void_p(_stream(stream)), C.byref(h))
+    _check(st, "dda_build_matrix")
+    return Matrix(h)
+
+
+def build_from_problem(P, device="cuda") -> Matrix:
+    """Copy a synth.SlopeProblem to the device and assemble it."""
+    t = problem_to_device(P, device)
+    return build_matrix(t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+
+
+def problem_to_device(P, device="cuda") -> dict:
+    torch = _torch()
+    return {"kdiag": torch.from_numpy(P.kdiag).to(device), "bi": torch.from_numpy(P.bi).to(device),
+            "bj": torch.from_numpy(P.bj).to(device), "pen": torch.from_numpy(P.pen).to(device),
+            "e": torch.from_numpy(P.e).to(device), "g": torch.from_numpy(P.g).to(device),
+            "F": torch.from_numpy(P.F).to(device)}
+
+
+def solve_host(kdiag, bi, bj, pen, e, g, F, d0=None, tol=1e-10, maxit=10000, precond="bj", omega=1.0,
+               out=None, stream=None):
+    """End-to-end: host (numpy / pinned CPU tensor) inputs -> host solution, via dda_solve_host."""
+    def ptr(a, dtype):
+        if hasattr(a, "data_ptr"):
+            return C.c_void_p(a.data_ptr())
+        assert a.dtype == dtype and a.flags["C_CONTIGUOUS"]
+        return a.ctypes.data_as(C.c_void_p)
+    n = int(kdiag.shape[0]); m = int(bi.shape[0])
+    if out is None:
+        out = np.empty(6 * n)
+    it, rr = C.c_int32(), C.c_double()
+    st = lib().dda_solve_host(n, ptr(kdiag, np.float64), m, ptr(bi, np.int32), ptr(bj, np.int32),
+                              ptr(pen, np.float64), ptr(e, np.float64), ptr(g, np.float64), ptr(F, np.float64),
+                              ptr(d0, np.float64) if d0 is not None else None, ptr(out, np.float64), float(tol),
+                              int(maxit), PRECOND[precond], float(omega), C.byref(it), C.byref(rr),
+                              C.c_void_p(_stream(stream)))
+    if st not in (OK, ERR_NO_CONVERGENCE, ERR_BREAKDOWN):
+        raise DDAError(st, "dda_solve_host")
+    return out, int(it.value), float(rr.value), int(st)

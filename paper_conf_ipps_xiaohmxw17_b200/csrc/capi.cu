@@ -1,0 +1,82 @@
+// Host-side bookkeeping of the C ABI: status strings, CUDA error capture,
+// launch counting, device properties.
+#include <atomic>
+#include <cstdio>
+#include <cstring>
+
+#include "dda_internal.cuh"
+
+namespace dda {
+namespace {
+std::atomic<int64_t> g_launches{0};
+thread_local char g_last_err[256] = "";
+}  // namespace
+
+void note_launch(int k) { g_launches.fetch_add(k, std::memory_order_relaxed); }
+
+dda_status_t cuda_fail(cudaError_t e) {
+    std::snprintf(g_last_err, sizeof g_last_err, "%s: %s", cudaGetErrorName(e), cudaGetErrorString(e));
+    return e == cudaErrorMemoryAllocation ? DDA_ERR_OOM : DDA_ERR_CUDA;
+}
+
+int device_sms() {
+    static int cached_dev = -1, cached = 148;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev != cached_dev) {
+        int v = 0;
+        if (cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev) == cudaSuccess && v > 0) cached = v;
+        cached_dev = dev;
+    }
+    return cached;
+}
+
+cudaError_t dev_alloc(void** p, size_t bytes, cudaStream_t st) {
+    static int configured = -1;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (configured != dev) {
+        cudaMemPool_t pool;
+        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+            uint64_t keep = UINT64_MAX;
+            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+        }
+        configured = dev;
+    }
+    return cudaMallocAsync(p, bytes, st);
+}
+
+void dev_free(void* p) { cudaFreeAsync(p, 0); }
+
+dda_status_t ensure_workspace(dda_matrix* K, size_t bytes, cudaStream_t st) {
+    if (K->ws_bytes >= bytes) return DDA_OK;
+    if (K->ws) {
+        cudaStreamSynchronize(st);
+        dev_free(K->ws);
+    }
+    K->ws = nullptr;
+    K->ws_bytes = 0;
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->ws), bytes, st));
+    K->ws_bytes = bytes;
+    return DDA_OK;
+}
+
+}  // namespace dda
+
+extern "C" int64_t dda_launch_count(void) { return dda::g_launches.load(); }
+
+extern "C" const char* dda_last_cuda_error(void) { return dda::g_last_err; }
+
+extern "C" const char* dda_status_string(dda_status_t s) {
+    switch (s) {
+        case DDA_OK: return "DDA_OK";
+        case DDA_ERR_ARG: return "DDA_ERR_ARG";
+        case DDA_ERR_CUDA: return "DDA_ERR_CUDA";
+        case DDA_ERR_OOM: return "DDA_ERR_OOM";
+        case DDA_ERR_NOT_SPD: return "DDA_ERR_NOT_SPD";
+        case DDA_ERR_BREAKDOWN: return "DDA_ERR_BREAKDOWN";
+        case DDA_ERR_NO_CONVERGENCE: return "DDA_ERR_NO_CONVERGENCE";
+        case DDA_ERR_NCCL: return "DDA_ERR_NCCL";
+    }
+    return "DDA_ERR_UNKNOWN";
+}

@@ -1,0 +1,115 @@
+// Internal definitions of the B200 DDA solver library (not part of the ABI).
+//
+// Device layout:
+//  * every 6x6 block (diagonal D_i and upper V_ij) is 36 doubles = 288 B, stored
+//    "2x2-tiled": chunk q = 3R + C (R, C in 0..2) holds the 2x2 sub-block
+//    rows 2R..2R+1, cols 2C..2C+1 as [a(2R,2C), a(2R,2C+1), a(2R+1,2C), a(2R+1,2C+1)];
+//    one chunk is 32 B = one 256-bit load, so a block is 9 lanes x 32 B;
+//  * blocks are 32 B aligned (cudaMalloc base + 288 B stride);
+//  * block-Jacobi inverses are packed upper triangles, 21 doubles padded to 24;
+//  * index arrays are int32 (row_ptr / low_ptr [n+1], col_idx / low_row / low_to_up [nnzb]).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <cstdint>
+#include <cstddef>
+
+#include "dda.h"
+
+#ifndef DDA_THREADS
+#define DDA_THREADS 256
+#endif
+
+namespace dda {
+
+constexpr int kBlk = 36;       // doubles per 6x6 block
+constexpr int kDinv = 24;      // doubles per packed inverse (21 used)
+
+// offset of element (r, c) in the 2x2-tiled block layout
+__host__ __device__ __forceinline__ int tile_off(int r, int c) {
+    return 4 * (3 * (r >> 1) + (c >> 1)) + 2 * (r & 1) + (c & 1);
+}
+// offset of (r, c), r <= c, in the packed upper triangle (row-major)
+__host__ __device__ __forceinline__ int pk_off(int r, int c) {
+    return r * 6 - (r * (r - 1)) / 2 + (c - r);
+}
+
+// ------------------------------------------------------------------ host-side bookkeeping
+void note_launch(int k = 1);               // counts kernel launches (dda_launch_count)
+dda_status_t cuda_fail(cudaError_t e);      // records the message, maps to a status
+int device_sms();
+// stream-ordered allocations from the device's default memory pool, which is
+// configured once to keep freed memory cached (repeated builds in the
+// open-close loop do not pay cudaMalloc/cudaFree)
+cudaError_t dev_alloc(void** p, size_t bytes, cudaStream_t st);
+void dev_free(void* p);
+
+#define DDA_CK(call)                                   \
+    do {                                               \
+        cudaError_t _e = (call);                       \
+        if (_e != cudaSuccess) return dda::cuda_fail(_e); \
+    } while (0)
+
+#define DDA_LAUNCHED()                                 \
+    do {                                               \
+        dda::note_launch();                            \
+        cudaError_t _e = cudaGetLastError();           \
+        if (_e != cudaSuccess) return dda::cuda_fail(_e); \
+    } while (0)
+
+// ------------------------------------------------------------------ device-side load helpers
+
+// 256-bit read-only load of one 2x2 chunk (ld.global.nc.v4.f64 -> LDG.E.ENL2.256)
+__device__ __forceinline__ double4 ld_chunk(const double* p) {
+    double4 v;
+    asm volatile("ld.global.nc.L1::no_allocate.v4.f64 {%0,%1,%2,%3}, [%4];"
+                 : "=d"(v.x), "=d"(v.y), "=d"(v.z), "=d"(v.w) : "l"(p));
+    return v;
+}
+// coherent (L2) loads for vectors written earlier in the same persistent kernel
+__device__ __forceinline__ double2 ld_cg2(const double* p) { return __ldcg(reinterpret_cast<const double2*>(p)); }
+__device__ __forceinline__ double ld_cg(const double* p) { return __ldcg(p); }
+
+__device__ __forceinline__ double warp_sum(double v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+}  // namespace dda
+
+// ------------------------------------------------------------------ the opaque handle
+struct dda_matrix {
+    int device = 0;
+    int32_t n = 0;
+    int64_t nnzb = 0;
+    int64_t m = 0;
+    // structure (device)
+    int32_t* row_ptr = nullptr;
+    int32_t* col_idx = nullptr;
+    int32_t* low_ptr = nullptr;
+    int32_t* low_row = nullptr;
+    int32_t* low_to_up = nullptr;
+    int32_t* urow = nullptr;        // [nnzb] block row of each upper block
+    double* diag = nullptr;         // [n][36] tiled
+    double* upper = nullptr;        // [nnzb][36] tiled
+    // cached assembly permutation for value-only re-assembly (NEXT-1)
+    int32_t* perm = nullptr;        // [m] spring ids sorted stably by (min,max)
+    int32_t* seg = nullptr;         // [nnzb+1] segment starts into perm
+    int32_t* dperm = nullptr;       // [2m] endpoint records 2s+side sorted stably by block
+    int32_t* dstart = nullptr;      // [n+1]
+    uint8_t* orient = nullptr;      // [m] 1 if bi[s] < bj[s]
+    // preconditioners
+    double* dinv = nullptr;         // [n][24] packed D_i^{-1}
+    bool dinv_valid = false;
+    // PCG workspace
+    double* ws = nullptr;
+    size_t ws_bytes = 0;
+    void* scratch = nullptr;        // small device scratch (result struct, flags)
+};
+
+namespace dda {
+dda_status_t ensure_workspace(dda_matrix* K, size_t bytes, cudaStream_t st);
+dda_status_t bj_setup(dda_matrix* K, cudaStream_t s, int32_t* bad_block);
+dda_status_t spmv(dda_matrix* K, const double* x, double* y, cudaStream_t s);
+}  // namespace dda

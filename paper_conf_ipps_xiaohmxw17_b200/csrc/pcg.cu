@@ -1,0 +1,429 @@
+// A5/A6 — the PCG solve of K d = F as ONE persistent cooperative kernel
+// (§IV.A; textbook PCG, Saad Alg. 9.1, reading Z1/Z2/Z19).
+//
+// Per iteration (block-Jacobi):
+//   phase A  q = K p (warp per block row, spmv_row) + CTA partial of p^T q
+//   -- grid barrier --  sigma = fixed-order sum of the partials (every CTA)
+//   phase B  alpha = rho/sigma; d += alpha p; r -= alpha q; z = D^{-1} r;
+//            partials of r^T r and r^T z
+//   -- grid barrier --  convergence test ||r|| <= tol ||F||, beta = rho'/rho
+//   phase C  p = z + beta p
+//   -- grid barrier --
+// SSOR-AI inserts its two half-passes (lower on t = D^{-1} r, upper on w)
+// between B and C, with a barrier after each.  Every CTA evaluates the scalars
+// itself from the same partials in the same order, so all CTAs take the same
+// branch and the result is bitwise reproducible for a given launch
+// configuration.  The host reads the outcome once, after the kernel.
+#include <cooperative_groups.h>
+
+#include <cmath>
+
+#include "precond_dev.cuh"
+
+namespace cg = cooperative_groups;
+
+namespace dda {
+namespace {
+
+constexpr int WPB = DDA_THREADS / 32;
+
+struct PcgOut {
+    int iters;
+    int status;
+    double rel_res;
+    double rr;
+    double FF;
+};
+
+struct PcgArgs {
+    BsrView A;
+    const double* __restrict__ dinv;
+    const double* __restrict__ F;
+    const double* d0;      // may be null; may alias d
+    double* d;
+    double* r;
+    double* z;
+    double* p;
+    double* q;
+    double* t;
+    double* w;
+    double* part;          // [4][G] CTA partials
+    PcgOut* out;
+    int pc;
+    double omega;
+    double tol;
+    int maxit;
+};
+
+// deterministic CTA reduction of NV values -> part[k*G + blockIdx.x]
+template <int NV>
+__device__ __forceinline__ void cta_partials(double (&v)[NV], double* part, int G, double (*red)[4]) {
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+#pragma unroll
+    for (int k = 0; k < NV; ++k) v[k] = warp_sum(v[k]);
+    if (lane == 0) {
+#pragma unroll
+        for (int k = 0; k < NV; ++k) red[wib][k] = v[k];
+    }
+    __syncthreads();
+    if (threadIdx.x < NV) {
+        double s = 0.0;
+        for (int w = 0; w < WPB; ++w) s += red[w][threadIdx.x];
+        part[threadIdx.x * G + blockIdx.x] = s;
+    }
+    __syncthreads();
+}
+
+// fixed-order sum of part[k*G .. k*G+G) for k < NV, identical in every CTA
+template <int NV>
+__device__ __forceinline__ void grid_sums(const double* part, int G, double (&out)[NV], double* bc) {
+    const int lane = threadIdx.x & 31;
+    if ((threadIdx.x >> 5) == 0) {
+#pragma unroll
+        for (int k = 0; k < NV; ++k) {
+            double s = 0.0;
+            for (int j = lane; j < G; j += 32) s += ld_cg(part + k * G + j);
+            s = warp_sum(s);
+            if (lane == 0) bc[k] = s;
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < NV; ++k) out[k] = bc[k];
+    __syncthreads();
+}
+
+__global__ void __launch_bounds__(DDA_THREADS) k_pcg(PcgArgs P) {
+    cg::grid_group grid = cg::this_grid();
+    __shared__ double red[WPB][4];
+    __shared__ double bc[4];
+    const int lane = threadIdx.x & 31;
+    const int G = gridDim.x;
+    const int gw = blockIdx.x * WPB + (threadIdx.x >> 5);
+    const int W = G * WPB;
+    const int n = P.A.n;
+    const int ngrp = (n + 4) / 5;
+    const bool use_dinv = (P.pc == DDA_PC_BJ || P.pc == DDA_PC_SSOR_AI);
+
+    // z = M^{-1} r for SSOR-AI given t = D^{-1} r already stored: two half passes.
+    // Writes z (and p = z when init); returns the CTA-local r^T z contribution.
+    auto ssor_passes = [&](bool init) -> double {
+        for (int i = gw; i < n; i += W) ssor_lower_row(P.A, P.dinv, i, P.r, P.t, P.omega, P.w, lane);
+        grid.sync();
+        double rz = 0.0;
+        for (int i = gw; i < n; i += W) {
+            const double zz = ssor_upper_row(P.A, P.dinv, i, P.w, P.omega, lane);
+            if (lane < 6) {
+                const size_t idx = 6 * (size_t)i + lane;
+                P.z[idx] = zz;
+                if (init) P.p[idx] = zz;
+                rz += ld_cg(P.r + idx) * zz;
+            }
+        }
+        return rz;
+    };
+
+    // ------------------------------------------------------------ setup: r = F - K d0
+    if (P.d0) {
+        for (int i = gw; i < n; i += W) {
+            double y0, y1;
+            spmv_row<SPMV_FULL>(P.A, i, XCg{P.d0}, lane, y0, y1);
+            if (lane < 9 && lane % 3 == 0)
+                *reinterpret_cast<double2*>(P.q + 6 * (size_t)i + 2 * (lane / 3)) = make_double2(y0, y1);
+        }
+        grid.sync();
+    }
+    {
+        double v[3] = {0.0, 0.0, 0.0};   // FF, rr, rz
+        for (int grp = gw; grp < ngrp; grp += W) {
+            const Row5 R = row5(grp, lane, n);
+            double rv = 0.0, fv = 0.0;
+            if (R.valid) {
+                fv = P.F[R.idx];
+                const double dv = P.d0 ? ld_cg(P.d0 + R.idx) : 0.0;
+                if (P.d != P.d0) P.d[R.idx] = dv;
+                rv = P.d0 ? fv - ld_cg(P.q + R.idx) : fv;
+                P.r[R.idx] = rv;
+            }
+            v[0] += fv * fv;
+            v[1] += rv * rv;
+            const double tz = use_dinv ? bj_lane(P.dinv, R, rv) : rv;
+            if (R.valid) {
+                if (P.pc == DDA_PC_SSOR_AI) {
+                    P.t[R.idx] = tz;
+                } else {
+                    P.z[R.idx] = tz;
+                    P.p[R.idx] = tz;
+                    v[2] += rv * tz;
+                }
+            }
+        }
+        cta_partials<3>(v, P.part, G, red);
+    }
+    grid.sync();
+    double FF, rr, rho;
+    {
+        double s[3];
+        grid_sums<3>(P.part, G, s, bc);
+        FF = s[0]; rr = s[1]; rho = s[2];
+    }
+    const double bnorm = sqrt(FF);
+    int status = DDA_ERR_NO_CONVERGENCE;
+    int iters = 0;
+    bool skip_final = false;
+    if (FF == 0.0) {                                    // reading Z2: d = 0, iters = 0, rel_res = 0
+        for (int grp = gw; grp < ngrp; grp += W) {
+            const Row5 R = row5(grp, lane, n);
+            if (R.valid) P.d[R.idx] = 0.0;
+        }
+        status = DDA_OK;
+        skip_final = true;
+    } else if (sqrt(rr) <= P.tol * bnorm) {
+        status = DDA_OK;
+    } else {
+        if (P.pc == DDA_PC_SSOR_AI) {
+            grid.sync();                                // t visible
+            double v[1] = {ssor_passes(true)};
+            cta_partials<1>(v, P.part + 2 * G, G, red);
+            grid.sync();
+            double s[1];
+            grid_sums<1>(P.part + 2 * G, G, s, bc);
+            rho = s[0];
+        }
+        if (!(rho > 0.0) || !isfinite(rho)) {
+            status = DDA_ERR_BREAKDOWN;
+        } else {
+            for (int k = 0; k < P.maxit; ++k) {
+                // ---- phase A: q = K p, partial p^T q
+                {
+                    double v[1] = {0.0};
+                    for (int i = gw; i < n; i += W) {
+                        double y0, y1;
+                        spmv_row<SPMV_FULL>(P.A, i, XCg{P.p}, lane, y0, y1);
+                        if (lane < 9 && lane % 3 == 0) {
+                            const size_t o = 6 * (size_t)i + 2 * (lane / 3);
+                            *reinterpret_cast<double2*>(P.q + o) = make_double2(y0, y1);
+                            const double2 pv = ld_cg2(P.p + o);
+                            v[0] += pv.x * y0 + pv.y * y1;
+                        }
+                    }
+                    cta_partials<1>(v, P.part, G, red);
+                }
+                grid.sync();
+                double sigma;
+                {
+                    double s[1];
+                    grid_sums<1>(P.part, G, s, bc);
+                    sigma = s[0];
+                }
+                if (!(sigma > 0.0) || !isfinite(sigma)) { status = DDA_ERR_BREAKDOWN; break; }
+                const double alpha = rho / sigma;
+                // ---- phase B: d += alpha p; r -= alpha q; z = M^{-1} r (BJ / none) or t = D^{-1} r
+                {
+                    double v[2] = {0.0, 0.0};   // rr, rz
+                    for (int grp = gw; grp < ngrp; grp += W) {
+                        const Row5 R = row5(grp, lane, n);
+                        double rv = 0.0;
+                        if (R.valid) {
+                            const double pv = ld_cg(P.p + R.idx);
+                            P.d[R.idx] = ld_cg(P.d + R.idx) + alpha * pv;
+                            rv = ld_cg(P.r + R.idx) - alpha * ld_cg(P.q + R.idx);
+                            P.r[R.idx] = rv;
+                        }
+                        v[0] += rv * rv;
+                        const double tz = use_dinv ? bj_lane(P.dinv, R, rv) : rv;
+                        if (R.valid) {
+                            if (P.pc == DDA_PC_SSOR_AI) {
+                                P.t[R.idx] = tz;
+                            } else {
+                                P.z[R.idx] = tz;
+                                v[1] += rv * tz;
+                            }
+                        }
+                    }
+                    cta_partials<2>(v, P.part + G, G, red);
+                }
+                grid.sync();
+                double rz;
+                {
+                    double s[2];
+                    grid_sums<2>(P.part + G, G, s, bc);
+                    rr = s[0]; rz = s[1];
+                }
+                iters = k + 1;
+                if (sqrt(rr) <= P.tol * bnorm) { status = DDA_OK; break; }
+                if (P.pc == DDA_PC_SSOR_AI) {
+                    double v[1] = {ssor_passes(false)};
+                    cta_partials<1>(v, P.part + 2 * G, G, red);
+                    grid.sync();
+                    double s[1];
+                    grid_sums<1>(P.part + 2 * G, G, s, bc);
+                    rz = s[0];
+                }
+                if (!(rz > 0.0) || !isfinite(rz)) { status = DDA_ERR_BREAKDOWN; break; }
+                const double beta = rz / rho;
+                rho = rz;
+                // ---- phase C: p = z + beta p
+                for (int grp = gw; grp < ngrp; grp += W) {
+                    const Row5 R = row5(grp, lane, n);
+                    if (R.valid) P.p[R.idx] = ld_cg(P.z + R.idx) + beta * ld_cg(P.p + R.idx);
+                }
+                grid.sync();
+            }
+        }
+    }
+
+    // ------------------------------------------------------------ true residual ||F - K d|| / ||F||
+    double rel = 0.0;
+    if (!skip_final) {
+        grid.sync();
+        for (int i = gw; i < n; i += W) {
+            double y0, y1;
+            spmv_row<SPMV_FULL>(P.A, i, XCg{P.d}, lane, y0, y1);
+            if (lane < 9 && lane % 3 == 0)
+                *reinterpret_cast<double2*>(P.q + 6 * (size_t)i + 2 * (lane / 3)) = make_double2(y0, y1);
+        }
+        grid.sync();
+        double v[1] = {0.0};
+        for (int grp = gw; grp < ngrp; grp += W) {
+            const Row5 R = row5(grp, lane, n);
+            if (R.valid) {
+                const double e = P.F[R.idx] - ld_cg(P.q + R.idx);
+                v[0] += e * e;
+            }
+        }
+        cta_partials<1>(v, P.part + 3 * G, G, red);
+        grid.sync();
+        double s[1];
+        grid_sums<1>(P.part + 3 * G, G, s, bc);
+        rel = sqrt(s[0]) / bnorm;
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        P.out->iters = iters;
+        P.out->status = status;
+        P.out->rel_res = rel;
+        P.out->rr = rr;
+        P.out->FF = FF;
+    }
+}
+
+int pcg_grid() {
+    static int cached_dev = -1, cached = 0;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev != cached_dev) {
+        int per_sm = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_pcg, DDA_THREADS, 0);
+        cached = device_sms() * (per_sm > 0 ? per_sm : 1);
+        cached_dev = dev;
+    }
+    return cached;
+}
+
+}  // namespace
+
+dda_status_t pcg_solve(dda_matrix* K, const double* F, const double* d0, double* d, double tol, int32_t maxit,
+                       dda_precond_t pc, double omega, int32_t* iters, double* rel_res, cudaStream_t st) {
+    if (iters) *iters = 0;
+    if (rel_res) *rel_res = 0.0;
+    if (!K || !F || !d || !(tol > 0.0) || maxit < 0) return DDA_ERR_ARG;
+    if (pc != DDA_PC_NONE && pc != DDA_PC_BJ && pc != DDA_PC_SSOR_AI) return DDA_ERR_ARG;
+    if ((pc == DDA_PC_BJ || pc == DDA_PC_SSOR_AI) && !K->dinv_valid) {
+        dda_status_t s = bj_setup(K, st, nullptr);
+        if (s != DDA_OK) return s;
+    }
+    const size_t N = 6 * (size_t)K->n;
+    int G = pcg_grid();
+    const int need = (K->n + WPB - 1) / WPB;
+    if (need < G) G = need > 0 ? need : 1;
+    const size_t bytes = (6 * N + 4 * (size_t)G) * sizeof(double);
+    {
+        dda_status_t s = ensure_workspace(K, bytes, st);
+        if (s != DDA_OK) return s;
+    }
+    PcgArgs a;
+    a.A = view_of(K);
+    a.dinv = K->dinv;
+    a.F = F;
+    a.d0 = d0;
+    a.d = d;
+    a.r = K->ws;
+    a.z = K->ws + N;
+    a.p = K->ws + 2 * N;
+    a.q = K->ws + 3 * N;
+    a.t = K->ws + 4 * N;
+    a.w = K->ws + 5 * N;
+    a.part = K->ws + 6 * N;
+    a.out = reinterpret_cast<PcgOut*>(reinterpret_cast<char*>(K->scratch) + 64);
+    a.pc = (int)pc;
+    a.omega = omega;
+    a.tol = tol;
+    a.maxit = maxit;
+    void* args[] = {&a};
+    DDA_CK(cudaLaunchCooperativeKernel((const void*)k_pcg, dim3(G), dim3(DDA_THREADS), args, 0, st));
+    note_launch();
+    PcgOut h;
+    DDA_CK(cudaMemcpyAsync(&h, a.out, sizeof h, cudaMemcpyDeviceToHost, st));
+    DDA_CK(cudaStreamSynchronize(st));
+    if (iters) *iters = h.iters;
+    if (rel_res) *rel_res = h.rel_res;
+    return (dda_status_t)h.status;
+}
+
+}  // namespace dda
+
+using namespace dda;
+
+extern "C" dda_status_t dda_pcg_solve(dda_matrix_t K, const double* F, const double* d0, double* d, double tol,
+                                      int32_t maxit, dda_precond_t pc, double omega, int32_t* iters,
+                                      double* rel_res, void* stream) {
+    return pcg_solve(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, reinterpret_cast<cudaStream_t>(stream));
+}
+
+extern "C" dda_status_t dda_solve_host(int32_t n, const double* kdiag, int64_t m, const int32_t* bi,
+                                       const int32_t* bj, const double* pen, const double* e, const double* g,
+                                       const double* F, const double* d0, double* d, double tol, int32_t maxit,
+                                       dda_precond_t pc, double omega, int32_t* iters, double* rel_res,
+                                       void* stream) {
+    if (n <= 0 || m < 0 || !kdiag || !F || !d) return DDA_ERR_ARG;
+    if (m > 0 && (!bi || !bj || !pen || !e || !g)) return DDA_ERR_ARG;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    const size_t N = 6 * (size_t)n;
+    const size_t bytes = sizeof(double) * ((size_t)36 * n + 3 * N + (size_t)13 * m) + sizeof(int32_t) * 2 * (size_t)m;
+    char* buf = nullptr;
+    DDA_CK(cudaMallocAsync(reinterpret_cast<void**>(&buf), bytes, st));
+    struct Free {
+        char* b; cudaStream_t s;
+        ~Free() { cudaFreeAsync(b, s); cudaStreamSynchronize(s); }
+    } fr{buf, st};
+    double* dk = reinterpret_cast<double*>(buf);
+    double* dF = dk + (size_t)36 * n;
+    double* dd0 = dF + N;
+    double* dd = dd0 + N;
+    double* dpen = dd + N;
+    double* de = dpen + m;
+    double* dg = de + 6 * (size_t)m;
+    int32_t* dbi = reinterpret_cast<int32_t*>(dg + 6 * (size_t)m);
+    int32_t* dbj = dbi + m;
+    DDA_CK(cudaMemcpyAsync(dk, kdiag, sizeof(double) * 36 * (size_t)n, cudaMemcpyHostToDevice, st));
+    DDA_CK(cudaMemcpyAsync(dF, F, sizeof(double) * N, cudaMemcpyHostToDevice, st));
+    if (d0) DDA_CK(cudaMemcpyAsync(dd0, d0, sizeof(double) * N, cudaMemcpyHostToDevice, st));
+    if (m > 0) {
+        DDA_CK(cudaMemcpyAsync(dpen, pen, sizeof(double) * m, cudaMemcpyHostToDevice, st));
+        DDA_CK(cudaMemcpyAsync(de, e, sizeof(double) * 6 * m, cudaMemcpyHostToDevice, st));
+        DDA_CK(cudaMemcpyAsync(dg, g, sizeof(double) * 6 * m, cudaMemcpyHostToDevice, st));
+        DDA_CK(cudaMemcpyAsync(dbi, bi, sizeof(int32_t) * m, cudaMemcpyHostToDevice, st));
+        DDA_CK(cudaMemcpyAsync(dbj, bj, sizeof(int32_t) * m, cudaMemcpyHostToDevice, st));
+    }
+    dda_matrix_t K = nullptr;
+    dda_status_t s = dda_build_matrix(n, dk, m, dbi, dbj, dpen, de, dg, stream, &K);
+    if (s != DDA_OK) return s;
+    s = pcg_solve(K, dF, d0 ? dd0 : nullptr, dd, tol, maxit, pc, omega, iters, rel_res, st);
+    if (s == DDA_OK || s == DDA_ERR_NO_CONVERGENCE || s == DDA_ERR_BREAKDOWN) {
+        cudaError_t ce = cudaMemcpyAsync(d, dd, sizeof(double) * N, cudaMemcpyDeviceToHost, st);
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(st);
+        if (ce != cudaSuccess) s = cuda_fail(ce);
+    }
+    dda_matrix_free(K);
+    return s;
+}

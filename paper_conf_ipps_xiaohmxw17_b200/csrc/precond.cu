@@ -1,0 +1,192 @@
+// A3 — block-Jacobi construction (Table I "construction time" P:174) and
+// standalone preconditioner application (A3/A7) for testing.
+//
+// BJ construction: per diagonal block, Cholesky D = L L^T (6 square roots),
+// L^{-1} by forward substitution, D^{-1} = L^{-T} L^{-1}, stored as the packed
+// upper triangle (21 doubles padded to 24 = 192 B).  One thread per block with
+// everything in registers; ~250 flops against 288 B read + 192 B written, so
+// the kernel is HBM-bound.  A non-positive or non-finite
+// pivot reports DDA_ERR_NOT_SPD with the smallest offending block index.
+#include <climits>
+
+#include "precond_dev.cuh"
+
+namespace dda {
+namespace {
+
+__global__ void __launch_bounds__(128) k_bj_inv(int32_t n, const double* __restrict__ diag, double* __restrict__ dinv,
+                                                double* __restrict__ full, int* __restrict__ bad) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const double* D = diag + (size_t)kBlk * i;
+        double A[6][6];
+#pragma unroll
+        for (int q = 0; q < 9; ++q) {
+            const double4 v = ld_chunk(D + 4 * q);
+            const int R = q / 3, C = q % 3;
+            A[2 * R][2 * C] = v.x; A[2 * R][2 * C + 1] = v.y;
+            A[2 * R + 1][2 * C] = v.z; A[2 * R + 1][2 * C + 1] = v.w;
+        }
+        double L[6][6];
+        bool ok = true;
+#pragma unroll
+        for (int j = 0; j < 6; ++j) {
+            double d = A[j][j];
+#pragma unroll
+            for (int k = 0; k < j; ++k) d -= L[j][k] * L[j][k];
+            ok = ok && (d > 0.0) && isfinite(d);
+            const double ljj = sqrt(d > 0.0 ? d : 1.0);
+            L[j][j] = ljj;
+            const double inv = 1.0 / ljj;
+#pragma unroll
+            for (int r = j + 1; r < 6; ++r) {
+                double s = A[r][j];
+#pragma unroll
+                for (int k = 0; k < j; ++k) s -= L[r][k] * L[j][k];
+                L[r][j] = s * inv;
+            }
+        }
+        if (!ok) atomicMin(bad, (int)i);
+        // Li = L^{-1} (lower triangular)
+        double Li[6][6];
+#pragma unroll
+        for (int c = 0; c < 6; ++c) {
+#pragma unroll
+            for (int r = 0; r < 6; ++r) {
+                if (r < c) { Li[r][c] = 0.0; continue; }
+                double s = (r == c) ? 1.0 : 0.0;
+#pragma unroll
+                for (int k = c; k < r; ++k) s -= L[r][k] * Li[k][c];
+                Li[r][c] = s / L[r][r];
+            }
+        }
+        double* out = dinv + (size_t)kDinv * i;
+        double P[24];
+#pragma unroll
+        for (int r = 0; r < 6; ++r)
+#pragma unroll
+            for (int c = r; c < 6; ++c) {
+                double s = 0.0;
+#pragma unroll
+                for (int k = c; k < 6; ++k) s += Li[k][r] * Li[k][c];
+                P[pk_off(r, c)] = s;
+            }
+        P[21] = P[22] = P[23] = 0.0;
+#pragma unroll
+        for (int q = 0; q < 12; ++q) reinterpret_cast<double2*>(out)[q] = make_double2(P[2 * q], P[2 * q + 1]);
+        if (full) {
+#pragma unroll
+            for (int r = 0; r < 6; ++r)
+#pragma unroll
+                for (int c = 0; c < 6; ++c) full[36 * i + 6 * r + c] = P[r <= c ? pk_off(r, c) : pk_off(c, r)];
+        }
+    }
+}
+
+__global__ void __launch_bounds__(DDA_THREADS) k_bj_apply(int32_t n, const double* __restrict__ dinv,
+                                                          const double* __restrict__ r, double* __restrict__ z) {
+    const int lane = threadIdx.x & 31;
+    const int W = gridDim.x * (DDA_THREADS / 32);
+    const int ngrp = (n + 4) / 5;
+    for (int grp = blockIdx.x * (DDA_THREADS / 32) + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        const double v = R.valid ? r[R.idx] : 0.0;
+        const double zz = bj_lane(dinv, R, v);
+        if (R.valid) z[R.idx] = zz;
+    }
+}
+
+__global__ void __launch_bounds__(DDA_THREADS) k_ssor_lower(BsrView A, const double* __restrict__ dinv, double omega,
+                                                            const double* r, const double* t, double* w) {
+    const int lane = threadIdx.x & 31;
+    const int W = gridDim.x * (DDA_THREADS / 32);
+    for (int i = blockIdx.x * (DDA_THREADS / 32) + (threadIdx.x >> 5); i < A.n; i += W)
+        ssor_lower_row(A, dinv, i, r, t, omega, w, lane);
+}
+
+__global__ void __launch_bounds__(DDA_THREADS) k_ssor_upper(BsrView A, const double* __restrict__ dinv, double omega,
+                                                            const double* w, double* z) {
+    const int lane = threadIdx.x & 31;
+    const int W = gridDim.x * (DDA_THREADS / 32);
+    for (int i = blockIdx.x * (DDA_THREADS / 32) + (threadIdx.x >> 5); i < A.n; i += W) {
+        const double zz = ssor_upper_row(A, dinv, i, w, omega, lane);
+        if (lane < 6) z[6 * (size_t)i + lane] = zz;
+    }
+}
+
+int grid_rows(int rows_per_warp, int n) {
+    const int warps = (n + rows_per_warp - 1) / rows_per_warp;
+    int g = (warps + DDA_THREADS / 32 - 1) / (DDA_THREADS / 32);
+    const int cap = device_sms() * 8;
+    return g < 1 ? 1 : (g > cap ? cap : g);
+}
+
+}  // namespace
+
+dda_status_t bj_setup(dda_matrix* K, cudaStream_t st, int32_t* bad_block, double* full) {
+    if (bad_block) *bad_block = -1;
+    int* bad = reinterpret_cast<int*>(K->scratch);
+    const int big = INT_MAX;
+    DDA_CK(cudaMemcpyAsync(bad, &big, sizeof(int), cudaMemcpyHostToDevice, st));
+    int g = (K->n + 127) / 128;
+    const int cap = device_sms() * 16;
+    if (g > cap) g = cap;
+    k_bj_inv<<<g, 128, 0, st>>>(K->n, K->diag, K->dinv, full, bad);
+    DDA_LAUNCHED();
+    int hbad = 0;
+    DDA_CK(cudaMemcpyAsync(&hbad, bad, sizeof(int), cudaMemcpyDeviceToHost, st));
+    DDA_CK(cudaStreamSynchronize(st));
+    if (hbad != INT_MAX) {
+        if (bad_block) *bad_block = hbad;
+        K->dinv_valid = false;
+        return DDA_ERR_NOT_SPD;
+    }
+    K->dinv_valid = true;
+    return DDA_OK;
+}
+
+dda_status_t bj_setup(dda_matrix* K, cudaStream_t st, int32_t* bad_block) { return bj_setup(K, st, bad_block, nullptr); }
+
+}  // namespace dda
+
+using namespace dda;
+
+extern "C" dda_status_t dda_bj_setup(dda_matrix_t K, double* dinv_full, int32_t* bad_block, void* stream) {
+    if (!K) return DDA_ERR_ARG;
+    return bj_setup(K, reinterpret_cast<cudaStream_t>(stream), bad_block, dinv_full);
+}
+
+extern "C" dda_status_t dda_precond_apply(dda_matrix_t K, dda_precond_t pc, double omega, const double* r, double* z,
+                                          void* stream) {
+    if (!K || !r || !z || r == z) return DDA_ERR_ARG;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    const size_t N = 6 * (size_t)K->n;
+    if (pc == DDA_PC_NONE) {
+        DDA_CK(cudaMemcpyAsync(z, r, N * sizeof(double), cudaMemcpyDeviceToDevice, st));
+        DDA_CK(cudaStreamSynchronize(st));
+        return DDA_OK;
+    }
+    if (pc != DDA_PC_BJ && pc != DDA_PC_SSOR_AI) return DDA_ERR_ARG;
+    if (!K->dinv_valid) {
+        dda_status_t s = bj_setup(K, st, nullptr);
+        if (s != DDA_OK) return s;
+    }
+    if (pc == DDA_PC_BJ) {
+        k_bj_apply<<<grid_rows(5, K->n), DDA_THREADS, 0, st>>>(K->n, K->dinv, r, z);
+        DDA_LAUNCHED();
+    } else {
+        {
+            dda_status_t ws = ensure_workspace(K, 2 * N * sizeof(double), st);
+            if (ws != DDA_OK) return ws;
+        }
+        double* t = K->ws;
+        double* w = K->ws + N;
+        k_bj_apply<<<grid_rows(5, K->n), DDA_THREADS, 0, st>>>(K->n, K->dinv, r, t);
+        DDA_LAUNCHED();
+        k_ssor_lower<<<grid_rows(1, K->n), DDA_THREADS, 0, st>>>(view_of(K), K->dinv, omega, r, t, w);
+        DDA_LAUNCHED();
+        k_ssor_upper<<<grid_rows(1, K->n), DDA_THREADS, 0, st>>>(view_of(K), K->dinv, omega, w, z);
+        DDA_LAUNCHED();
+    }
+    DDA_CK(cudaStreamSynchronize(st));
+    return DDA_OK;
+}

@@ -1,0 +1,293 @@
+"""GPU parity: the CUDA path through the C ABI vs the oracle.
+
+Bars (BASELINE.json north_star, readings Z8/Z16/Z17):
+* structure and index arrays: bit-exact;
+* assembled values: bit-exact (both sides round (p*e[r])*g[c] as written);
+* SpMV: componentwise |dy_i| <= 1e-12 (|K||x|)_i; unit-vector columns exact;
+* PCG: true relative residual <= 1e-10; iterations within max(2, 1%) of the
+  oracle; at matched iteration count the solution differs by <= 1e-9 relative.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import oracle
+from synth import make_slope, preset, random_vector, warm_start
+
+pytestmark = pytest.mark.gpu
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden", "two_block.json")
+
+
+@pytest.fixture(scope="module")
+def dda():
+    if not torch.cuda.is_available():
+        pytest.fail("GPU tests need a CUDA device (no CPU fallback exists)")
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_ipps_xiaohmxw17_b200 as m
+    return m
+
+
+CASES = {
+    "tiny": lambda: make_slope(preset("tiny")),
+    "tiny_shuffled": lambda: make_slope(preset("tiny", shuffle=True)),
+    "chain": lambda: make_slope(preset("tiny", courses=1, base_bricks=40)),
+    "ragged_1k": lambda: make_slope(preset(1000, seed=1041)),
+    "paper": lambda: make_slope(preset("paper")),
+}
+_cache = {}
+
+
+def case(name):
+    if name not in _cache:
+        P = CASES[name]()
+        _cache[name] = (P, oracle.assemble(P))
+    return _cache[name]
+
+
+def _abs_bound(O, n, x):
+    ip, ix, dv = O.full_csr()
+    b = np.zeros(6 * n)
+    np.add.at(b, np.repeat(np.arange(6 * n), np.diff(ip)), np.abs(dv) * np.abs(x[ix]))
+    return b
+
+
+# ------------------------------------------------------------------ A1 / A2 assembly
+
+@pytest.mark.parametrize("name", list(CASES))
+def test_assembly_bit_exact(dda, name):
+    P, O = case(name)
+    K = dda.build_from_problem(P)
+    S = O.export()
+    ex = K.export()
+    assert K.n == O.n and K.nnzb == O.nnzb
+    for k in ("row_ptr", "col_idx", "low_ptr", "low_row", "low_to_up"):
+        assert np.array_equal(ex[k], getattr(S, k)), k
+    assert np.array_equal(ex["diag"], S.diag)
+    assert np.array_equal(ex["upper"], S.upper)
+
+
+def test_golden_two_block(dda):
+    G = json.load(open(GOLDEN))
+    dev = lambda a, dt: torch.tensor(np.array(a), dtype=dt, device="cuda").contiguous()
+    K = dda.build_matrix(dev(G["kdiag"], torch.float64), dev(G["bi"], torch.int32), dev(G["bj"], torch.int32),
+                         dev(G["pen"], torch.float64), dev(G["e"], torch.float64), dev(G["g"], torch.float64))
+    ex, X = K.export(), G["expect"]
+    for k in ("row_ptr", "col_idx", "low_ptr", "low_row", "low_to_up"):
+        assert ex[k].tolist() == X[k], k
+    assert np.array_equal(ex["diag"], np.array(X["diag"], float))
+    assert np.array_equal(ex["upper"], np.array(X["upper"], float))
+    y = K.spmv(dev(X["x"], torch.float64)).cpu().numpy()
+    assert np.array_equal(y, np.array(X["y"], float))
+
+
+def test_no_springs(dda):
+    P = make_slope(preset("tiny"))
+    dev = "cuda"
+    K = dda.build_matrix(torch.from_numpy(P.kdiag).to(dev), torch.zeros(0, dtype=torch.int32, device=dev),
+                         torch.zeros(0, dtype=torch.int32, device=dev), torch.zeros(0, dtype=torch.float64, device=dev),
+                         torch.zeros((0, 6), dtype=torch.float64, device=dev),
+                         torch.zeros((0, 6), dtype=torch.float64, device=dev))
+    assert K.nnzb == 0
+    ex = K.export()
+    U = np.triu(P.kdiag)
+    assert np.array_equal(ex["diag"], U + np.transpose(np.triu(U, 1), (0, 2, 1)))
+    d, it, rr, st = K.pcg_solve(torch.from_numpy(P.F).cuda(), tol=1e-10)
+    assert st == dda.OK and it == 1 and rr <= 1e-10       # block diagonal: BJ is exact
+
+
+@pytest.mark.parametrize("bad", ["self", "range", "neg_pen", "nan_pen"])
+def test_invalid_input(dda, bad):
+    P = make_slope(preset("tiny"))
+    t = dda.problem_to_device(P)
+    if bad == "self":
+        t["bj"][3] = t["bi"][3]
+    elif bad == "range":
+        t["bi"][5] = P.n
+    elif bad == "neg_pen":
+        t["pen"][7] = -1.0
+    else:
+        t["pen"][7] = float("nan")
+    with pytest.raises(dda.DDAError) as ei:
+        dda.build_matrix(t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+    assert ei.value.status == dda.ERR_ARG
+
+
+def test_update_values_matches_fresh_build(dda):
+    P, _ = case("tiny")
+    t = dda.problem_to_device(P)
+    K = dda.build_matrix(t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+    rng = np.random.default_rng(5)
+    pen2 = P.pen * rng.uniform(0.5, 1.5, P.m)
+    pen2[::7] = 0.0                                      # contacts opened in the open-close loop
+    kd2 = P.kdiag * 1.1
+    K.update_values(torch.from_numpy(kd2).cuda(), torch.from_numpy(pen2).cuda(), t["e"], t["g"])
+    O2 = oracle.OracleMatrix(P.n, kd2, P.bi, P.bj, pen2, P.e, P.g)
+    ex, S2 = K.export(), O2.export()
+    assert np.array_equal(ex["diag"], S2.diag) and np.array_equal(ex["upper"], S2.upper)
+
+
+# ------------------------------------------------------------------ A4 SpMV
+
+@pytest.mark.parametrize("name", list(CASES))
+def test_spmv_parity(dda, name):
+    P, O = case(name)
+    K = dda.build_from_problem(P)
+    x = random_vector(P.n, 42)
+    y = K.spmv(torch.from_numpy(x).cuda()).cpu().numpy()
+    yo = O.spmv(x)
+    bound = _abs_bound(O, P.n, x)
+    err = np.abs(y - yo) / bound
+    assert err.max() <= 1e-12, err.max()
+    assert np.linalg.norm(y - yo) / np.linalg.norm(yo) <= 1e-13
+
+
+def test_spmv_unit_vectors_exact(dda):
+    P, O = case("tiny")
+    K = dda.build_from_problem(P)
+    ip, ix, dv = O.full_csr()
+    import scipy.sparse as sp
+    A = sp.csr_matrix((dv, ix, ip), shape=(6 * P.n,) * 2).toarray()
+    for k in [0, 1, 5, 6, 100, 6 * P.n // 2, 6 * P.n - 1]:
+        x = torch.zeros(6 * P.n, dtype=torch.float64, device="cuda")
+        x[k] = 1.0
+        assert np.array_equal(K.spmv(x).cpu().numpy(), A[:, k]), k
+
+
+def test_spmv_deterministic(dda):
+    P, O = case("paper")
+    K = dda.build_from_problem(P)
+    x = torch.from_numpy(random_vector(P.n, 3)).cuda()
+    a = K.spmv(x).cpu().numpy()
+    b = K.spmv(x).cpu().numpy()
+    assert np.array_equal(a, b)
+
+
+# ------------------------------------------------------------------ A3 / A7 preconditioners
+
+def test_bj_inverse(dda):
+    P, O = case("tiny")
+    K = dda.build_from_problem(P)
+    dinv = K.bj_setup(full=True).cpu().numpy()
+    ref = O.bj_inv()
+    D = O.export().diag
+    kappa = np.linalg.cond(D)
+    for i in range(P.n):
+        assert np.linalg.norm(dinv[i] - ref[i]) <= 1e-13 * kappa[i] * np.linalg.norm(ref[i])
+
+
+def test_bj_not_spd(dda):
+    P = make_slope(preset("tiny"))
+    kd = P.kdiag.copy()
+    kd[17] = -1e6 * np.eye(6)
+    t = dda.problem_to_device(P)
+    K = dda.build_matrix(torch.from_numpy(kd).cuda(), t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+    with pytest.raises(dda.DDAError) as ei:
+        K.bj_setup()
+    assert ei.value.status == dda.ERR_NOT_SPD
+    d, it, rr, st = None, 0, 0, None
+    with pytest.raises(dda.DDAError):
+        K.pcg_solve(t["F"])
+
+
+@pytest.mark.parametrize("pc,omega", [("bj", 1.0), ("ssor_ai", 1.0), ("ssor_ai", 0.8)])
+def test_precond_apply(dda, pc, omega):
+    P, O = case("paper")
+    K = dda.build_from_problem(P)
+    r = np.random.default_rng(8).standard_normal(6 * P.n)
+    z = K.precond_apply(torch.from_numpy(r).cuda(), pc, omega).cpu().numpy()
+    if pc == "bj":
+        zo = np.einsum("bij,bj->bi", O.bj_inv(), r.reshape(-1, 6)).ravel()
+    else:
+        zo = O.ssor_ai_apply(r, omega=omega)
+    assert np.linalg.norm(z - zo) <= 1e-12 * np.linalg.norm(zo)
+
+
+# ------------------------------------------------------------------ A5 / A6 PCG
+
+def _pcg_parity(dda, P, O, pc, omega=1.0, d0=None, tol=1e-10):
+    K = dda.build_from_problem(P)
+    F = torch.from_numpy(P.F).cuda()
+    d0t = torch.from_numpy(d0).cuda() if d0 is not None else None
+    d, it, rr, st = K.pcg_solve(F, d0=d0t, tol=tol, precond=pc, omega=omega)
+    assert st == dda.OK and rr <= tol * 1.01, (st, rr)
+    do, ito, rro, sto = O.pcg(P.F, d0=d0, tol=tol, precond=pc, omega=omega)
+    assert sto == oracle.OK and rro <= tol * 1.01
+    assert abs(it - ito) <= max(2, int(0.01 * ito)), (it, ito)
+    # matched-iteration comparison (reading Z17)
+    dm, itm, _, _ = O.pcg(P.F, d0=d0, tol=1e-300, maxit=it, precond=pc, omega=omega)
+    assert itm == it
+    d = d.cpu().numpy()
+    assert np.linalg.norm(d - dm) / np.linalg.norm(dm) <= 1e-9
+    return d, it
+
+
+@pytest.mark.parametrize("name", ["tiny", "tiny_shuffled", "ragged_1k", "paper"])
+def test_pcg_bj(dda, name):
+    P, O = case(name)
+    _pcg_parity(dda, P, O, "bj")
+
+
+@pytest.mark.parametrize("name", ["tiny", "paper"])
+def test_pcg_ssor_ai(dda, name):
+    P, O = case(name)
+    _pcg_parity(dda, P, O, "ssor_ai")
+
+
+def test_pcg_none(dda):
+    P, O = case("tiny")
+    _pcg_parity(dda, P, O, "none")
+
+
+def test_pcg_tiny_vs_dense_ldlt(dda):
+    P, O = case("tiny")
+    d, _ = _pcg_parity(dda, P, O, "bj")
+    ref = O.ldlt_solve(P.F)
+    import scipy.linalg as sla
+    from conftest import dense_from_springs
+    Kd = dense_from_springs(P)
+    ev = np.linalg.eigvalsh(Kd)
+    assert np.linalg.norm(d - ref) / np.linalg.norm(ref) <= (ev.max() / ev.min()) * 1e-10
+
+
+def test_pcg_warm_start_and_edge_cases(dda):
+    P, O = case("paper")
+    K = dda.build_from_problem(P)
+    F = torch.from_numpy(P.F).cuda()
+    d1, it1, rr1, st1 = K.pcg_solve(F)
+    d0 = warm_start(d1.cpu().numpy(), 9)
+    _, it2 = _pcg_parity(dda, P, O, "bj", d0=d0)
+    assert it2 < it1
+    # d0 aliasing d
+    dd = torch.from_numpy(d0).cuda()
+    _, it3, rr3, st3 = K.pcg_solve(F, d0=dd, d=dd)
+    assert st3 == dda.OK and it3 == it2 and rr3 <= 1.01e-10
+    # F = 0 -> d = 0, 0 iterations (reading Z2)
+    z, itz, rrz, stz = K.pcg_solve(torch.zeros_like(F), d0=torch.ones_like(F))
+    assert stz == dda.OK and itz == 0 and rrz == 0.0 and not z.any()
+    # iteration cap (the paper's DDA policy caps at 200)
+    _, it5, rr5, st5 = K.pcg_solve(F, maxit=200)
+    assert st5 == dda.ERR_NO_CONVERGENCE and it5 == 200 and rr5 > 1e-10
+
+
+def test_pcg_deterministic(dda):
+    P, O = case("paper")
+    K = dda.build_from_problem(P)
+    F = torch.from_numpy(P.F).cuda()
+    a = K.pcg_solve(F)[0].cpu().numpy()
+    b = K.pcg_solve(F)[0].cpu().numpy()
+    assert np.array_equal(a, b)
+
+
+def test_solve_host_e2e(dda):
+    P, O = case("paper")
+    d, it, rr, st = dda.solve_host(P.kdiag, P.bi, P.bj, P.pen, P.e, P.g, P.F)
+    K = dda.build_from_problem(P)
+    d2, it2, rr2, st2 = K.pcg_solve(torch.from_numpy(P.F).cuda())
+    assert st == st2 == dda.OK and it == it2
+    assert np.array_equal(d, d2.cpu().numpy())
