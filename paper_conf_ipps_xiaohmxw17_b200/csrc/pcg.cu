@@ -17,6 +17,7 @@
 #include <cooperative_groups.h>
 
 #include <cmath>
+#include <cstdlib>
 
 #include "precond_dev.cuh"
 
@@ -93,71 +94,167 @@ __device__ __forceinline__ void grid_sums(const double* part, int G, double (&ou
     __syncthreads();
 }
 
-__global__ void __launch_bounds__(DDA_THREADS) k_pcg(PcgArgs P) {
+// ---------------------------------------------------------------- phases
+// Each phase is a separate non-inlined function so that the persistent kernel
+// keeps one copy of each row loop and a small register footprint (40 registers:
+// 6 CTAs x 8 warps per SM), instead of the union of all phases' live ranges.
+
+__device__ __forceinline__ int warp_id_global() { return blockIdx.x * WPB + (threadIdx.x >> 5); }
+
+// q = K x (all rows); returns this lane's share of x^T q when `dot`
+__device__ __noinline__ double ph_spmv(const PcgArgs& P, const double* x, bool dot) {
+    const int lane = threadIdx.x & 31;
+    double acc = 0.0;
+    for_rows<SPMV_FULL>(P.A, warp_id_global(), gridDim.x * WPB, XCg{x}, lane,
+                        [&](int i, bool ok, double y0, double y1) {
+                            if (ok && is_out_lane(lane)) {
+                                const size_t o = 6 * (size_t)i + 2 * (q_of(lane) / 3);
+                                *reinterpret_cast<double2*>(P.q + o) = make_double2(y0, y1);
+                                if (dot) {
+                                    const double2 xv = ld_cg2(x + o);
+                                    acc += xv.x * y0 + xv.y * y1;
+                                }
+                            }
+                        });
+    return acc;
+}
+
+// setup: d = d0 (or 0), r = F - q (or F), t/z/p = M^{-1} r pieces; partials (F^T F, r^T r, r^T z)
+__device__ __noinline__ double3 ph_init(const PcgArgs& P) {
+    const int lane = threadIdx.x & 31;
+    const int n = P.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    const bool use_dinv = (P.pc == DDA_PC_BJ || P.pc == DDA_PC_SSOR_AI);
+    double FF = 0.0, rr = 0.0, rz = 0.0;
+    for (int grp = warp_id_global(); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        double rv = 0.0, fv = 0.0;
+        if (R.valid) {
+            fv = P.F[R.idx];
+            const double dv = P.d0 ? ld_cg(P.d0 + R.idx) : 0.0;
+            if (P.d != P.d0) P.d[R.idx] = dv;
+            rv = P.d0 ? fv - ld_cg(P.q + R.idx) : fv;
+            P.r[R.idx] = rv;
+        }
+        FF += fv * fv;
+        rr += rv * rv;
+        const double tz = use_dinv ? bj_lane(P.dinv, R, rv) : rv;
+        if (R.valid) {
+            if (P.pc == DDA_PC_SSOR_AI) {
+                P.t[R.idx] = tz;
+            } else {
+                P.z[R.idx] = tz;
+                P.p[R.idx] = tz;
+                rz += rv * tz;
+            }
+        }
+    }
+    return make_double3(FF, rr, rz);
+}
+
+// phase B: d += alpha p; r -= alpha q; z = D^{-1} r (BJ) / t = D^{-1} r (SSOR) / z = r; partials (r^T r, r^T z)
+__device__ __noinline__ double2 ph_update(const PcgArgs& P, double alpha) {
+    const int lane = threadIdx.x & 31;
+    const int n = P.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    const bool use_dinv = (P.pc == DDA_PC_BJ || P.pc == DDA_PC_SSOR_AI);
+    double rr = 0.0, rz = 0.0;
+    for (int grp = warp_id_global(); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        double rv = 0.0;
+        if (R.valid) {
+            const double pv = ld_cg(P.p + R.idx);
+            P.d[R.idx] = ld_cg(P.d + R.idx) + alpha * pv;
+            rv = ld_cg(P.r + R.idx) - alpha * ld_cg(P.q + R.idx);
+            P.r[R.idx] = rv;
+        }
+        rr += rv * rv;
+        const double tz = use_dinv ? bj_lane(P.dinv, R, rv) : rv;
+        if (R.valid) {
+            if (P.pc == DDA_PC_SSOR_AI) {
+                P.t[R.idx] = tz;
+            } else {
+                P.z[R.idx] = tz;
+                rz += rv * tz;
+            }
+        }
+    }
+    return make_double2(rr, rz);
+}
+
+// phase C: p = z + beta p
+__device__ __noinline__ void ph_p(const PcgArgs& P, double beta) {
+    const int lane = threadIdx.x & 31;
+    const int n = P.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    for (int grp = warp_id_global(); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        if (R.valid) P.p[R.idx] = ld_cg(P.z + R.idx) + beta * ld_cg(P.p + R.idx);
+    }
+}
+
+// SSOR-AI lower half pass: w = D^{-1} (r - omega L t)
+__device__ __noinline__ void ph_ssor_lower(const PcgArgs& P) {
+    const int lane = threadIdx.x & 31;
+    for_rows<SPMV_LOWER_T>(P.A, warp_id_global(), gridDim.x * WPB, XCg{P.t}, lane,
+                           [&](int i, bool ok, double y0, double y1) {
+                               ssor_lower_row(P.dinv, i, ok, y0, y1, P.r, P.omega, P.w, lane);
+                           });
+}
+
+// SSOR-AI upper half pass: z = w - omega D^{-1} U w (and p = z at setup); returns r^T z share
+__device__ __noinline__ double ph_ssor_upper(const PcgArgs& P, bool init) {
+    const int lane = threadIdx.x & 31;
+    double rz = 0.0;
+    for_rows<SPMV_UPPER>(P.A, warp_id_global(), gridDim.x * WPB, XCg{P.w}, lane,
+                         [&](int i, bool ok, double y0, double y1) {
+                             const double zz = ssor_upper_row(P.dinv, i, ok, y0, y1, P.w, P.omega, lane);
+                             if (ok && q_of(lane) < 6) {
+                                 const size_t idx = 6 * (size_t)i + q_of(lane);
+                                 P.z[idx] = zz;
+                                 if (init) P.p[idx] = zz;
+                                 rz += ld_cg(P.r + idx) * zz;
+                             }
+                         });
+    return rz;
+}
+
+// true residual share: sum (F - q)^2 with q = K d
+__device__ __noinline__ double ph_resid(const PcgArgs& P) {
+    const int lane = threadIdx.x & 31;
+    const int n = P.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    double acc = 0.0;
+    for (int grp = warp_id_global(); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        if (R.valid) {
+            const double e = P.F[R.idx] - ld_cg(P.q + R.idx);
+            acc += e * e;
+        }
+    }
+    return acc;
+}
+
+__device__ __noinline__ void ph_zero_d(const PcgArgs& P) {
+    const int lane = threadIdx.x & 31;
+    const int n = P.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    for (int grp = warp_id_global(); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        if (R.valid) P.d[R.idx] = 0.0;
+    }
+}
+
+template <int MINB>
+__global__ void __launch_bounds__(DDA_THREADS, MINB) k_pcg(const __grid_constant__ PcgArgs P) {
     cg::grid_group grid = cg::this_grid();
     __shared__ double red[WPB][4];
     __shared__ double bc[4];
-    const int lane = threadIdx.x & 31;
     const int G = gridDim.x;
-    const int gw = blockIdx.x * WPB + (threadIdx.x >> 5);
-    const int W = G * WPB;
-    const int n = P.A.n;
-    const int ngrp = (n + 4) / 5;
-    const bool use_dinv = (P.pc == DDA_PC_BJ || P.pc == DDA_PC_SSOR_AI);
-
-    // z = M^{-1} r for SSOR-AI given t = D^{-1} r already stored: two half passes.
-    // Writes z (and p = z when init); returns the CTA-local r^T z contribution.
-    auto ssor_passes = [&](bool init) -> double {
-        for (int i = gw; i < n; i += W) ssor_lower_row(P.A, P.dinv, i, P.r, P.t, P.omega, P.w, lane);
-        grid.sync();
-        double rz = 0.0;
-        for (int i = gw; i < n; i += W) {
-            const double zz = ssor_upper_row(P.A, P.dinv, i, P.w, P.omega, lane);
-            if (lane < 6) {
-                const size_t idx = 6 * (size_t)i + lane;
-                P.z[idx] = zz;
-                if (init) P.p[idx] = zz;
-                rz += ld_cg(P.r + idx) * zz;
-            }
-        }
-        return rz;
-    };
 
     // ------------------------------------------------------------ setup: r = F - K d0
     if (P.d0) {
-        for (int i = gw; i < n; i += W) {
-            double y0, y1;
-            spmv_row<SPMV_FULL>(P.A, i, XCg{P.d0}, lane, y0, y1);
-            if (lane < 9 && lane % 3 == 0)
-                *reinterpret_cast<double2*>(P.q + 6 * (size_t)i + 2 * (lane / 3)) = make_double2(y0, y1);
-        }
+        ph_spmv(P, P.d0, false);
         grid.sync();
     }
     {
-        double v[3] = {0.0, 0.0, 0.0};   // FF, rr, rz
-        for (int grp = gw; grp < ngrp; grp += W) {
-            const Row5 R = row5(grp, lane, n);
-            double rv = 0.0, fv = 0.0;
-            if (R.valid) {
-                fv = P.F[R.idx];
-                const double dv = P.d0 ? ld_cg(P.d0 + R.idx) : 0.0;
-                if (P.d != P.d0) P.d[R.idx] = dv;
-                rv = P.d0 ? fv - ld_cg(P.q + R.idx) : fv;
-                P.r[R.idx] = rv;
-            }
-            v[0] += fv * fv;
-            v[1] += rv * rv;
-            const double tz = use_dinv ? bj_lane(P.dinv, R, rv) : rv;
-            if (R.valid) {
-                if (P.pc == DDA_PC_SSOR_AI) {
-                    P.t[R.idx] = tz;
-                } else {
-                    P.z[R.idx] = tz;
-                    P.p[R.idx] = tz;
-                    v[2] += rv * tz;
-                }
-            }
-        }
+        const double3 v3 = ph_init(P);
+        double v[3] = {v3.x, v3.y, v3.z};
         cta_partials<3>(v, P.part, G, red);
     }
     grid.sync();
@@ -172,18 +269,17 @@ __global__ void __launch_bounds__(DDA_THREADS) k_pcg(PcgArgs P) {
     int iters = 0;
     bool skip_final = false;
     if (FF == 0.0) {                                    // reading Z2: d = 0, iters = 0, rel_res = 0
-        for (int grp = gw; grp < ngrp; grp += W) {
-            const Row5 R = row5(grp, lane, n);
-            if (R.valid) P.d[R.idx] = 0.0;
-        }
+        ph_zero_d(P);
         status = DDA_OK;
         skip_final = true;
     } else if (sqrt(rr) <= P.tol * bnorm) {
         status = DDA_OK;
     } else {
         if (P.pc == DDA_PC_SSOR_AI) {
-            grid.sync();                                // t visible
-            double v[1] = {ssor_passes(true)};
+            grid.sync();                                // t visible; part[2G..] free again
+            ph_ssor_lower(P);
+            grid.sync();
+            double v[1] = {ph_ssor_upper(P, true)};
             cta_partials<1>(v, P.part + 2 * G, G, red);
             grid.sync();
             double s[1];
@@ -196,17 +292,7 @@ __global__ void __launch_bounds__(DDA_THREADS) k_pcg(PcgArgs P) {
             for (int k = 0; k < P.maxit; ++k) {
                 // ---- phase A: q = K p, partial p^T q
                 {
-                    double v[1] = {0.0};
-                    for (int i = gw; i < n; i += W) {
-                        double y0, y1;
-                        spmv_row<SPMV_FULL>(P.A, i, XCg{P.p}, lane, y0, y1);
-                        if (lane < 9 && lane % 3 == 0) {
-                            const size_t o = 6 * (size_t)i + 2 * (lane / 3);
-                            *reinterpret_cast<double2*>(P.q + o) = make_double2(y0, y1);
-                            const double2 pv = ld_cg2(P.p + o);
-                            v[0] += pv.x * y0 + pv.y * y1;
-                        }
-                    }
+                    double v[1] = {ph_spmv(P, P.p, true)};
                     cta_partials<1>(v, P.part, G, red);
                 }
                 grid.sync();
@@ -220,27 +306,8 @@ __global__ void __launch_bounds__(DDA_THREADS) k_pcg(PcgArgs P) {
                 const double alpha = rho / sigma;
                 // ---- phase B: d += alpha p; r -= alpha q; z = M^{-1} r (BJ / none) or t = D^{-1} r
                 {
-                    double v[2] = {0.0, 0.0};   // rr, rz
-                    for (int grp = gw; grp < ngrp; grp += W) {
-                        const Row5 R = row5(grp, lane, n);
-                        double rv = 0.0;
-                        if (R.valid) {
-                            const double pv = ld_cg(P.p + R.idx);
-                            P.d[R.idx] = ld_cg(P.d + R.idx) + alpha * pv;
-                            rv = ld_cg(P.r + R.idx) - alpha * ld_cg(P.q + R.idx);
-                            P.r[R.idx] = rv;
-                        }
-                        v[0] += rv * rv;
-                        const double tz = use_dinv ? bj_lane(P.dinv, R, rv) : rv;
-                        if (R.valid) {
-                            if (P.pc == DDA_PC_SSOR_AI) {
-                                P.t[R.idx] = tz;
-                            } else {
-                                P.z[R.idx] = tz;
-                                v[1] += rv * tz;
-                            }
-                        }
-                    }
+                    const double2 v2 = ph_update(P, alpha);
+                    double v[2] = {v2.x, v2.y};
                     cta_partials<2>(v, P.part + G, G, red);
                 }
                 grid.sync();
@@ -253,7 +320,9 @@ __global__ void __launch_bounds__(DDA_THREADS) k_pcg(PcgArgs P) {
                 iters = k + 1;
                 if (sqrt(rr) <= P.tol * bnorm) { status = DDA_OK; break; }
                 if (P.pc == DDA_PC_SSOR_AI) {
-                    double v[1] = {ssor_passes(false)};
+                    ph_ssor_lower(P);
+                    grid.sync();
+                    double v[1] = {ph_ssor_upper(P, false)};
                     cta_partials<1>(v, P.part + 2 * G, G, red);
                     grid.sync();
                     double s[1];
@@ -264,10 +333,7 @@ __global__ void __launch_bounds__(DDA_THREADS) k_pcg(PcgArgs P) {
                 const double beta = rz / rho;
                 rho = rz;
                 // ---- phase C: p = z + beta p
-                for (int grp = gw; grp < ngrp; grp += W) {
-                    const Row5 R = row5(grp, lane, n);
-                    if (R.valid) P.p[R.idx] = ld_cg(P.z + R.idx) + beta * ld_cg(P.p + R.idx);
-                }
+                ph_p(P, beta);
                 grid.sync();
             }
         }
@@ -277,21 +343,9 @@ __global__ void __launch_bounds__(DDA_THREADS) k_pcg(PcgArgs P) {
     double rel = 0.0;
     if (!skip_final) {
         grid.sync();
-        for (int i = gw; i < n; i += W) {
-            double y0, y1;
-            spmv_row<SPMV_FULL>(P.A, i, XCg{P.d}, lane, y0, y1);
-            if (lane < 9 && lane % 3 == 0)
-                *reinterpret_cast<double2*>(P.q + 6 * (size_t)i + 2 * (lane / 3)) = make_double2(y0, y1);
-        }
+        ph_spmv(P, P.d, false);
         grid.sync();
-        double v[1] = {0.0};
-        for (int grp = gw; grp < ngrp; grp += W) {
-            const Row5 R = row5(grp, lane, n);
-            if (R.valid) {
-                const double e = P.F[R.idx] - ld_cg(P.q + R.idx);
-                v[0] += e * e;
-            }
-        }
+        double v[1] = {ph_resid(P)};
         cta_partials<1>(v, P.part + 3 * G, G, red);
         grid.sync();
         double s[1];
@@ -307,13 +361,27 @@ __global__ void __launch_bounds__(DDA_THREADS) k_pcg(PcgArgs P) {
     }
 }
 
+typedef void (*PcgKernel)(const PcgArgs);
+// occupancy variants (tuning aid, DDA_PCG_VARIANT): min CTAs of 256 threads per SM
+const PcgKernel kPcgVariants[] = {k_pcg<5>, k_pcg<6>, k_pcg<4>};
+
+PcgKernel pcg_kernel() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("DDA_PCG_VARIANT");
+        v = e ? atoi(e) : 0;
+        if (v < 0 || v > 2) v = 0;
+    }
+    return kPcgVariants[v];
+}
+
 int pcg_grid() {
     static int cached_dev = -1, cached = 0;
     int dev = 0;
     cudaGetDevice(&dev);
     if (dev != cached_dev) {
         int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_pcg, DDA_THREADS, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, pcg_kernel(), DDA_THREADS, 0);
         cached = device_sms() * (per_sm > 0 ? per_sm : 1);
         cached_dev = dev;
     }
@@ -334,7 +402,7 @@ dda_status_t pcg_solve(dda_matrix* K, const double* F, const double* d0, double*
     }
     const size_t N = 6 * (size_t)K->n;
     int G = pcg_grid();
-    const int need = (K->n + WPB - 1) / WPB;
+    const int need = (K->n + 3 * WPB - 1) / (3 * WPB);
     if (need < G) G = need > 0 ? need : 1;
     const size_t bytes = (6 * N + 4 * (size_t)G) * sizeof(double);
     {
@@ -360,7 +428,7 @@ dda_status_t pcg_solve(dda_matrix* K, const double* F, const double* d0, double*
     a.tol = tol;
     a.maxit = maxit;
     void* args[] = {&a};
-    DDA_CK(cudaLaunchCooperativeKernel((const void*)k_pcg, dim3(G), dim3(DDA_THREADS), args, 0, st));
+    DDA_CK(cudaLaunchCooperativeKernel((const void*)pcg_kernel(), dim3(G), dim3(DDA_THREADS), args, 0, st));
     note_launch();
     PcgOut h;
     DDA_CK(cudaMemcpyAsync(&h, a.out, sizeof h, cudaMemcpyDeviceToHost, st));

@@ -99,18 +99,21 @@ __global__ void __launch_bounds__(DDA_THREADS) k_ssor_lower(BsrView A, const dou
                                                             const double* r, const double* t, double* w) {
     const int lane = threadIdx.x & 31;
     const int W = gridDim.x * (DDA_THREADS / 32);
-    for (int i = blockIdx.x * (DDA_THREADS / 32) + (threadIdx.x >> 5); i < A.n; i += W)
-        ssor_lower_row(A, dinv, i, r, t, omega, w, lane);
+    for_rows<SPMV_LOWER_T>(A, blockIdx.x * (DDA_THREADS / 32) + (threadIdx.x >> 5), W, XCg{t}, lane,
+                           [&](int i, bool ok, double y0, double y1) {
+                               ssor_lower_row(dinv, i, ok, y0, y1, r, omega, w, lane);
+                           });
 }
 
 __global__ void __launch_bounds__(DDA_THREADS) k_ssor_upper(BsrView A, const double* __restrict__ dinv, double omega,
                                                             const double* w, double* z) {
     const int lane = threadIdx.x & 31;
     const int W = gridDim.x * (DDA_THREADS / 32);
-    for (int i = blockIdx.x * (DDA_THREADS / 32) + (threadIdx.x >> 5); i < A.n; i += W) {
-        const double zz = ssor_upper_row(A, dinv, i, w, omega, lane);
-        if (lane < 6) z[6 * (size_t)i + lane] = zz;
-    }
+    for_rows<SPMV_UPPER>(A, blockIdx.x * (DDA_THREADS / 32) + (threadIdx.x >> 5), W, XCg{w}, lane,
+                         [&](int i, bool ok, double y0, double y1) {
+                             const double zz = ssor_upper_row(dinv, i, ok, y0, y1, w, omega, lane);
+                             if (ok && q_of(lane) < 6) z[6 * (size_t)i + q_of(lane)] = zz;
+                         });
 }
 
 int grid_rows(int rows_per_warp, int n) {
@@ -182,9 +185,9 @@ extern "C" dda_status_t dda_precond_apply(dda_matrix_t K, dda_precond_t pc, doub
         double* w = K->ws + N;
         k_bj_apply<<<grid_rows(5, K->n), DDA_THREADS, 0, st>>>(K->n, K->dinv, r, t);
         DDA_LAUNCHED();
-        k_ssor_lower<<<grid_rows(1, K->n), DDA_THREADS, 0, st>>>(view_of(K), K->dinv, omega, r, t, w);
+        k_ssor_lower<<<grid_rows(3, K->n), DDA_THREADS, 0, st>>>(view_of(K), K->dinv, omega, r, t, w);
         DDA_LAUNCHED();
-        k_ssor_upper<<<grid_rows(1, K->n), DDA_THREADS, 0, st>>>(view_of(K), K->dinv, omega, w, z);
+        k_ssor_upper<<<grid_rows(3, K->n), DDA_THREADS, 0, st>>>(view_of(K), K->dinv, omega, w, z);
         DDA_LAUNCHED();
     }
     DDA_CK(cudaStreamSynchronize(st));

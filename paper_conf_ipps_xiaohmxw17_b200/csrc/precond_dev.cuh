@@ -44,30 +44,30 @@ __device__ __forceinline__ double bj_lane(const double* __restrict__ dinv, const
     return dinv_apply6(blk, v, R.a, R.base);
 }
 
-// SSOR-AI lower half-pass, warp per row i (reading Z14, A7 step 2-3):
+// SSOR-AI lower half-pass epilogue (reading Z14, A7 steps 2-3) for the lane's
+// group row i, given (y0, y1) = the SPMV_LOWER_T row product of t:
 //   s_i = r_i - omega * sum_{k<i} V_ki^T t_k ;  w_i = D_i^{-1} s_i
-__device__ __forceinline__ void ssor_lower_row(const BsrView& A, const double* __restrict__ dinv, int i,
-                                               const double* r, const double* t, double omega, double* w,
-                                               int lane) {
-    double y0, y1;
-    spmv_row<SPMV_LOWER_T>(A, i, XCg{t}, lane, y0, y1);
+__device__ __forceinline__ void ssor_lower_row(const double* __restrict__ dinv, int i, bool ok, double y0, double y1,
+                                               const double* r, double omega, double* w, int lane) {
     const double lt = pairs_to_dof(y0, y1, lane);
-    const int a = lane < 6 ? lane : 0;
-    const double s = (lane < 6) ? ld_cg(r + 6 * (size_t)i + a) - omega * lt : 0.0;
-    const double wv = dinv_apply6(dinv + (size_t)kDinv * i, s, a, 0);
-    if (lane < 6) w[6 * (size_t)i + a] = wv;
+    const int q = q_of(lane);
+    const int a = q < 6 ? q : 0;
+    const bool mine = ok && q < 6;
+    const double s = mine ? ld_cg(r + 6 * (size_t)i + a) - omega * lt : 0.0;
+    const double wv = dinv_apply6(dinv + (size_t)kDinv * (ok ? i : 0), s, a, 9 * grp_of(lane));
+    if (mine) w[6 * (size_t)i + a] = wv;
 }
 
-// SSOR-AI upper half-pass, warp per row i (A7 step 4):
-//   z_i = w_i - omega * D_i^{-1} sum_{j>i} V_ij w_j      (returned on lanes 0..5)
-__device__ __forceinline__ double ssor_upper_row(const BsrView& A, const double* __restrict__ dinv, int i,
-                                                 const double* w, double omega, int lane) {
-    double y0, y1;
-    spmv_row<SPMV_UPPER>(A, i, XCg{w}, lane, y0, y1);
+// SSOR-AI upper half-pass epilogue (A7 step 4) for the lane's group row i, given
+// (y0, y1) = the SPMV_UPPER row product of w:
+//   z_i = w_i - omega * D_i^{-1} sum_{j>i} V_ij w_j   (valid on lanes q < 6 of groups with a row)
+__device__ __forceinline__ double ssor_upper_row(const double* __restrict__ dinv, int i, bool ok, double y0,
+                                                 double y1, const double* w, double omega, int lane) {
     const double uw = pairs_to_dof(y0, y1, lane);
-    const int a = lane < 6 ? lane : 0;
-    const double du = dinv_apply6(dinv + (size_t)kDinv * i, uw, a, 0);
-    return ld_cg(w + 6 * (size_t)i + a) - omega * du;
+    const int q = q_of(lane);
+    const int a = q < 6 ? q : 0;
+    const double du = dinv_apply6(dinv + (size_t)kDinv * (ok ? i : 0), uw, a, 9 * grp_of(lane));
+    return (ok && q < 6) ? ld_cg(w + 6 * (size_t)i + a) - omega * du : 0.0;
 }
 
 }  // namespace dda

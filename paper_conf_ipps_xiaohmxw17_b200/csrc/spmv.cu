@@ -5,6 +5,8 @@
 // and the transposed block V_ki needed by row i was streamed from HBM by the
 // warp of row k a short time earlier (one course of the slope ~ 1-3 MB of
 // traffic ago): it is re-read from the 126 MB L2, not from HBM.
+#include <cstdlib>
+
 #include "spmv_warp.cuh"
 
 namespace dda {
@@ -17,39 +19,50 @@ struct XLdg {
     }
 };
 
-template <int MODE>
-__global__ void __launch_bounds__(DDA_THREADS) k_spmv(BsrView A, const double* __restrict__ x,
-                                                      double* __restrict__ y) {
+template <int MODE, int MINB>
+__global__ void __launch_bounds__(DDA_THREADS, MINB) k_spmv(BsrView A, const double* __restrict__ x,
+                                                            double* __restrict__ y) {
     const int lane = threadIdx.x & 31;
     const int W = gridDim.x * (DDA_THREADS / 32);
-    for (int i = blockIdx.x * (DDA_THREADS / 32) + (threadIdx.x >> 5); i < A.n; i += W) {
-        double y0, y1;
-        spmv_row<MODE>(A, i, XLdg{x}, lane, y0, y1);
-        if (lane < 9 && (lane % 3) == 0)
-            *reinterpret_cast<double2*>(y + 6 * (size_t)i + 2 * (lane / 3)) = make_double2(y0, y1);
-    }
+    auto st = [&](int i, bool ok, double y0, double y1) {
+        if (ok && is_out_lane(lane))
+            *reinterpret_cast<double2*>(y + 6 * (size_t)i + 2 * (q_of(lane) / 3)) = make_double2(y0, y1);
+    };
+    for_rows<MODE>(A, blockIdx.x * (DDA_THREADS / 32) + (threadIdx.x >> 5), W, XLdg{x}, lane, st);
 }
 
-int spmv_grid() {
-    static int cached_dev = -1, cached = 0;
-    int dev = 0;
-    cudaGetDevice(&dev);
-    if (dev != cached_dev) {
-        int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_spmv<SPMV_FULL>, DDA_THREADS, 0);
-        cached = device_sms() * (per_sm > 0 ? per_sm : 1);
-        cached_dev = dev;
+// occupancy variants for tuning (DDA_SPMV_VARIANT): min CTAs per SM of 256 threads
+typedef void (*SpmvKernel)(BsrView, const double*, double*);
+struct Variant { SpmvKernel k; const char* name; };
+const Variant kVariants[] = {
+    {k_spmv<SPMV_FULL, 6>, "b6"}, {k_spmv<SPMV_FULL, 4>, "b4"}, {k_spmv<SPMV_FULL, 8>, "b8"},
+};
+constexpr int kNumVariants = sizeof(kVariants) / sizeof(kVariants[0]);
+
+int variant() {
+    static int v = -2;
+    if (v == -2) {
+        const char* e = getenv("DDA_SPMV_VARIANT");
+        v = e ? atoi(e) : 0;
+        if (v < 0 || v >= kNumVariants) v = 0;
     }
-    return cached;
+    return v;
+}
+
+int spmv_grid(SpmvKernel k) {
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, DDA_THREADS, 0);
+    return device_sms() * (per_sm > 0 ? per_sm : 1);
 }
 
 }  // namespace
 
 dda_status_t spmv(dda_matrix* K, const double* x, double* y, cudaStream_t s) {
-    int g = spmv_grid();
-    const int need = (K->n + DDA_THREADS / 32 - 1) / (DDA_THREADS / 32);
+    const SpmvKernel k = kVariants[variant()].k;
+    int g = spmv_grid(k);
+    const int need = (K->n + 3 * (DDA_THREADS / 32) - 1) / (3 * (DDA_THREADS / 32));
     if (need < g) g = need > 0 ? need : 1;
-    k_spmv<SPMV_FULL><<<g, DDA_THREADS, 0, s>>>(view_of(K), x, y);
+    k<<<g, DDA_THREADS, 0, s>>>(view_of(K), x, y);
     DDA_LAUNCHED();
     return DDA_OK;
 }
