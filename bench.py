@@ -57,11 +57,13 @@ def bytes_per_row_spmv(u: float) -> float:
 
 def pcg_launch_bytes(n: int, u: float, iters: int) -> float:
     """Algorithmic bytes of one k_pcg launch with block-Jacobi, d0 = 0:
-    init 432 B/row (F, Dinv read; d, r, z, p written), per iteration SpMV + 528 (phase B:
-    p, d, r, q, Dinv read; d, r, z written) + 144 (phase C: z, p read, p written), final
+    init 432 B/row (F, Dinv read; d, r, z, p written); iteration 0: SpMV of p + phase B 528
+    (p, d, r, q, Dinv read; d, r, z written); iterations k >= 1: SpMV whose x = z + beta p_old
+    is two vectors (+48) and whose owner writes p_new (+48), + phase B 528; final
     true-residual SpMV + 96 (F, q read)."""
     S = bytes_per_row_spmv(u)
-    return n * (432.0 + iters * (S + 528.0 + 144.0) + S + 96.0)
+    it = max(iters, 1)
+    return n * (432.0 + (S + 528.0) + (it - 1) * (S + 96.0 + 528.0) + S + 96.0)
 
 
 class ClockSampler:

@@ -282,7 +282,7 @@ extern "C" dda_status_t dda_build_matrix(int32_t n, const double* kdiag, int64_t
         void* tsort = nullptr;
         DDA_CK(tmp.get(reinterpret_cast<char**>(&tsort), tb));
         DDA_CK(cub::DeviceRadixSort::SortPairs(tsort, tb, key, skey, val, K->perm, (int)m, 0, kbits, st));
-        note_launch(2 * ((kbits + 6) / 7) + 1);
+        note_launch(2 + (kbits + 7) / 8);   // onesweep: histogram + exclusive sum + one pass per 8 bits
         // ---- (3) boundary flags + scan
         k_heads<<<grid_for(m), TPB, 0, st>>>(m, skey, flag);
         DDA_LAUNCHED();
@@ -338,7 +338,7 @@ extern "C" dda_status_t dda_build_matrix(int32_t n, const double* kdiag, int64_t
             void* tsort = nullptr;
             DDA_CK(tmp.get(reinterpret_cast<char**>(&tsort), tb));
             DDA_CK(cub::DeviceRadixSort::SortPairs(tsort, tb, dkey, dskey, dval, K->dperm, (int)(2 * m), 0, dbits, st));
-            note_launch(2 * ((dbits + 6) / 7) + 1);
+            note_launch(2 + (dbits + 7) / 8);
         }
         k_bounds<<<grid_for(2 * m + 1), TPB, 0, st>>>(n, 2 * m, dskey, K->dstart);
         DDA_LAUNCHED();
@@ -366,7 +366,7 @@ extern "C" dda_status_t dda_build_matrix(int32_t n, const double* kdiag, int64_t
         void* tsort = nullptr;
         DDA_CK(tmp.get(reinterpret_cast<char**>(&tsort), tb));
         DDA_CK(cub::DeviceRadixSort::SortPairs(tsort, tb, tkey, tskey, tval, K->low_to_up, nnzb, 0, kbits, st));
-        note_launch(2 * ((kbits + 6) / 7) + 1);
+        note_launch(2 + (kbits + 7) / 8);   // onesweep: histogram + exclusive sum + one pass per 8 bits
         k_tfill<<<grid_for(nnzb), TPB, 0, st>>>(n, nnzb, tskey, K->low_row, tcol);
         DDA_LAUNCHED();
         k_bounds<<<grid_for((int64_t)nnzb + 1), TPB, 0, st>>>(n, nnzb, tcol, K->low_ptr);

@@ -1,16 +1,17 @@
 // A5/A6 — the PCG solve of K d = F as ONE persistent cooperative kernel
 // (§IV.A; textbook PCG, Saad Alg. 9.1, reading Z1/Z2/Z19).
 //
-// Per iteration (block-Jacobi):
-//   phase A  q = K p (warp per block row, spmv_row) + CTA partial of p^T q
+// Per iteration k (block-Jacobi):
+//   phase A  p^(k) = z + beta p^(k-1) formed on the fly for every gathered
+//            neighbour and written by the owner of each row (the textbook
+//            "phase C" fused into the SpMV, ping-pong p buffers), q = K p^(k),
+//            CTA partial of p^T q
 //   -- grid barrier --  sigma = fixed-order sum of the partials (every CTA)
 //   phase B  alpha = rho/sigma; d += alpha p; r -= alpha q; z = D^{-1} r;
 //            partials of r^T r and r^T z
 //   -- grid barrier --  convergence test ||r|| <= tol ||F||, beta = rho'/rho
-//   phase C  p = z + beta p
-//   -- grid barrier --
-// SSOR-AI inserts its two half-passes (lower on t = D^{-1} r, upper on w)
-// between B and C, with a barrier after each.  Every CTA evaluates the scalars
+// Two grid barriers per iteration.  SSOR-AI inserts its two half-passes
+// (lower on t = D^{-1} r, upper on w) after B, with a barrier after each.  Every CTA evaluates the scalars
 // itself from the same partials in the same order, so all CTAs take the same
 // branch and the result is bitwise reproducible for a given launch
 // configuration.  The host reads the outcome once, after the kernel.
@@ -44,7 +45,8 @@ struct PcgArgs {
     double* d;
     double* r;
     double* z;
-    double* p;
+    double* p;             // p buffer 0 (p^(k) lives in buffer k % 2)
+    double* p1;            // p buffer 1
     double* q;
     double* t;
     double* w;
@@ -119,6 +121,37 @@ __device__ __noinline__ double ph_spmv(const PcgArgs& P, const double* x, bool d
     return acc;
 }
 
+// x_j = z_j + beta * p_j formed on the fly (phase C fused into the next SpMV)
+struct XFused {
+    const double* z;
+    const double* p;
+    double beta;
+    __device__ __forceinline__ double2 operator()(int vec, int pair) const {
+        const size_t o = 6 * (size_t)vec + 2 * pair;
+        const double2 zz = ld_cg2(z + o), pp = ld_cg2(p + o);
+        return make_double2(fma(beta, pp.x, zz.x), fma(beta, pp.y, zz.y));
+    }
+};
+
+// p_new = z + beta p_old (own rows, written), q = K p_new; returns this lane's share of p_new^T q
+__device__ __noinline__ double ph_spmv_fused(const PcgArgs& P, const double* pold, double* pnew, double beta) {
+    const int lane = threadIdx.x & 31;
+    const XFused xf{P.z, pold, beta};
+    double acc = 0.0;
+    for_rows<SPMV_FULL>(P.A, warp_id_global(), gridDim.x * WPB, xf, lane,
+                        [&](int i, bool ok, double y0, double y1) {
+                            const int q = q_of(lane);
+                            if (ok && is_out_lane(lane)) {
+                                const size_t o = 6 * (size_t)i + 2 * (q / 3);
+                                *reinterpret_cast<double2*>(P.q + o) = make_double2(y0, y1);
+                                const double2 pv = xf(i, q / 3);
+                                *reinterpret_cast<double2*>(pnew + o) = pv;
+                                acc += pv.x * y0 + pv.y * y1;
+                            }
+                        });
+    return acc;
+}
+
 // setup: d = d0 (or 0), r = F - q (or F), t/z/p = M^{-1} r pieces; partials (F^T F, r^T r, r^T z)
 __device__ __noinline__ double3 ph_init(const PcgArgs& P) {
     const int lane = threadIdx.x & 31;
@@ -152,7 +185,7 @@ __device__ __noinline__ double3 ph_init(const PcgArgs& P) {
 }
 
 // phase B: d += alpha p; r -= alpha q; z = D^{-1} r (BJ) / t = D^{-1} r (SSOR) / z = r; partials (r^T r, r^T z)
-__device__ __noinline__ double2 ph_update(const PcgArgs& P, double alpha) {
+__device__ __noinline__ double2 ph_update(const PcgArgs& P, const double* pk, double alpha) {
     const int lane = threadIdx.x & 31;
     const int n = P.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
     const bool use_dinv = (P.pc == DDA_PC_BJ || P.pc == DDA_PC_SSOR_AI);
@@ -161,7 +194,7 @@ __device__ __noinline__ double2 ph_update(const PcgArgs& P, double alpha) {
         const Row5 R = row5(grp, lane, n);
         double rv = 0.0;
         if (R.valid) {
-            const double pv = ld_cg(P.p + R.idx);
+            const double pv = ld_cg(pk + R.idx);
             P.d[R.idx] = ld_cg(P.d + R.idx) + alpha * pv;
             rv = ld_cg(P.r + R.idx) - alpha * ld_cg(P.q + R.idx);
             P.r[R.idx] = rv;
@@ -178,16 +211,6 @@ __device__ __noinline__ double2 ph_update(const PcgArgs& P, double alpha) {
         }
     }
     return make_double2(rr, rz);
-}
-
-// phase C: p = z + beta p
-__device__ __noinline__ void ph_p(const PcgArgs& P, double beta) {
-    const int lane = threadIdx.x & 31;
-    const int n = P.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
-    for (int grp = warp_id_global(); grp < ngrp; grp += W) {
-        const Row5 R = row5(grp, lane, n);
-        if (R.valid) P.p[R.idx] = ld_cg(P.z + R.idx) + beta * ld_cg(P.p + R.idx);
-    }
 }
 
 // SSOR-AI lower half pass: w = D^{-1} (r - omega L t)
@@ -289,10 +312,13 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_pcg(const __grid_constant
         if (!(rho > 0.0) || !isfinite(rho)) {
             status = DDA_ERR_BREAKDOWN;
         } else {
+            double beta = 0.0;
             for (int k = 0; k < P.maxit; ++k) {
-                // ---- phase A: q = K p, partial p^T q
+                double* pk = (k & 1) ? P.p1 : P.p;
+                // ---- phase A: p^(k) = z + beta p^(k-1) (k > 0), q = K p^(k), partial p^T q
                 {
-                    double v[1] = {ph_spmv(P, P.p, true)};
+                    double v[1] = {k == 0 ? ph_spmv(P, P.p, true)
+                                          : ph_spmv_fused(P, (k & 1) ? P.p : P.p1, pk, beta)};
                     cta_partials<1>(v, P.part, G, red);
                 }
                 grid.sync();
@@ -306,7 +332,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_pcg(const __grid_constant
                 const double alpha = rho / sigma;
                 // ---- phase B: d += alpha p; r -= alpha q; z = M^{-1} r (BJ / none) or t = D^{-1} r
                 {
-                    const double2 v2 = ph_update(P, alpha);
+                    const double2 v2 = ph_update(P, pk, alpha);
                     double v[2] = {v2.x, v2.y};
                     cta_partials<2>(v, P.part + G, G, red);
                 }
@@ -330,11 +356,9 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_pcg(const __grid_constant
                     rz = s[0];
                 }
                 if (!(rz > 0.0) || !isfinite(rz)) { status = DDA_ERR_BREAKDOWN; break; }
-                const double beta = rz / rho;
+                beta = rz / rho;
                 rho = rz;
-                // ---- phase C: p = z + beta p
-                ph_p(P, beta);
-                grid.sync();
+                // (phase C, p = z + beta p, is fused into the next phase A)
             }
         }
     }
@@ -404,7 +428,7 @@ dda_status_t pcg_solve(dda_matrix* K, const double* F, const double* d0, double*
     int G = pcg_grid();
     const int need = (K->n + 3 * WPB - 1) / (3 * WPB);
     if (need < G) G = need > 0 ? need : 1;
-    const size_t bytes = (6 * N + 4 * (size_t)G) * sizeof(double);
+    const size_t bytes = (7 * N + 4 * (size_t)G) * sizeof(double);
     {
         dda_status_t s = ensure_workspace(K, bytes, st);
         if (s != DDA_OK) return s;
@@ -421,7 +445,8 @@ dda_status_t pcg_solve(dda_matrix* K, const double* F, const double* d0, double*
     a.q = K->ws + 3 * N;
     a.t = K->ws + 4 * N;
     a.w = K->ws + 5 * N;
-    a.part = K->ws + 6 * N;
+    a.p1 = K->ws + 6 * N;
+    a.part = K->ws + 7 * N;
     a.out = reinterpret_cast<PcgOut*>(reinterpret_cast<char*>(K->scratch) + 64);
     a.pc = (int)pc;
     a.omega = omega;
