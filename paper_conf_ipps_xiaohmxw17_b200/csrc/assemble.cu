@@ -229,6 +229,7 @@ extern "C" void dda_matrix_free(dda_matrix_t K) {
     cudaGetDevice(&prev);
     cudaSetDevice(K->device);
     cudaDeviceSynchronize();   // no stream may still use the arrays
+    if (K->graph_engine) pcg_graph_free(K->graph_engine);
     void* ptrs[] = {K->row_ptr, K->col_idx, K->low_ptr, K->low_row, K->low_to_up, K->urow, K->diag, K->upper,
                     K->perm, K->seg, K->dperm, K->dstart, K->orient, K->dinv, K->ws, K->scratch};
     for (void* p : ptrs)

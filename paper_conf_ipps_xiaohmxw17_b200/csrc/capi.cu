@@ -50,6 +50,10 @@ void dev_free(void* p) { cudaFreeAsync(p, 0); }
 
 dda_status_t ensure_workspace(dda_matrix* K, size_t bytes, cudaStream_t st) {
     if (K->ws_bytes >= bytes) return DDA_OK;
+    if (K->graph_engine) {          // its graph has the old workspace pointers baked in
+        pcg_graph_free(K->graph_engine);
+        K->graph_engine = nullptr;
+    }
     if (K->ws) {
         cudaStreamSynchronize(st);
         dev_free(K->ws);

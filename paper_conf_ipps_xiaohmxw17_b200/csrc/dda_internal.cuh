@@ -66,9 +66,17 @@ __device__ __forceinline__ double4 ld_chunk(const double* p) {
                  : "=d"(v.x), "=d"(v.y), "=d"(v.z), "=d"(v.w) : "l"(p));
     return v;
 }
-// coherent (L2) loads for vectors written earlier in the same persistent kernel
+// Loads of vectors written earlier in the same persistent kernel.  They are only
+// read after a grid barrier (cooperative_groups grid.sync: a gpu-scope fence,
+// which also invalidates L1), so plain weak loads are coherent; they must not
+// use the read-only .nc path.  DDA_VEC_CG selects L2-only (.cg) loads instead.
+#ifdef DDA_VEC_CG
 __device__ __forceinline__ double2 ld_cg2(const double* p) { return __ldcg(reinterpret_cast<const double2*>(p)); }
 __device__ __forceinline__ double ld_cg(const double* p) { return __ldcg(p); }
+#else
+__device__ __forceinline__ double2 ld_cg2(const double* p) { return *reinterpret_cast<const double2*>(p); }
+__device__ __forceinline__ double ld_cg(const double* p) { return *p; }
+#endif
 
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
@@ -106,10 +114,16 @@ struct dda_matrix {
     double* ws = nullptr;
     size_t ws_bytes = 0;
     void* scratch = nullptr;        // small device scratch (result struct, flags)
+    void* graph_engine = nullptr;   // cached CUDA-graph PCG engine (pcg_graph.cu)
+    int64_t graph_iters = 0;        // loop-body launches issued inside graphs (launch accounting)
 };
 
 namespace dda {
 dda_status_t ensure_workspace(dda_matrix* K, size_t bytes, cudaStream_t st);
 dda_status_t bj_setup(dda_matrix* K, cudaStream_t s, int32_t* bad_block);
 dda_status_t spmv(dda_matrix* K, const double* x, double* y, cudaStream_t s);
+void pcg_graph_free(void* g);
+dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, double* d, double tol,
+                             int32_t maxit, dda_precond_t pc, double omega, int32_t* iters, double* rel_res,
+                             cudaStream_t st);
 }  // namespace dda

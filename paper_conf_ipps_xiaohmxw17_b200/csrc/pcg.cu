@@ -213,6 +213,16 @@ __device__ __noinline__ double2 ph_update(const PcgArgs& P, const double* pk, do
     return make_double2(rr, rz);
 }
 
+// phase C (unfused variant): p = z + beta p
+__device__ __noinline__ void ph_p(const PcgArgs& P, double beta) {
+    const int lane = threadIdx.x & 31;
+    const int n = P.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    for (int grp = warp_id_global(); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        if (R.valid) P.p[R.idx] = fma(beta, ld_cg(P.p + R.idx), ld_cg(P.z + R.idx));
+    }
+}
+
 // SSOR-AI lower half pass: w = D^{-1} (r - omega L t)
 __device__ __noinline__ void ph_ssor_lower(const PcgArgs& P) {
     const int lane = threadIdx.x & 31;
@@ -263,7 +273,7 @@ __device__ __noinline__ void ph_zero_d(const PcgArgs& P) {
     }
 }
 
-template <int MINB>
+template <int MINB, bool FUSED>
 __global__ void __launch_bounds__(DDA_THREADS, MINB) k_pcg(const __grid_constant__ PcgArgs P) {
     cg::grid_group grid = cg::this_grid();
     __shared__ double red[WPB][4];
@@ -314,11 +324,11 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_pcg(const __grid_constant
         } else {
             double beta = 0.0;
             for (int k = 0; k < P.maxit; ++k) {
-                double* pk = (k & 1) ? P.p1 : P.p;
+                double* pk = (FUSED && (k & 1)) ? P.p1 : P.p;
                 // ---- phase A: p^(k) = z + beta p^(k-1) (k > 0), q = K p^(k), partial p^T q
                 {
-                    double v[1] = {k == 0 ? ph_spmv(P, P.p, true)
-                                          : ph_spmv_fused(P, (k & 1) ? P.p : P.p1, pk, beta)};
+                    double v[1] = {(k == 0 || !FUSED) ? ph_spmv(P, FUSED ? P.p : P.p, true)
+                                                      : ph_spmv_fused(P, (k & 1) ? P.p : P.p1, pk, beta)};
                     cta_partials<1>(v, P.part, G, red);
                 }
                 grid.sync();
@@ -358,7 +368,10 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_pcg(const __grid_constant
                 if (!(rz > 0.0) || !isfinite(rz)) { status = DDA_ERR_BREAKDOWN; break; }
                 beta = rz / rho;
                 rho = rz;
-                // (phase C, p = z + beta p, is fused into the next phase A)
+                if (!FUSED) {   // phase C: p = z + beta p (else fused into the next phase A)
+                    ph_p(P, beta);
+                    grid.sync();
+                }
             }
         }
     }
@@ -387,14 +400,14 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_pcg(const __grid_constant
 
 typedef void (*PcgKernel)(const PcgArgs);
 // occupancy variants (tuning aid, DDA_PCG_VARIANT): min CTAs of 256 threads per SM
-const PcgKernel kPcgVariants[] = {k_pcg<5>, k_pcg<6>, k_pcg<4>};
+const PcgKernel kPcgVariants[] = {k_pcg<5, true>, k_pcg<5, false>, k_pcg<6, true>, k_pcg<6, false>};
 
 PcgKernel pcg_kernel() {
     static int v = -1;
     if (v < 0) {
         const char* e = getenv("DDA_PCG_VARIANT");
         v = e ? atoi(e) : 0;
-        if (v < 0 || v > 2) v = 0;
+        if (v < 0 || v > 3) v = 0;
     }
     return kPcgVariants[v];
 }
@@ -467,10 +480,36 @@ dda_status_t pcg_solve(dda_matrix* K, const double* F, const double* d0, double*
 
 using namespace dda;
 
+// Engine choice: the CUDA-graph while loop (one kernel per phase, each at its
+// own occupancy) wins when the phases are HBM-bound; the persistent cooperative
+// kernel (grid barriers instead of kernel boundaries) wins for L2-resident
+// block-Jacobi solves (10k blocks: 15.5 vs 18.6 us/iteration on B200).
+// DDA_PCG_ENGINE=graph|persistent overrides.
+static int pcg_engine(const dda_matrix* K, dda_precond_t pc) {   // 0 = graph, 1 = persistent
+    static int forced = -2;
+    if (forced == -2) {
+        const char* v = getenv("DDA_PCG_ENGINE");
+        forced = !v ? -1 : ((v[0] == 'p' || v[0] == '1') ? 1 : 0);
+    }
+    if (forced >= 0) return forced;
+    return (pc != DDA_PC_SSOR_AI && K->n < 65536) ? 1 : 0;
+}
+
 extern "C" dda_status_t dda_pcg_solve(dda_matrix_t K, const double* F, const double* d0, double* d, double tol,
                                       int32_t maxit, dda_precond_t pc, double omega, int32_t* iters,
                                       double* rel_res, void* stream) {
-    return pcg_solve(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, reinterpret_cast<cudaStream_t>(stream));
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    if (!K) return DDA_ERR_ARG;
+    if (pcg_engine(K, pc) == 1) return pcg_solve(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, st);
+    if (iters) *iters = 0;
+    if (rel_res) *rel_res = 0.0;
+    if (!K || !F || !d || !(tol > 0.0) || maxit < 0) return DDA_ERR_ARG;
+    if (pc != DDA_PC_NONE && pc != DDA_PC_BJ && pc != DDA_PC_SSOR_AI) return DDA_ERR_ARG;
+    if ((pc == DDA_PC_BJ || pc == DDA_PC_SSOR_AI) && !K->dinv_valid) {
+        dda_status_t s = bj_setup(K, st, nullptr);
+        if (s != DDA_OK) return s;
+    }
+    return pcg_graph_solve(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, st);
 }
 
 extern "C" dda_status_t dda_solve_host(int32_t n, const double* kdiag, int64_t m, const int32_t* bi,
@@ -511,7 +550,7 @@ extern "C" dda_status_t dda_solve_host(int32_t n, const double* kdiag, int64_t m
     dda_matrix_t K = nullptr;
     dda_status_t s = dda_build_matrix(n, dk, m, dbi, dbj, dpen, de, dg, stream, &K);
     if (s != DDA_OK) return s;
-    s = pcg_solve(K, dF, d0 ? dd0 : nullptr, dd, tol, maxit, pc, omega, iters, rel_res, st);
+    s = dda_pcg_solve(K, dF, d0 ? dd0 : nullptr, dd, tol, maxit, pc, omega, iters, rel_res, stream);
     if (s == DDA_OK || s == DDA_ERR_NO_CONVERGENCE || s == DDA_ERR_BREAKDOWN) {
         cudaError_t ce = cudaMemcpyAsync(d, dd, sizeof(double) * N, cudaMemcpyDeviceToHost, st);
         if (ce == cudaSuccess) ce = cudaStreamSynchronize(st);
