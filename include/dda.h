@@ -51,7 +51,7 @@ typedef enum {
     DDA_PC_NONE = 0,     /* plain CG */
     DDA_PC_BJ = 1,       /* block Jacobi: z_i = D_i^{-1} r_i (Table I) */
     DDA_PC_SSOR_AI = 2,  /* SSOR approximate inverse (ref [36]; reading Z14) */
-    DDA_PC_ILU0 = 3      /* block ILU(0) = IC(0) for symmetric K (reading Z15) */
+    DDA_PC_ILU0 = 3      /* block ILU(0) = IC(0) for symmetric K (reading Z15); sync-free sweeps */
 } dda_precond_t;
 
 /*
@@ -138,7 +138,10 @@ dda_status_t dda_bj_setup(dda_matrix_t K, double *dinv, int32_t *bad_block, void
 /*
  * A7/A8 — Preconditioner application z = M^{-1} r (device [6n] each) for
  * testing the preconditioners in isolation.  Sets the preconditioner up first
- * if needed.  omega is used by DDA_PC_SSOR_AI only.  Synchronising.
+ * if needed (block-Jacobi inverses; for DDA_PC_ILU0 the block IC(0) factor
+ * U_ij = A_ij - sum_k U_ki^T U_kk^{-1} U_kj on the stored pattern, which may
+ * return DDA_ERR_NOT_SPD for a non-SPD pivot).  omega is used by
+ * DDA_PC_SSOR_AI only.  Synchronising.
  */
 dda_status_t dda_precond_apply(dda_matrix_t K, dda_precond_t pc, double omega, const double *r, double *z,
                                void *stream);

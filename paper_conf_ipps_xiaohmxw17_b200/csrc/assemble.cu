@@ -212,6 +212,7 @@ dda_status_t run_values(dda_matrix* K, const double* kdiag, const double* pen, c
     k_diag<<<grid_for((int64_t)K->n * 6), TPB, 0, st>>>(K->n, K->dstart, K->dperm, pen, e, g, kdiag, K->diag);
     DDA_LAUNCHED();
     K->dinv_valid = false;
+    K->ilu_valid = false;
     return DDA_OK;
 }
 
@@ -231,7 +232,8 @@ extern "C" void dda_matrix_free(dda_matrix_t K) {
     cudaDeviceSynchronize();   // no stream may still use the arrays
     if (K->graph_engine) pcg_graph_free(K->graph_engine);
     void* ptrs[] = {K->row_ptr, K->col_idx, K->low_ptr, K->low_row, K->low_to_up, K->urow, K->diag, K->upper,
-                    K->perm, K->seg, K->dperm, K->dstart, K->orient, K->dinv, K->ws, K->scratch};
+                    K->perm, K->seg, K->dperm, K->dstart, K->orient, K->dinv, K->ws, K->scratch,
+                    K->ilu_up, K->ilu_inv, K->ilu_flags, K->ilu_order};
     for (void* p : ptrs)
         if (p) dev_free(p);
     cudaSetDevice(prev);

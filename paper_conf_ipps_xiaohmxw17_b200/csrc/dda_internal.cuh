@@ -110,6 +110,12 @@ struct dda_matrix {
     // preconditioners
     double* dinv = nullptr;         // [n][24] packed D_i^{-1}
     bool dinv_valid = false;
+    double* ilu_up = nullptr;       // [nnzb][36] tiled: U_ij of the block IC(0) = ILU(0) factor
+    double* ilu_inv = nullptr;      // [n][36] tiled: U_ii^{-1}
+    int* ilu_flags = nullptr;       // [3n + 8]: factor / forward / backward ready flags, counters
+    int* ilu_order = nullptr;       // [2n]: forward-level schedule, backward-level schedule
+    int ilu_levels_f = 0, ilu_levels_b = 0;
+    bool ilu_valid = false;
     // PCG workspace
     double* ws = nullptr;
     size_t ws_bytes = 0;
@@ -123,6 +129,9 @@ dda_status_t ensure_workspace(dda_matrix* K, size_t bytes, cudaStream_t st);
 dda_status_t bj_setup(dda_matrix* K, cudaStream_t s, int32_t* bad_block);
 dda_status_t spmv(dda_matrix* K, const double* x, double* y, cudaStream_t s);
 void pcg_graph_free(void* g);
+dda_status_t ilu_setup(dda_matrix* K, cudaStream_t st, int32_t* bad_block);
+dda_status_t ilu_apply(dda_matrix* K, const double* r, double* z, double* y, double* yh, cudaStream_t st);
+int ilu_grid();
 dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, double* d, double tol,
                              int32_t maxit, dda_precond_t pc, double omega, int32_t* iters, double* rel_res,
                              cudaStream_t st);

@@ -1,0 +1,262 @@
+// A8 — block ILU(0) preconditioner ("ILU ... provided by
+// cuSPARSE"; Table I; reading Z15): incomplete LU without pivoting on
+// the 6x6 block pattern.  K and its pattern are symmetric, so the factor is the
+// block incomplete Cholesky in upper form and only U is stored:
+//     U_ii = A_ii - sum_{k<i, (k,i) in P}            U_ki^T U_kk^{-1} U_ki
+//     U_ij = A_ij - sum_{k<i, (k,i),(k,j) in P}      U_ki^T U_kk^{-1} U_kj      (j > i in P)
+// i.e. L_ik = U_ki^T U_kk^{-1} (the oracle computes the full-pattern IKJ LU
+// instead; tests compare the applications).  Application z = M^{-1} r:
+//     forward   y_i = r_i - sum_{k<i} U_ki^T yh_k,   yh_i = U_ii^{-1} y_i
+//     backward  z_i = U_ii^{-1} (y_i - sum_{j>i} U_ij z_j)
+//
+// GPU mapping: every phase is SYNC-FREE — one warp per block row, rows taken
+// from an atomic counter in dependency order (increasing for the factor and the
+// forward sweep, decreasing for the backward sweep), each row spinning on the
+// ready flags of the rows it depends on.  A warp only ever waits on rows that
+// were taken earlier by resident warps, so there is no deadlock; no level-set
+// analysis is needed.  The critical path is the dependency chain of the slope
+// ordering (~ courses + bricks per course), so these kernels are latency-bound,
+// as the paper observed for its triangular solves (TSS ~ 11x SpMV).
+#include <climits>
+#include <vector>
+
+#include "ilu_dev.cuh"
+
+namespace dda {
+namespace {
+
+constexpr int WPB = DDA_THREADS / 32;
+
+// ------------------------------------------------------------------ factor
+
+// per-warp 6x6 scratch in shared memory, row-major
+struct WarpMats {
+    double Uii[36], S[36], Pinv[36], W[36];
+};
+
+// C -= A * B (row-major 6x6 in shared memory), one warp; C may be global (tiled) via ctile
+__device__ __forceinline__ void mm_sub_smem(double* C, const double* A, const double* B, int lane) {
+    for (int e = lane; e < 36; e += 32) {
+        const int r = e / 6, c = e - 6 * (e / 6);
+        double s = 0.0;
+#pragma unroll
+        for (int m = 0; m < 6; ++m) s = fma(A[6 * r + m], B[6 * m + c], s);
+        C[e] -= s;
+    }
+    __syncwarp();
+}
+
+__global__ void __launch_bounds__(DDA_THREADS) k_ilu_factor(BsrView A, double* __restrict__ Fup,
+                                                            double* __restrict__ Finv, int* __restrict__ flags,
+                                                            int* __restrict__ counter, int* __restrict__ bad,
+                                                            const int* __restrict__ order) {
+    __shared__ WarpMats sm[WPB];
+    const int lane = threadIdx.x & 31;
+    WarpMats& M = sm[threadIdx.x >> 5];
+    for (int i = next_row(counter, order, A.n, lane); i < A.n; i = next_row(counter, order, A.n, lane)) {
+        // U_ii starts from A_ii
+        for (int e = lane; e < 36; e += 32) M.Uii[e] = A.diag[(size_t)kBlk * i + tile_off(e / 6, e % 6)];
+        __syncwarp();
+        const int lo0 = A.low_ptr[i], lo1 = A.low_ptr[i + 1];
+        const int up0 = A.row_ptr[i], up1 = A.row_ptr[i + 1];
+        for (int t = lo0; t < lo1; ++t) {
+            const int k = A.low_row[t];
+            const int uk = A.low_to_up[t];           // block (k, i) in the upper storage
+            if (lane == 0) wait_ready(flags, k);
+            __syncwarp();
+            for (int e = lane; e < 36; e += 32) {
+                M.S[e] = __ldcg(Fup + (size_t)kBlk * uk + tile_off(e / 6, e % 6));      // U_ki
+                M.Pinv[e] = __ldcg(Finv + (size_t)kBlk * k + tile_off(e / 6, e % 6));   // U_kk^{-1}
+            }
+            __syncwarp();
+            for (int e = lane; e < 36; e += 32) {    // W = U_ki^T U_kk^{-1}
+                const int r = e / 6, c = e - 6 * (e / 6);
+                double s = 0.0;
+#pragma unroll
+                for (int m = 0; m < 6; ++m) s = fma(M.S[6 * m + r], M.Pinv[6 * m + c], s);
+                M.W[e] = s;
+            }
+            __syncwarp();
+            mm_sub_smem(M.Uii, M.W, M.S, lane);       // U_ii -= W U_ki
+            // U_ij -= W U_kj for j in row i's pattern that is also in row k's
+            const int k0 = A.row_ptr[k], k1 = A.row_ptr[k + 1];
+            int v = k0;
+            for (int u = up0; u < up1; ++u) {
+                const int j = A.col_idx[u];
+                while (v < k1 && A.col_idx[v] < j) ++v;
+                if (v < k1 && A.col_idx[v] == j) {
+                    for (int e = lane; e < 36; e += 32) M.S[e] = __ldcg(Fup + (size_t)kBlk * v + tile_off(e / 6, e % 6));
+                    __syncwarp();
+                    for (int e = lane; e < 36; e += 32) {
+                        const int r = e / 6, c = e - 6 * (e / 6);
+                        double s = 0.0;
+#pragma unroll
+                        for (int m = 0; m < 6; ++m) s = fma(M.W[6 * r + m], M.S[6 * m + c], s);
+                        double* dst = Fup + (size_t)kBlk * u + tile_off(r, c);
+                        *dst = *dst - s;
+                    }
+                    __syncwarp();
+                }
+            }
+        }
+        // pivot inverse: symmetrise, Cholesky, inverse (lane 0, registers)
+        if (lane == 0) {
+            double P[6][6], L[6][6], Li[6][6];
+            for (int r = 0; r < 6; ++r)
+                for (int c = 0; c < 6; ++c) P[r][c] = 0.5 * (M.Uii[6 * r + c] + M.Uii[6 * c + r]);
+            bool ok = true;
+            for (int j = 0; j < 6; ++j) {
+                double d = P[j][j];
+                for (int k = 0; k < j; ++k) d -= L[j][k] * L[j][k];
+                ok = ok && d > 0.0 && isfinite(d);
+                L[j][j] = sqrt(d > 0.0 ? d : 1.0);
+                for (int r = j + 1; r < 6; ++r) {
+                    double s = P[r][j];
+                    for (int k = 0; k < j; ++k) s -= L[r][k] * L[j][k];
+                    L[r][j] = s / L[j][j];
+                }
+                for (int r = 0; r < j; ++r) L[r][j] = 0.0;
+            }
+            if (!ok) atomicMin(bad, i);
+            for (int c = 0; c < 6; ++c)
+                for (int r = 0; r < 6; ++r) {
+                    if (r < c) { Li[r][c] = 0.0; continue; }
+                    double s = (r == c) ? 1.0 : 0.0;
+                    for (int k = c; k < r; ++k) s -= L[r][k] * Li[k][c];
+                    Li[r][c] = s / L[r][r];
+                }
+            for (int r = 0; r < 6; ++r)
+                for (int c = 0; c < 6; ++c) {
+                    double s = 0.0;
+                    for (int k = (r > c ? r : c); k < 6; ++k) s += Li[k][r] * Li[k][c];
+                    Finv[(size_t)kBlk * i + tile_off(r, c)] = s;
+                }
+            __threadfence();
+            st_release(flags + i, 1);
+        }
+        __syncwarp();
+    }
+}
+
+__global__ void __launch_bounds__(DDA_THREADS) k_ilu_fwd(BsrView A, const double* Fup, const double* Finv,
+                                                         const double* r, double* y, double* yh, int* flags,
+                                                         int* counter, const int* order) {
+    ilu_forward_rows(A, Fup, Finv, r, y, yh, flags, counter, order);
+}
+
+__global__ void __launch_bounds__(DDA_THREADS) k_ilu_bwd(BsrView A, const double* Fup, const double* Finv,
+                                                         const double* y, double* z, const double* r, int* flags,
+                                                         int* counter, const int* order) {
+    ilu_backward_rows(A, Fup, Finv, y, z, r, nullptr, flags, counter, order);
+}
+
+}  // namespace
+
+int ilu_grid() {
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_ilu_fwd, DDA_THREADS, 0);
+    if (per_sm < 1) per_sm = 1;
+    // rows are taken in dependency order by warps that are already running, so the
+    // sync-free scheme needs no co-residency; one full wave is enough parallelism
+    return device_sms() * per_sm;
+}
+
+// Analysis (once per structure, like a triangular-solve analysis phase): the
+// dependency levels of the forward DAG (row i after every k < i with (k,i)
+// stored) and of the backward DAG (row i after every j > i with (i,j) stored),
+// and the two schedules = rows sorted by level (stable).  Host C++, O(n + nnzb).
+static dda_status_t ilu_schedule(dda_matrix* K, cudaStream_t st) {
+    const int32_t n = K->n;
+    const int64_t z = K->nnzb;
+    std::vector<int32_t> row_ptr(n + 1), col(z), low_ptr(n + 1), low_row(z);
+    DDA_CK(cudaMemcpyAsync(row_ptr.data(), K->row_ptr, sizeof(int32_t) * (n + 1), cudaMemcpyDeviceToHost, st));
+    DDA_CK(cudaMemcpyAsync(low_ptr.data(), K->low_ptr, sizeof(int32_t) * (n + 1), cudaMemcpyDeviceToHost, st));
+    if (z) {
+        DDA_CK(cudaMemcpyAsync(col.data(), K->col_idx, sizeof(int32_t) * z, cudaMemcpyDeviceToHost, st));
+        DDA_CK(cudaMemcpyAsync(low_row.data(), K->low_row, sizeof(int32_t) * z, cudaMemcpyDeviceToHost, st));
+    }
+    DDA_CK(cudaStreamSynchronize(st));
+    std::vector<int32_t> lev(n), order(2 * (size_t)n);
+    auto sort_by_level = [&](int32_t* out) {
+        int32_t maxl = 0;
+        for (int32_t i = 0; i < n; ++i) maxl = lev[i] > maxl ? lev[i] : maxl;
+        std::vector<int32_t> cnt(maxl + 2, 0);
+        for (int32_t i = 0; i < n; ++i) ++cnt[lev[i] + 1];
+        for (int32_t l = 0; l <= maxl; ++l) cnt[l + 1] += cnt[l];
+        for (int32_t i = 0; i < n; ++i) out[cnt[lev[i]]++] = i;
+        return maxl + 1;
+    };
+    for (int32_t i = 0; i < n; ++i) {            // forward levels
+        int32_t l = 0;
+        for (int32_t t = low_ptr[i]; t < low_ptr[i + 1]; ++t) l = lev[low_row[t]] + 1 > l ? lev[low_row[t]] + 1 : l;
+        lev[i] = l;
+    }
+    K->ilu_levels_f = sort_by_level(order.data());
+    for (int32_t i = n - 1; i >= 0; --i) {       // backward levels
+        int32_t l = 0;
+        for (int32_t u = row_ptr[i]; u < row_ptr[i + 1]; ++u) l = lev[col[u]] + 1 > l ? lev[col[u]] + 1 : l;
+        lev[i] = l;
+    }
+    // (lev[] now holds backward levels; forward values of higher rows were already consumed)
+    K->ilu_levels_b = sort_by_level(order.data() + n);
+    DDA_CK(cudaMemcpyAsync(K->ilu_order, order.data(), sizeof(int32_t) * 2 * (size_t)n, cudaMemcpyHostToDevice, st));
+    DDA_CK(cudaStreamSynchronize(st));
+    return DDA_OK;
+}
+
+dda_status_t ilu_setup(dda_matrix* K, cudaStream_t st, int32_t* bad_block) {
+    if (bad_block) *bad_block = -1;
+    const size_t n = (size_t)K->n;
+    if (!K->ilu_up) {
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->ilu_up), (K->nnzb ? K->nnzb : 1) * kBlk * sizeof(double), st));
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->ilu_inv), n * kBlk * sizeof(double), st));
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->ilu_flags), (3 * n + 8) * sizeof(int), st));
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->ilu_order), 2 * n * sizeof(int), st));
+        dda_status_t s = ilu_schedule(K, st);
+        if (s != DDA_OK) return s;
+    }
+    if (K->nnzb)
+        DDA_CK(cudaMemcpyAsync(K->ilu_up, K->upper, K->nnzb * kBlk * sizeof(double), cudaMemcpyDeviceToDevice, st));
+    int* flags = K->ilu_flags;
+    int* counter = K->ilu_flags + 3 * n;
+    int* bad = counter + 1;
+    DDA_CK(cudaMemsetAsync(flags, 0, n * sizeof(int), st));
+    DDA_CK(cudaMemsetAsync(counter, 0, sizeof(int), st));
+    const int big = INT_MAX;
+    DDA_CK(cudaMemcpyAsync(bad, &big, sizeof(int), cudaMemcpyHostToDevice, st));
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_ilu_factor, DDA_THREADS, 0);
+    const int g = device_sms() * (per_sm > 0 ? per_sm : 1);
+    k_ilu_factor<<<g, DDA_THREADS, 0, st>>>(view_of(K), K->ilu_up, K->ilu_inv, flags, counter, bad, K->ilu_order);
+    DDA_LAUNCHED();
+    int hbad = 0;
+    DDA_CK(cudaMemcpyAsync(&hbad, bad, sizeof(int), cudaMemcpyDeviceToHost, st));
+    DDA_CK(cudaStreamSynchronize(st));
+    if (hbad != INT_MAX) {
+        if (bad_block) *bad_block = hbad;
+        K->ilu_valid = false;
+        return DDA_ERR_NOT_SPD;
+    }
+    K->ilu_valid = true;
+    return DDA_OK;
+}
+
+// standalone application z = M^{-1} r (y, yh: device scratch of 6n each)
+dda_status_t ilu_apply(dda_matrix* K, const double* r, double* z, double* y, double* yh, cudaStream_t st) {
+    const size_t n = (size_t)K->n;
+    int* fl_f = K->ilu_flags + n;
+    int* fl_b = K->ilu_flags + 2 * n;
+    int* counters = K->ilu_flags + 3 * n + 2;
+    DDA_CK(cudaMemsetAsync(fl_f, 0, 2 * n * sizeof(int), st));
+    DDA_CK(cudaMemsetAsync(counters, 0, 2 * sizeof(int), st));
+    const int g = ilu_grid();
+    k_ilu_fwd<<<g, DDA_THREADS, 0, st>>>(view_of(K), K->ilu_up, K->ilu_inv, r, y, yh, fl_f, counters,
+                                         K->ilu_order);
+    DDA_LAUNCHED();
+    k_ilu_bwd<<<g, DDA_THREADS, 0, st>>>(view_of(K), K->ilu_up, K->ilu_inv, y, z, r, fl_b, counters + 1,
+                                         K->ilu_order + n);
+    DDA_LAUNCHED();
+    return DDA_OK;
+}
+
+}  // namespace dda

@@ -491,6 +491,7 @@ static int pcg_engine(const dda_matrix* K, dda_precond_t pc) {   // 0 = graph, 1
         const char* v = getenv("DDA_PCG_ENGINE");
         forced = !v ? -1 : ((v[0] == 'p' || v[0] == '1') ? 1 : 0);
     }
+    if (pc == DDA_PC_ILU0) return 0;   // the sync-free ILU sweeps exist in the graph engine only
     if (forced >= 0) return forced;
     return (pc != DDA_PC_SSOR_AI && K->n < 65536) ? 1 : 0;
 }
@@ -504,9 +505,13 @@ extern "C" dda_status_t dda_pcg_solve(dda_matrix_t K, const double* F, const dou
     if (iters) *iters = 0;
     if (rel_res) *rel_res = 0.0;
     if (!K || !F || !d || !(tol > 0.0) || maxit < 0) return DDA_ERR_ARG;
-    if (pc != DDA_PC_NONE && pc != DDA_PC_BJ && pc != DDA_PC_SSOR_AI) return DDA_ERR_ARG;
+    if (pc != DDA_PC_NONE && pc != DDA_PC_BJ && pc != DDA_PC_SSOR_AI && pc != DDA_PC_ILU0) return DDA_ERR_ARG;
     if ((pc == DDA_PC_BJ || pc == DDA_PC_SSOR_AI) && !K->dinv_valid) {
         dda_status_t s = bj_setup(K, st, nullptr);
+        if (s != DDA_OK) return s;
+    }
+    if (pc == DDA_PC_ILU0 && !K->ilu_valid) {
+        dda_status_t s = ilu_setup(K, st, nullptr);
         if (s != DDA_OK) return s;
     }
     return pcg_graph_solve(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, st);

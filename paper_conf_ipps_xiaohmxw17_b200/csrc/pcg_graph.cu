@@ -20,7 +20,7 @@
 #include <cmath>
 #include <cstdlib>
 
-#include "precond_dev.cuh"
+#include "ilu_dev.cuh"
 
 namespace dda {
 namespace {
@@ -52,6 +52,12 @@ struct GArgs {           // constant for a (matrix, preconditioner): baked into 
     State* st;
     const CallArgs* ca;
     int* out;            // iters, status, rel (double at +8 bytes)
+    const double* ilu_up;
+    const double* ilu_inv;
+    int* ilu_flags_f;    // forward / backward ready flags and their row counters
+    int* ilu_flags_b;
+    int* ilu_counters;
+    const int* ilu_order;
     int use_cond;        // 0 only for the internal phase-timing hook (kernels launched outside the graph)
 };
 
@@ -221,7 +227,7 @@ __global__ void __launch_bounds__(DDA_THREADS) k_g_update(const GArgs a, cudaGra
         if (R.valid) {
             if (a.pc == DDA_PC_SSOR_AI) {
                 a.t[R.idx] = tz;
-            } else {
+            } else if (a.pc != DDA_PC_ILU0) {
                 a.z[R.idx] = tz;
                 rz += rv * tz;
             }
@@ -237,7 +243,7 @@ __global__ void __launch_bounds__(DDA_THREADS) k_g_update(const GArgs a, cudaGra
             st->k = k + 1;
             st->done = 1;
             set_cond(a, h, 0);
-        } else if (a.pc != DDA_PC_SSOR_AI) {
+        } else if (a.pc != DDA_PC_SSOR_AI && a.pc != DDA_PC_ILU0) {
             finish_iteration(a, tot[1], h);
         }
     }
@@ -283,6 +289,30 @@ __global__ void __launch_bounds__(DDA_THREADS) k_g_ssor_upper(const GArgs a, cud
     }
 }
 
+// ILU(0) sweeps (sync-free, ilu.cu): y = t, yh = w scratch; z (and p0 at setup); rz -> beta / rho
+template <bool INIT>
+__global__ void __launch_bounds__(DDA_THREADS) k_g_ilu_fwd(const GArgs a) {
+    if (loop_done(a.st)) return;
+    ilu_forward_rows(a.A, a.ilu_up, a.ilu_inv, a.r, a.t, a.w, a.ilu_flags_f, a.ilu_counters, a.ilu_order);
+}
+
+template <bool INIT>
+__global__ void __launch_bounds__(DDA_THREADS) k_g_ilu_bwd(const GArgs a, cudaGraphConditionalHandle h) {
+    if (loop_done(a.st)) return;
+    const double rz = ilu_backward_rows(a.A, a.ilu_up, a.ilu_inv, a.t, a.z, a.r, INIT ? a.p0 : nullptr,
+                                        a.ilu_flags_b, a.ilu_counters + 1, a.ilu_order + a.A.n);
+    double v[1] = {rz}, tot[1];
+    if (grid_reduce_last<1>(a, v, tot) && threadIdx.x == 0) {
+        if (INIT) {
+            State* st = a.st;
+            st->rho = tot[0];
+            if (!(tot[0] > 0.0) || !isfinite(tot[0])) { st->status = DDA_ERR_BREAKDOWN; st->done = 1; }
+        } else {
+            finish_iteration(a, tot[0], h);
+        }
+    }
+}
+
 // ---------------------------------------------------------------- prelude / epilogue
 
 // d = d0 (or 0), r = F - q (or F); BJ/none: z = p0 = M^{-1} r; SSOR: t = D^{-1} r;
@@ -311,7 +341,7 @@ __global__ void __launch_bounds__(DDA_THREADS) k_g_init(const GArgs a) {
         if (R.valid) {
             if (a.pc == DDA_PC_SSOR_AI) {
                 a.t[R.idx] = tz;
-            } else {
+            } else if (a.pc != DDA_PC_ILU0) {
                 a.z[R.idx] = tz;
                 a.p0[R.idx] = tz;
                 rz += rv * tz;
@@ -337,7 +367,7 @@ __global__ void __launch_bounds__(DDA_THREADS) k_g_init(const GArgs a) {
             st->zero_d = 1; st->status = DDA_OK; st->done = 1;
         } else if (sqrt(tot[1]) <= ca->tol * st->bnorm) {
             st->status = DDA_OK; st->done = 1;
-        } else if (a.pc != DDA_PC_SSOR_AI && (!(tot[2] > 0.0) || !isfinite(tot[2]))) {
+        } else if (a.pc != DDA_PC_SSOR_AI && a.pc != DDA_PC_ILU0 && (!(tot[2] > 0.0) || !isfinite(tot[2]))) {
             st->status = DDA_ERR_BREAKDOWN; st->done = 1;
         } else if (ca->maxit <= 0) {
             st->status = DDA_ERR_NO_CONVERGENCE; st->done = 1;
@@ -403,7 +433,7 @@ struct PcgGraph {
     cudaGraphExec_t exec = nullptr;
     cudaGraph_t graph = nullptr;
     cudaGraphConditionalHandle h = 0;
-    int G_spmv = 0, G_vec = 0;
+    int G_spmv = 0, G_vec = 0, g_ilu = 0;
 };
 
 void pcg_graph_free(void* p) {
@@ -430,7 +460,8 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         const int need_vec = ((K->n + 4) / 5 + WPB - 1) / WPB;
         int g_vec = occ_grid((const void*)k_g_update, 8);
         if (g_vec > need_vec) g_vec = need_vec > 0 ? need_vec : 1;
-        const int Gmax = g_spmv > g_vec ? g_spmv : g_vec;
+        int Gmax = g_spmv > g_vec ? g_spmv : g_vec;
+        if (ilu_grid() > Gmax) Gmax = ilu_grid();
         const size_t bytes = (7 * N + 3 * (size_t)Gmax) * sizeof(double) + sizeof(CallArgs) + sizeof(State) + 64;
         // may reallocate the workspace (and drop any engine holding the old pointers): do it first
         dda_status_t s = ensure_workspace(K, bytes, st);
@@ -453,6 +484,13 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         a.pc = (int)pc;
         a.out = reinterpret_cast<int*>(reinterpret_cast<char*>(K->scratch) + 128);
         a.use_cond = 1;
+        a.ilu_up = K->ilu_up;
+        a.ilu_inv = K->ilu_inv;
+        a.ilu_flags_f = K->ilu_flags ? K->ilu_flags + K->n : nullptr;
+        a.ilu_flags_b = K->ilu_flags ? K->ilu_flags + 2 * (size_t)K->n : nullptr;
+        a.ilu_counters = K->ilu_flags ? K->ilu_flags + 3 * (size_t)K->n + 2 : nullptr;
+        a.ilu_order = K->ilu_order;
+        G->g_ilu = ilu_grid();
         DDA_CK(cudaMemsetAsync(a.st, 0, sizeof(State), st));       // ticket = 0
 
         // ---- the loop: a while conditional node whose body is captured from a stream
@@ -474,6 +512,11 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         if (pc == DDA_PC_SSOR_AI) {
             k_g_ssor_lower<false><<<G->G_spmv, DDA_THREADS, 0, cs>>>(a);
             k_g_ssor_upper<false><<<G->G_spmv, DDA_THREADS, 0, cs>>>(a, G->h);
+        } else if (pc == DDA_PC_ILU0) {
+            cudaMemsetAsync(a.ilu_flags_f, 0, 2 * (size_t)K->n * sizeof(int), cs);
+            cudaMemsetAsync(a.ilu_counters, 0, 2 * sizeof(int), cs);
+            k_g_ilu_fwd<false><<<G->g_ilu, DDA_THREADS, 0, cs>>>(a);
+            k_g_ilu_bwd<false><<<G->g_ilu, DDA_THREADS, 0, cs>>>(a, G->h);
         }
         cudaError_t ce = cudaStreamEndCapture(cs, nullptr);
         cudaStreamDestroy(cs);
@@ -495,6 +538,13 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         k_g_ssor_lower<true><<<G->G_spmv, DDA_THREADS, 0, st>>>(a);
         DDA_LAUNCHED();
         k_g_ssor_upper<true><<<G->G_spmv, DDA_THREADS, 0, st>>>(a, G->h);
+        DDA_LAUNCHED();
+    } else if (pc == DDA_PC_ILU0) {
+        DDA_CK(cudaMemsetAsync(a.ilu_flags_f, 0, 2 * (size_t)K->n * sizeof(int), st));
+        DDA_CK(cudaMemsetAsync(a.ilu_counters, 0, 2 * sizeof(int), st));
+        k_g_ilu_fwd<true><<<G->g_ilu, DDA_THREADS, 0, st>>>(a);
+        DDA_LAUNCHED();
+        k_g_ilu_bwd<true><<<G->g_ilu, DDA_THREADS, 0, st>>>(a, G->h);
         DDA_LAUNCHED();
     }
     // ---- the device-side loop (counted as one launch; each iteration runs 2 (BJ) or 4 (SSOR) kernels)

@@ -168,6 +168,18 @@ extern "C" dda_status_t dda_precond_apply(dda_matrix_t K, dda_precond_t pc, doub
         DDA_CK(cudaStreamSynchronize(st));
         return DDA_OK;
     }
+    if (pc == DDA_PC_ILU0) {
+        if (!K->ilu_valid) {
+            dda_status_t s = ilu_setup(K, st, nullptr);
+            if (s != DDA_OK) return s;
+        }
+        dda_status_t ws = ensure_workspace(K, 2 * N * sizeof(double), st);
+        if (ws != DDA_OK) return ws;
+        dda_status_t s = ilu_apply(K, r, z, K->ws, K->ws + N, st);
+        if (s != DDA_OK) return s;
+        DDA_CK(cudaStreamSynchronize(st));
+        return DDA_OK;
+    }
     if (pc != DDA_PC_BJ && pc != DDA_PC_SSOR_AI) return DDA_ERR_ARG;
     if (!K->dinv_valid) {
         dda_status_t s = bj_setup(K, st, nullptr);
