@@ -178,6 +178,46 @@ dda_status_t dda_solve_host(int32_t n_blocks, const double *kdiag, int64_t n_spr
                             const double *F, const double *d0, double *d, double tol, int32_t maxit,
                             dda_precond_t pc, double omega, int32_t *iters, double *rel_res, void *stream);
 
+/*
+ * (e) — Multi-GPU block-row partitioned PCG (beyond the paper: multi-GPU is its
+ * future work).  A partition is an ordinary dda_matrix_t built on the
+ * partition's LOCAL numbering: own rows 0..n_own-1 (a contiguous range of
+ * global rows, same order) followed by halo rows grouped by owning peer
+ * (ascending peer, global order within a peer); it is assembled from every
+ * spring that touches an own row, so its own rows are exact global rows.
+ * (paper_conf_ipps_xiaohmxw17_b200/partition.py builds these inputs.)
+ *
+ * Transports: NCCL (dda_comm_init: one partition per process / GPU; rank 0
+ * creates the 128-byte id with dda_comm_unique_id and the caller broadcasts it)
+ * or LOOPBACK (dda_comm_init_loopback: all partitions in this process on the
+ * current GPU — the same partitioned algorithm, exchanges by device copy).
+ *
+ * dda_dist_attach: partition `part` (0 for NCCL; 0..nparts-1 for loopback) is
+ * matrix K with n_own own rows; send_counts[q] own rows go to peer q, listed
+ * (local ids, host) in send_idx concatenated by peer, in the peer's halo order;
+ * recv_counts[q] halo rows come from q (sum = K's rows - n_own).  Host arrays
+ * [nranks].  K must outlive the communicator's use of it.
+ *
+ * dda_pcg_solve_dist: F[p], d0[p] (entry or whole array may be NULL), d[p]:
+ * device [6 n_own] per local partition (one entry for NCCL).  Same stop rule,
+ * statuses and reported TRUE residual as dda_pcg_solve; DDA_PC_BJ or
+ * DDA_PC_NONE (SSOR-AI and ILU(0) are single-GPU only).  Per iteration: one
+ * halo exchange of p, the symmetric SpMV over own rows, two allreduces
+ * (p^T q; r^T r and r^T z).  Synchronising.  dda_spmv_dist: y = K x over own
+ * rows (x, y device [6 n_own] per partition).
+ */
+typedef struct dda_comm *dda_comm_t;
+dda_status_t dda_comm_unique_id(void *id128);
+dda_status_t dda_comm_init(int32_t nranks, int32_t rank, const void *id128, dda_comm_t *out);
+dda_status_t dda_comm_init_loopback(int32_t nparts, dda_comm_t *out);
+dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t K, int32_t n_own, const int32_t *send_counts,
+                             const int32_t *send_idx, const int32_t *recv_counts, void *stream);
+dda_status_t dda_spmv_dist(dda_comm_t c, const double *const *x_own, double *const *y_own, void *stream);
+dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double *const *F, const double *const *d0, double *const *d,
+                                double tol, int32_t maxit, dda_precond_t pc, int32_t *iters, double *rel_res,
+                                void *stream);
+void dda_comm_free(dda_comm_t c);
+
 /* Number of kernel launches the library has issued in this process (for the
  * benchmark's gpu_launches count). */
 int64_t dda_launch_count(void);

@@ -25,7 +25,9 @@ PRECOND = {"none": 0, "bj": 1, "ssor_ai": 2, "ilu0": 3}
 # symbols declared in include/dda.h (checked by tests/test_abi.py)
 ABI_SYMBOLS = ("dda_build_matrix", "dda_update_values", "dda_matrix_info", "dda_matrix_export", "dda_spmv",
                "dda_bj_setup", "dda_precond_apply", "dda_pcg_solve", "dda_solve_host", "dda_launch_count",
-               "dda_matrix_free", "dda_status_string", "dda_last_cuda_error")
+               "dda_matrix_free", "dda_status_string", "dda_last_cuda_error", "dda_comm_unique_id",
+               "dda_comm_init", "dda_comm_init_loopback", "dda_dist_attach", "dda_spmv_dist",
+               "dda_pcg_solve_dist", "dda_comm_free")
 
 _lib = None
 
@@ -74,6 +76,20 @@ def lib() -> C.CDLL:
         L.dda_status_string.restype = C.c_char_p
         L.dda_last_cuda_error.argtypes = []
         L.dda_last_cuda_error.restype = C.c_char_p
+        L.dda_comm_unique_id.argtypes = [P]
+        L.dda_comm_unique_id.restype = st
+        L.dda_comm_init.argtypes = [I32, I32, P, C.POINTER(P)]
+        L.dda_comm_init.restype = st
+        L.dda_comm_init_loopback.argtypes = [I32, C.POINTER(P)]
+        L.dda_comm_init_loopback.restype = st
+        L.dda_dist_attach.argtypes = [P, I32, P, I32, P, P, P, P]
+        L.dda_dist_attach.restype = st
+        L.dda_spmv_dist.argtypes = [P, P, P, P]
+        L.dda_spmv_dist.restype = st
+        L.dda_pcg_solve_dist.argtypes = [P, P, P, P, D, I32, st, C.POINTER(I32), C.POINTER(D), P]
+        L.dda_pcg_solve_dist.restype = st
+        L.dda_comm_free.argtypes = [P]
+        L.dda_comm_free.restype = None
         _lib = L
     return _lib
 
@@ -250,3 +266,84 @@ def solve_host(kdiag, bi, bj, pen, e, g, F, d0=None, tol=1e-10, maxit=10000, pre
     if st not in (OK, ERR_NO_CONVERGENCE, ERR_BREAKDOWN):
         raise DDAError(st, "dda_solve_host")
     return out, int(it.value), float(rr.value), int(st)
+
+
+# ----------------------------------------------------------------------------- multi-GPU (§8(e))
+
+class Comm:
+    """Partitioned-solve communicator: NCCL (one partition per process / GPU) or
+    loopback (all partitions in this process, for single-GPU testing)."""
+
+    def __init__(self, handle, nparts_local: int):
+        self._h = handle
+        self.nparts_local = nparts_local
+        self.parts = [None] * nparts_local     # (Matrix, LocalProblem) kept alive
+
+    @staticmethod
+    def unique_id() -> bytes:
+        buf = C.create_string_buffer(128)
+        _check(lib().dda_comm_unique_id(buf), "dda_comm_unique_id")
+        return buf.raw
+
+    @classmethod
+    def nccl(cls, nranks: int, rank: int, uid: bytes) -> "Comm":
+        h = C.c_void_p()
+        buf = C.create_string_buffer(uid, 128)
+        _check(lib().dda_comm_init(int(nranks), int(rank), buf, C.byref(h)), "dda_comm_init")
+        return cls(h, 1)
+
+    @classmethod
+    def loopback(cls, nparts: int) -> "Comm":
+        h = C.c_void_p()
+        _check(lib().dda_comm_init_loopback(int(nparts), C.byref(h)), "dda_comm_init_loopback")
+        return cls(h, nparts)
+
+    def attach(self, part: int, K: "Matrix", lp, stream=None):
+        sc = np.ascontiguousarray(lp.send_counts, np.int32)
+        si = np.ascontiguousarray(lp.send_idx, np.int32)
+        rc = np.ascontiguousarray(lp.recv_counts, np.int32)
+        _check(lib().dda_dist_attach(self._h, int(part), K.handle, int(lp.n_own), sc.ctypes.data_as(C.c_void_p),
+                                     si.ctypes.data_as(C.c_void_p), rc.ctypes.data_as(C.c_void_p),
+                                     C.c_void_p(_stream(stream))), "dda_dist_attach")
+        self.parts[part if self.nparts_local > 1 else 0] = (K, lp)
+
+    @staticmethod
+    def _ptrs(ts):
+        arr = (C.c_void_p * len(ts))(*[C.c_void_p(t.data_ptr()) if t is not None else None for t in ts])
+        return arr
+
+    def spmv(self, xs, stream=None):
+        torch = _torch()
+        ys = [torch.empty_like(x) for x in xs]
+        _check(lib().dda_spmv_dist(self._h, self._ptrs(xs), self._ptrs(ys), C.c_void_p(_stream(stream))),
+               "dda_spmv_dist")
+        return ys
+
+    def pcg_solve(self, Fs, d0s=None, tol=1e-10, maxit=10000, precond="bj", stream=None):
+        torch = _torch()
+        ds = [torch.empty_like(F) for F in Fs]
+        it, rr = C.c_int32(), C.c_double()
+        st = lib().dda_pcg_solve_dist(self._h, self._ptrs(Fs), self._ptrs(d0s) if d0s is not None else None,
+                                      self._ptrs(ds), float(tol), int(maxit), PRECOND[precond], C.byref(it),
+                                      C.byref(rr), C.c_void_p(_stream(stream)))
+        if st not in (OK, ERR_NO_CONVERGENCE, ERR_BREAKDOWN):
+            raise DDAError(st, "dda_pcg_solve_dist")
+        return ds, int(it.value), float(rr.value), int(st)
+
+    def free(self):
+        if self._h is not None and _lib is not None:
+            _lib.dda_comm_free(self._h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def build_local(lp, device="cuda") -> Matrix:
+    """Assemble a partition's local matrix (partition.LocalProblem) on the device."""
+    torch = _torch()
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(device)
+    return build_matrix(t(lp.kdiag), t(lp.bi), t(lp.bj), t(lp.pen), t(lp.e), t(lp.g))

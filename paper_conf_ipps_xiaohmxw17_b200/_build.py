@@ -19,6 +19,16 @@ NVCC_FLAGS = [
 ]
 
 
+def nccl_dirs():
+    """Torch's bundled NCCL (the process must load a single NCCL: link the same one)."""
+    try:
+        import nvidia.nccl
+        base = list(nvidia.nccl.__path__)[0]
+    except Exception:  # pragma: no cover
+        base = "/usr"
+    return os.path.join(base, "include"), os.path.join(base, "lib")
+
+
 def sources():
     return sorted(glob.glob(os.path.join(CSRC, "*.cu")))
 
@@ -38,7 +48,9 @@ def build(force: bool = False, verbose: bool = False, extra=()) -> str:
     if not force and not needs_build():
         return LIB
     nvcc = os.environ.get("NVCC", "nvcc")
-    cmd = [nvcc, *NVCC_FLAGS, *extra, "-I", INCLUDE, "-I", CSRC, *sources(), "-o", LIB + ".tmp"]
+    ninc, nlib = nccl_dirs()
+    cmd = [nvcc, *NVCC_FLAGS, *extra, "-I", INCLUDE, "-I", CSRC, "-I", ninc, *sources(), "-o", LIB + ".tmp",
+           "-L", nlib, "-l:libnccl.so.2", "-Xlinker", "-rpath=" + nlib]
     if verbose:
         print(" ".join(cmd))
     subprocess.check_call(cmd)

@@ -125,15 +125,15 @@ int grid_rows(int rows_per_warp, int n) {
 
 }  // namespace
 
-dda_status_t bj_setup(dda_matrix* K, cudaStream_t st, int32_t* bad_block, double* full) {
+static dda_status_t bj_setup_n(dda_matrix* K, int32_t nrows, cudaStream_t st, int32_t* bad_block, double* full) {
     if (bad_block) *bad_block = -1;
     int* bad = reinterpret_cast<int*>(K->scratch);
     const int big = INT_MAX;
     DDA_CK(cudaMemcpyAsync(bad, &big, sizeof(int), cudaMemcpyHostToDevice, st));
-    int g = (K->n + 127) / 128;
+    int g = (nrows + 127) / 128;
     const int cap = device_sms() * 16;
     if (g > cap) g = cap;
-    k_bj_inv<<<g, 128, 0, st>>>(K->n, K->diag, K->dinv, full, bad);
+    k_bj_inv<<<g, 128, 0, st>>>(nrows, K->diag, K->dinv, full, bad);
     DDA_LAUNCHED();
     int hbad = 0;
     DDA_CK(cudaMemcpyAsync(&hbad, bad, sizeof(int), cudaMemcpyDeviceToHost, st));
@@ -143,11 +143,18 @@ dda_status_t bj_setup(dda_matrix* K, cudaStream_t st, int32_t* bad_block, double
         K->dinv_valid = false;
         return DDA_ERR_NOT_SPD;
     }
-    K->dinv_valid = true;
+    K->dinv_valid = nrows == K->n;
     return DDA_OK;
 }
 
+dda_status_t bj_setup(dda_matrix* K, cudaStream_t st, int32_t* bad_block, double* full) {
+    return bj_setup_n(K, K->n, st, bad_block, full);
+}
 dda_status_t bj_setup(dda_matrix* K, cudaStream_t st, int32_t* bad_block) { return bj_setup(K, st, bad_block, nullptr); }
+// block-Jacobi inverses of the first nrows blocks only (the own rows of a partition)
+dda_status_t bj_setup_rows(dda_matrix* K, int32_t nrows, cudaStream_t st, int32_t* bad_block) {
+    return bj_setup_n(K, nrows, st, bad_block, nullptr);
+}
 
 }  // namespace dda
 
