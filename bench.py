@@ -49,6 +49,21 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def traffic_for(n_blocks: int, which: str):
+    """DRAM bytes per launch from the committed ncu --set full capture of the same
+    workload (profiles/traffic.json), or None."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        with open(p) as f:
+            t = json.load(f)
+        if int(t.get("n_blocks", -1)) != n_blocks:
+            return None
+        e = t[which]
+        return {"bytes": e["traffic_bytes_per_launch"], "source": e["source"]}
+    except Exception:
+        return None
+
+
 def bytes_per_row_spmv(u: float) -> float:
     """Algorithmic bytes of one symmetric SpMV per block row:
     D 288 + u*(V 288 + col 4 + low_row 4 + low_to_up 4) + row_ptr/low_ptr 8 + x 48 + y 48."""
@@ -223,10 +238,10 @@ def main():
     import paper_conf_ipps_xiaohmxw17_b200 as dda
     from synth import make_slope, preset
 
-    if world > 1:
-        raise SystemExit("row-partitioned multi-GPU solve: not in this build yet (DESIGN.md §7)")
-
     P = make_slope(preset(args.blocks, seed=1005))
+    if world > 1:
+        run_dist(args, P, world, rank, local)
+        return
     t = dda.problem_to_device(P)
     stream = torch.cuda.current_stream()
     hbm_peak, peak_src = measured_peaks()
@@ -340,11 +355,12 @@ def main():
                    "step": "dda_build_matrix + dda_bj_setup + dda_pcg_solve"},
         "phases_ms": {"assemble": ph_build, "bj_setup": ph_bj, "pcg": pcg_ms, "pcg_iters": iters,
                       "pcg_us_per_iter": 1000.0 * pcg_ms / max(iters, 1), "true_rel_res": rel_res},
-        "roofline": {"kernel": "k_pcg (persistent PCG: SpMV + fused vector phases)", "bound": "hbm",
-                     "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
-                     "traffic": None, "peak_source": peak_src,
+        "roofline": {"kernel": "dda_pcg_solve: one CUDA-graph while loop (k_g_spmv + k_g_update per "
+                               "iteration) with its prelude/epilogue kernels",
+                     "bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
+                     "traffic": traffic_for(n, "pcg"), "peak_source": peak_src,
                      "algorithmic_bytes_per_launch": pcg_bytes},
-        "spmv": {"kernel": "k_spmv<FULL>", "ms": spmv_ms, "gbs": spmv_gbs, "frac_hbm": spmv_gbs / hbm_peak,
+        "spmv": {"kernel": "k_spmv<FULL,6>", "ms": spmv_ms, "traffic": traffic_for(n, "spmv"), "gbs": spmv_gbs, "frac_hbm": spmv_gbs / hbm_peak,
                  "gflops": n * (72 + 144 * u) / (spmv_ms * 1e-3) / 1e9, "bytes": spmv_bytes,
                  "timing": "back to back (hot), inputs > L2"},
         "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": int(launches),
@@ -354,6 +370,107 @@ def main():
         print(json.dumps(line), flush=True)
     if world > 1:
         torch.distributed.destroy_process_group()
+
+
+def run_dist(args, P, world, rank, local):
+    """N > 1: block-row partitioned BJ-PCG over NCCL.  One step per
+    rank = assemble the local matrix (springs touching own rows) + distributed
+    PCG to 1e-10; value = max over ranks of the device time."""
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ipps_xiaohmxw17_b200 as dda
+    from paper_conf_ipps_xiaohmxw17_b200.partition import row_bounds, local_from_slope
+
+    bounds = row_bounds(P.n, world)
+    lp = local_from_slope(P, bounds, rank)
+    dev = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    t = {k: dev(getattr(lp, k)) for k in ("kdiag", "bi", "bj", "pen", "e", "g", "F")}
+    obj = [dda.Comm.unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=0)
+    comm = dda.Comm.nccl(world, rank, obj[0])
+    stream = torch.cuda.current_stream()
+    hbm_peak, peak_src = measured_peaks()
+
+    def step(ev=None):
+        if ev: ev[0].record(stream)
+        K = dda.build_matrix(t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+        comm.attach(0, K, lp)
+        if ev: ev[1].record(stream)
+        ds, it, rr, st = comm.pcg_solve([t["F"]], tol=1e-10, maxit=10000, precond=args.precond)
+        if ev: ev[2].record(stream)
+        return K, it, rr, st
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    evs = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    start, stop = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    l0 = dda.launch_count()
+    dist.barrier()
+    torch.cuda.synchronize()
+    res = []
+    with ClockSampler(local) as clk:
+        start.record(stream)
+        for k in range(args.steps):
+            res.append(step(evs[k]))
+        stop.record(stream)
+        torch.cuda.synchronize()
+    dist.barrier()
+    launches = dda.launch_count() - l0
+    ms = start.elapsed_time(stop) / args.steps
+    asm = statistics.median(e[0].elapsed_time(e[1]) for e in evs)
+    pcg = statistics.mean(e[1].elapsed_time(e[2]) for e in evs)
+    K, iters, rel_res, status = res[-1]
+    assert status == dda.OK and rel_res <= 1.01e-10, (status, rel_res)
+    u = K.nnzb / max(lp.n_local, 1)
+    local_bytes = lp.n_own * (bytes_per_row_spmv(u) + 672.0) * iters
+    ach = local_bytes / (pcg * 1e-3) / 1e9
+    tt = torch.tensor([ms, pcg, asm], device="cuda")
+    dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    ms, pcg_max, asm_max = (float(v) for v in tt.tolist())
+    # e2e: pinned host local inputs -> device, assemble, solve, d -> host (max over ranks)
+    e2e = None
+    if not args.no_e2e:
+        pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
+        h = {k: pin(getattr(lp, k)) for k in ("kdiag", "bi", "bj", "pen", "e", "g", "F")}
+        hd = torch.empty(6 * lp.n_own, dtype=torch.float64).pin_memory()
+        a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        dist.barrier()
+        a0.record(stream)
+        dd = {k: v.cuda(non_blocking=True) for k, v in h.items()}
+        K2 = dda.build_matrix(dd["kdiag"], dd["bi"], dd["bj"], dd["pen"], dd["e"], dd["g"])
+        comm.attach(0, K2, lp)
+        ds, _, _, _ = comm.pcg_solve([dd["F"]], tol=1e-10, precond=args.precond)
+        hd.copy_(ds[0], non_blocking=True)
+        a1.record(stream)
+        torch.cuda.synchronize()
+        e2 = torch.tensor([a0.elapsed_time(a1)], device="cuda")
+        dist.all_reduce(e2, op=dist.ReduceOp.MAX)
+        h2d = sum(v.numel() * v.element_size() for v in h.values())
+        e2e = {"value": float(e2.item()), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": int(hd.numel() * 8),
+               "api": "dda_build_matrix + dda_dist_attach + dda_pcg_solve_dist (per-rank pinned host inputs)"}
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": ms, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": workload_name(args.blocks), "n_blocks": P.n, "dof": 6 * P.n, "springs": P.m,
+                       "precond": args.precond, "tol": 1e-10, "start": "cold (d0 = 0)",
+                       "parallelism": f"block-row partition over {world} ranks (NCCL halo + allreduce)",
+                       "rank0_rows": lp.n_own, "rank0_halo": lp.n_halo,
+                       "step": "local dda_build_matrix + dda_dist_attach + dda_pcg_solve_dist",
+                       "l2": "inputs larger than L2 per rank at 1M/N; no flush"},
+            "phases_ms": {"assemble_max": asm_max, "pcg_max": pcg_max, "pcg_iters": iters,
+                          "pcg_us_per_iter": 1000.0 * pcg_max / max(iters, 1), "true_rel_res": rel_res},
+            "roofline": {"kernel": "rank 0: k_spmv_own + k_update_own (+ NCCL halo/allreduce)", "bound": "hbm",
+                         "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
+                         "traffic": None, "peak_source": peak_src, "per": "GPU (rank 0)"},
+            "e2e": e2e, "cpu_baseline": None, "gpu_launches": int(launches), "clocks": clk.summary(),
+        }
+        print(json.dumps(line), flush=True)
+    comm.free()
+    dist.destroy_process_group()
 
 
 if __name__ == "__main__":

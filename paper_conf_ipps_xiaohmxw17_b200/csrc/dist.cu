@@ -266,6 +266,13 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     if (slot < 0 || slot >= (int)c->parts.size() || n_own < 1 || n_own > K->n) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     DistPart& D = c->parts[slot];
+    if (D.K) {                                   // re-attach (e.g. a rebuilt matrix): release the old buffers
+        cudaStreamSynchronize(st);
+        void* ptrs[] = {D.send_idx, D.sendbuf, D.x, D.q, D.r, D.z, D.part, D.scal};
+        for (void* v : ptrs)
+            if (v) dev_free(v);
+        D = DistPart();
+    }
     D.K = K;
     D.n_own = n_own;
     D.n_local = K->n;

@@ -547,9 +547,8 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         k_g_ilu_bwd<true><<<G->g_ilu, DDA_THREADS, 0, st>>>(a, G->h);
         DDA_LAUNCHED();
     }
-    // ---- the device-side loop (counted as one launch; each iteration runs 2 (BJ) or 4 (SSOR) kernels)
+    // ---- the device-side loop (its kernel launches are counted below from the iteration count)
     DDA_CK(cudaGraphLaunch(G->exec, st));
-    note_launch(1);
     // ---- epilogue: true residual
     k_g_spmv_x<false><<<G->G_spmv, DDA_THREADS, 0, st>>>(a);
     DDA_LAUNCHED();
@@ -558,6 +557,10 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     struct { int it, status; double rel; } hres;
     DDA_CK(cudaMemcpyAsync(&hres, a.out, sizeof hres, cudaMemcpyDeviceToHost, st));
     DDA_CK(cudaStreamSynchronize(st));
+    // loop body: k_g_spmv + k_g_update (+ 2 SSOR-AI halves or 2 ILU sweeps) per pass; the body runs
+    // max(iterations, 1) times (once, as a no-op pass, when the setup already decided the result)
+    const int per_pass = (pc == DDA_PC_SSOR_AI || pc == DDA_PC_ILU0) ? 4 : 2;
+    note_launch(per_pass * (hres.it > 0 ? hres.it : 1));
     if (iters) *iters = hres.it;
     if (rel_res) *rel_res = hres.rel;
     return (dda_status_t)hres.status;
