@@ -485,8 +485,12 @@ using namespace dda;
 // kernel (grid barriers instead of kernel boundaries) wins for L2-resident
 // block-Jacobi solves (10k blocks: 15.5 vs 18.6 us/iteration on B200).
 // DDA_PCG_ENGINE=graph|persistent overrides.
+static int g_forced_engine = -2;
+// Internal testing hook (not in include/dda.h): -1 = automatic, 0 = graph, 1 = persistent.
+extern "C" void dda__set_pcg_engine(int e) { g_forced_engine = e; }
+
 static int pcg_engine(const dda_matrix* K, dda_precond_t pc) {   // 0 = graph, 1 = persistent
-    static int forced = -2;
+    int& forced = g_forced_engine;
     if (forced == -2) {
         const char* v = getenv("DDA_PCG_ENGINE");
         forced = !v ? -1 : ((v[0] == 'p' || v[0] == '1') ? 1 : 0);

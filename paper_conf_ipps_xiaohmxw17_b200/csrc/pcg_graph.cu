@@ -214,23 +214,29 @@ __global__ void __launch_bounds__(DDA_THREADS) k_g_update(const GArgs a, cudaGra
     const int n = a.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
     const bool use_dinv = (a.pc == DDA_PC_BJ || a.pc == DDA_PC_SSOR_AI);
     double rr = 0.0, rz = 0.0;
-    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
-        const Row5 R = row5(grp, lane, n);
-        double rv = 0.0;
-        if (R.valid) {
-            d[R.idx] = d[R.idx] + alpha * pk[R.idx];
-            rv = a.r[R.idx] - alpha * a.q[R.idx];
-            a.r[R.idx] = rv;
-        }
-        rr += rv * rv;
-        const double tz = use_dinv ? bj_lane(a.dinv, R, rv) : rv;
-        if (R.valid) {
-            if (a.pc == DDA_PC_SSOR_AI) {
-                a.t[R.idx] = tz;
-            } else if (a.pc != DDA_PC_ILU0) {
-                a.z[R.idx] = tz;
-                rz += rv * tz;
-            }
+    // two 5-row groups per warp iteration, every load issued before any shuffle / arithmetic
+    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += 2 * W) {
+        const Row5 RA = row5(grp, lane, n);
+        const Row5 RB = row5(grp + W, lane, n);
+        double pa = 0, da = 0, ra = 0, qa = 0, pb = 0, db = 0, rb = 0, qb = 0;
+        if (RA.valid) { pa = pk[RA.idx]; da = d[RA.idx]; ra = a.r[RA.idx]; qa = a.q[RA.idx]; }
+        if (RB.valid) { pb = pk[RB.idx]; db = d[RB.idx]; rb = a.r[RB.idx]; qb = a.q[RB.idx]; }
+        DinvRow DA, DB;
+        if (use_dinv) { DA = dinv_row(a.dinv, RA); DB = dinv_row(a.dinv, RB); }
+        const double rva = RA.valid ? ra - alpha * qa : 0.0;
+        const double rvb = RB.valid ? rb - alpha * qb : 0.0;
+        if (RA.valid) { d[RA.idx] = da + alpha * pa; a.r[RA.idx] = rva; }
+        if (RB.valid) { d[RB.idx] = db + alpha * pb; a.r[RB.idx] = rvb; }
+        rr += rva * rva + rvb * rvb;
+        const double tza = use_dinv ? dinv_row_apply(DA, rva, RA) : rva;
+        const double tzb = use_dinv ? dinv_row_apply(DB, rvb, RB) : rvb;
+        if (a.pc == DDA_PC_SSOR_AI) {
+            if (RA.valid) a.t[RA.idx] = tza;
+            if (RB.valid) a.t[RB.idx] = tzb;
+        } else if (a.pc != DDA_PC_ILU0) {
+            if (RA.valid) a.z[RA.idx] = tza;
+            if (RB.valid) a.z[RB.idx] = tzb;
+            rz += rva * tza + rvb * tzb;
         }
     }
     double v[2] = {rr, rz}, tot[2];

@@ -38,6 +38,28 @@ __device__ __forceinline__ Row5 row5(int grp, int lane, int n) {
     return r;
 }
 
+// Row a of the packed D_i^{-1} for the lane's DOF (6 values), loaded ahead of use
+struct DinvRow {
+    double v[6];
+};
+__device__ __forceinline__ DinvRow dinv_row(const double* __restrict__ dinv, const Row5& R) {
+    const double* blk = dinv + (size_t)kDinv * (R.valid ? R.i : 0);
+    DinvRow d;
+#pragma unroll
+    for (int c = 0; c < 6; ++c) {
+        const int r0 = R.a < c ? R.a : c, c0 = R.a < c ? c : R.a;
+        d.v[c] = __ldg(blk + pk_off(r0, c0));
+    }
+    return d;
+}
+// z_a = sum_c D[a][c] v_c with the preloaded row; every lane of the warp must call
+__device__ __forceinline__ double dinv_row_apply(const DinvRow& d, double v, const Row5& R) {
+    double z = 0.0;
+#pragma unroll
+    for (int c = 0; c < 6; ++c) z = fma(d.v[c], __shfl_sync(0xffffffffu, v, R.base + c), z);
+    return z;
+}
+
 // z = D_i^{-1} v for the lane's DOF (packed inverse); all lanes must call
 __device__ __forceinline__ double bj_lane(const double* __restrict__ dinv, const Row5& R, double v) {
     const double* blk = dinv + (size_t)kDinv * (R.valid ? R.i : 0);

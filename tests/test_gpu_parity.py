@@ -231,14 +231,26 @@ def _pcg_parity(dda, P, O, pc, omega=1.0, d0=None, tol=1e-10):
     return d, it
 
 
+@pytest.fixture(params=["auto", "graph", "persistent"])
+def engine(request, dda):
+    """PCG engine: the CUDA-graph while loop or the persistent cooperative kernel
+    (internal hook; 'auto' picks by size and preconditioner)."""
+    import ctypes
+    f = dda.lib().dda__set_pcg_engine
+    f.argtypes = [ctypes.c_int]
+    f({"auto": -1, "graph": 0, "persistent": 1}[request.param])
+    yield request.param
+    f(-1)
+
+
 @pytest.mark.parametrize("name", ["tiny", "tiny_shuffled", "ragged_1k", "paper"])
-def test_pcg_bj(dda, name):
+def test_pcg_bj(dda, name, engine):
     P, O = case(name)
     _pcg_parity(dda, P, O, "bj")
 
 
 @pytest.mark.parametrize("name", ["tiny", "paper"])
-def test_pcg_ssor_ai(dda, name):
+def test_pcg_ssor_ai(dda, name, engine):
     P, O = case(name)
     _pcg_parity(dda, P, O, "ssor_ai")
 
@@ -265,7 +277,7 @@ def test_preconditioner_trend(dda):
     assert its["ilu0"] < its["ssor_ai"] < its["bj"], its
 
 
-def test_pcg_none(dda):
+def test_pcg_none(dda, engine):
     P, O = case("tiny")
     _pcg_parity(dda, P, O, "none")
 
@@ -281,7 +293,7 @@ def test_pcg_tiny_vs_dense_ldlt(dda):
     assert np.linalg.norm(d - ref) / np.linalg.norm(ref) <= (ev.max() / ev.min()) * 1e-10
 
 
-def test_pcg_warm_start_and_edge_cases(dda):
+def test_pcg_warm_start_and_edge_cases(dda, engine):
     P, O = case("paper")
     K = dda.build_from_problem(P)
     F = torch.from_numpy(P.F).cuda()
