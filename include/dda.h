@@ -126,6 +126,15 @@ dda_status_t dda_matrix_export(dda_matrix_t K, int32_t *row_ptr, int32_t *col_id
 dda_status_t dda_spmv(dda_matrix_t K, const double *x, double *y, void *stream);
 
 /*
+ * configs[3] comparison — the same product from FULL-storage BSR6: on first use
+ * the library expands K (every off-diagonal block stored in both rows, the
+ * representation "most of the proposed SpMV methods need to recover")
+ * and then runs the same warp kernel with every block forward.  Reads
+ * (1 + 2u) blocks per row instead of (1 + u).  x, y device [6n], no alias.
+ */
+dda_status_t dda_spmv_full(dda_matrix_t K, const double *x, double *y, void *stream);
+
+/*
  * A3 — Block-Jacobi setup (Table I "construction" P:174): D_i^{-1} for
  * every diagonal block by 6x6 Cholesky.  Called implicitly by dda_pcg_solve;
  * exposed for testing.  If dinv (device, [n][36] row-major) is non-NULL the

@@ -27,7 +27,7 @@ ABI_SYMBOLS = ("dda_build_matrix", "dda_update_values", "dda_matrix_info", "dda_
                "dda_bj_setup", "dda_precond_apply", "dda_pcg_solve", "dda_solve_host", "dda_launch_count",
                "dda_matrix_free", "dda_status_string", "dda_last_cuda_error", "dda_comm_unique_id",
                "dda_comm_init", "dda_comm_init_loopback", "dda_dist_attach", "dda_spmv_dist",
-               "dda_pcg_solve_dist", "dda_comm_free")
+               "dda_pcg_solve_dist", "dda_comm_free", "dda_spmv_full")
 
 _lib = None
 
@@ -59,6 +59,8 @@ def lib() -> C.CDLL:
         L.dda_matrix_export.restype = st
         L.dda_spmv.argtypes = [P, P, P, P]
         L.dda_spmv.restype = st
+        L.dda_spmv_full.argtypes = [P, P, P, P]
+        L.dda_spmv_full.restype = st
         L.dda_bj_setup.argtypes = [P, P, C.POINTER(I32), P]
         L.dda_bj_setup.restype = st
         L.dda_precond_apply.argtypes = [P, st, D, P, P, P]
@@ -171,6 +173,17 @@ class Matrix:
             y = torch.empty_like(x)
         yp = _dev(y, torch.float64, (N,), "y")
         _check(lib().dda_spmv(self.handle, xp, yp, C.c_void_p(_stream(stream))), "dda_spmv")
+        return y
+
+    def spmv_full(self, x, y=None, stream=None):
+        """configs[3] comparison: y = K x from full-storage BSR6 (expanded on first use)."""
+        torch = _torch()
+        N = 6 * self.n
+        xp = _dev(x, torch.float64, (N,), "x")
+        if y is None:
+            y = torch.empty_like(x)
+        yp = _dev(y, torch.float64, (N,), "y")
+        _check(lib().dda_spmv_full(self.handle, xp, yp, C.c_void_p(_stream(stream))), "dda_spmv_full")
         return y
 
     def bj_setup(self, full: bool = False, stream=None):

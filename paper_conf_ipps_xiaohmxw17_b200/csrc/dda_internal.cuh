@@ -121,6 +121,9 @@ struct dda_matrix {
     size_t ws_bytes = 0;
     void* scratch = nullptr;        // small device scratch (result struct, flags)
     void* graph_engine = nullptr;   // cached CUDA-graph PCG engine (pcg_graph.cu)
+    int32_t* full_ptr = nullptr;    // full-storage BSR6 copy for the configs[3] comparison (dda_spmv_full)
+    int32_t* full_col = nullptr;
+    double* full_val = nullptr;
     int64_t graph_iters = 0;        // loop-body launches issued inside graphs (launch accounting)
 };
 

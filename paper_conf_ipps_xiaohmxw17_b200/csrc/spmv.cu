@@ -55,6 +55,59 @@ int spmv_grid(SpmvKernel k) {
     return device_sms() * (per_sm > 0 ? per_sm : 1);
 }
 
+// Full-storage BSR6 expansion (configs[3] comparison): row i lists the lower blocks
+// V_ki^T (k < i, ascending), D_i, then the upper blocks V_ij, all stored explicitly.
+__global__ void k_full_ptr(int32_t n, const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ low_ptr,
+                           int32_t* __restrict__ fptr) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i <= n; i += gridDim.x * blockDim.x)
+        fptr[i] = row_ptr[i] + low_ptr[i] + i;
+}
+
+// one thread per (output block, entry chunk q)
+__global__ void k_full_fill(int32_t n, BsrView A, const int32_t* __restrict__ fptr, int32_t* __restrict__ fcol,
+                            double* __restrict__ fval) {
+    const int64_t total = (int64_t)fptr[n] * 9;
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t ob = t / 9;
+        const int q = (int)(t - 9 * ob);
+        // row of ob: binary search in fptr
+        int lo = 0, hi = n - 1;
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (fptr[mid] <= ob) lo = mid; else hi = mid - 1;
+        }
+        const int i = lo;
+        const int k = (int)(ob - fptr[i]);
+        const int nl = A.low_ptr[i + 1] - A.low_ptr[i];
+        const double* src;
+        int col;
+        bool tr = false;
+        if (k < nl) {
+            const int tt = A.low_ptr[i] + k;
+            src = A.upper + (size_t)kBlk * A.low_to_up[tt];
+            col = A.low_row[tt];
+            tr = true;
+        } else if (k == nl) {
+            src = A.diag + (size_t)kBlk * i;
+            col = i;
+        } else {
+            const int u = A.row_ptr[i] + (k - nl - 1);
+            src = A.upper + (size_t)kBlk * u;
+            col = A.col_idx[u];
+        }
+        if (q == 0) fcol[ob] = col;
+        const int R = q / 3, C = q % 3;
+        double4 v;
+        if (!tr) {
+            v = *reinterpret_cast<const double4*>(src + 4 * q);
+        } else {                                   // chunk (R,C) of V^T = transpose of chunk (C,R) of V
+            const double4 c = *reinterpret_cast<const double4*>(src + 4 * (3 * C + R));
+            v = make_double4(c.x, c.z, c.y, c.w);
+        }
+        *reinterpret_cast<double4*>(fval + (size_t)kBlk * ob + 4 * q) = v;
+    }
+}
+
 }  // namespace
 
 dda_status_t spmv(dda_matrix* K, const double* x, double* y, cudaStream_t s) {
@@ -68,6 +121,34 @@ dda_status_t spmv(dda_matrix* K, const double* x, double* y, cudaStream_t s) {
 }
 
 }  // namespace dda
+
+// configs[3]: full-storage BSR6 SpMV (every off-diagonal block stored twice), built on first use
+extern "C" dda_status_t dda_spmv_full(dda_matrix_t K, const double* x, double* y, void* stream) {
+    using namespace dda;
+    if (!K || !x || !y || x == y) return DDA_ERR_ARG;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    if (!K->full_ptr) {
+        const size_t nb = (size_t)K->n + 2 * (size_t)K->nnzb;
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->full_ptr), ((size_t)K->n + 1) * sizeof(int32_t), st));
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->full_col), nb * sizeof(int32_t), st));
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->full_val), nb * kBlk * sizeof(double), st));
+        k_full_ptr<<<(K->n + 256) / 256, 256, 0, st>>>(K->n, K->row_ptr, K->low_ptr, K->full_ptr);
+        DDA_LAUNCHED();
+        k_full_fill<<<device_sms() * 8, 256, 0, st>>>(K->n, view_of(K), K->full_ptr, K->full_col, K->full_val);
+        DDA_LAUNCHED();
+    }
+    BsrView F = view_of(K);
+    F.row_ptr = K->full_ptr;
+    F.col_idx = K->full_col;
+    F.upper = K->full_val;
+    const SpmvKernel k = k_spmv<SPMV_UPPER, 6>;
+    int g = spmv_grid(k);
+    const int need = (K->n + 3 * (DDA_THREADS / 32) - 1) / (3 * (DDA_THREADS / 32));
+    if (need < g) g = need > 0 ? need : 1;
+    k<<<g, DDA_THREADS, 0, st>>>(F, x, y);
+    DDA_LAUNCHED();
+    return DDA_OK;
+}
 
 extern "C" dda_status_t dda_spmv(dda_matrix_t K, const double* x, double* y, void* stream) {
     if (!K || !x || !y || x == y) return DDA_ERR_ARG;

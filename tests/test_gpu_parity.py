@@ -147,6 +147,18 @@ def test_spmv_parity(dda, name):
     assert np.linalg.norm(y - yo) / np.linalg.norm(yo) <= 1e-13
 
 
+@pytest.mark.parametrize("name", ["tiny", "tiny_shuffled", "ragged_1k"])
+def test_spmv_full_storage(dda, name):
+    # configs[3] comparison path: the same product from the expanded full-storage BSR6
+    P, O = case(name)
+    K = dda.build_from_problem(P)
+    x = torch.from_numpy(random_vector(P.n, 5)).cuda()
+    yf = K.spmv_full(x).cpu().numpy()
+    yo = O.spmv(x.cpu().numpy())
+    bound = _abs_bound(O, P.n, x.cpu().numpy())
+    assert (np.abs(yf - yo) <= 1e-12 * bound).all()
+
+
 def test_spmv_unit_vectors_exact(dda):
     P, O = case("tiny")
     K = dda.build_from_problem(P)
