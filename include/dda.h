@@ -76,7 +76,7 @@ typedef enum {
  *  n_springs    m >= 0
  *  bi, bj       device, [m] int32 block ids in [0, n), bi[s] != bj[s]
  *  pen          device, [m] penalties, finite and >= 0
- *  e, g         device, [m][6] spring vectors of block bi / bj
+ *  e, g         device, [m][6] spring vectors of block bi / bj (16-byte aligned)
  *  stream       cudaStream_t
  *  out          receives the new handle (NULL on failure)
  * Errors: DDA_ERR_ARG for n <= 0, m < 0, a NULL pointer with m > 0, an id out

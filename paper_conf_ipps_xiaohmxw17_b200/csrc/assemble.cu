@@ -91,66 +91,103 @@ __global__ void k_bounds(int32_t n, int64_t cnt, const int32_t* __restrict__ sk,
     }
 }
 
-// V_u row r: sum over the segment, in increasing spring index, of
+// V_u: sum over the segment, in increasing spring index, of
 //   (p*e[r])*g[c]  if i < j   (K_ij)      or      (p*e[c])*g[r]  if i > j   (K_ij^T)
-__global__ void k_offdiag(int64_t nnzb, const int32_t* __restrict__ seg, const int32_t* __restrict__ perm,
-                          const uint8_t* __restrict__ orient, const double* __restrict__ pen,
-                          const double* __restrict__ e, const double* __restrict__ g, double* __restrict__ upper) {
-    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < nnzb * 6;
-         idx += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t u = idx / 6;
-        const int r = (int)(idx - 6 * u);
-        double acc[6] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
+// One thread per unique block with its 36 entries in registers: every spring of the
+// segment is read once (pen, e row, g row: five 32 B sectors), instead of once per
+// (block, row) thread.
+__global__ void __launch_bounds__(128) k_offdiag(int64_t nnzb, const int32_t* __restrict__ seg,
+                                                 const int32_t* __restrict__ perm, const uint8_t* __restrict__ orient,
+                                                 const double* __restrict__ pen, const double* __restrict__ e,
+                                                 const double* __restrict__ g, double* __restrict__ upper) {
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < nnzb; u += (int64_t)gridDim.x * blockDim.x) {
+        double acc[6][6];
+#pragma unroll
+        for (int r = 0; r < 6; ++r)
+#pragma unroll
+            for (int c = 0; c < 6; ++c) acc[r][c] = 0.0;
         const int32_t t1 = seg[u + 1];
         for (int32_t t = seg[u]; t < t1; ++t) {
             const int64_t s = perm[t];
             const double p = pen[s];
-            const double* es = e + 6 * s;
-            const double* gs = g + 6 * s;
+            double es[6], gs[6];
+#pragma unroll
+            for (int k = 0; k < 3; ++k) {
+                const double2 a = *reinterpret_cast<const double2*>(e + 6 * s + 2 * k);
+                const double2 b = *reinterpret_cast<const double2*>(g + 6 * s + 2 * k);
+                es[2 * k] = a.x; es[2 * k + 1] = a.y; gs[2 * k] = b.x; gs[2 * k + 1] = b.y;
+            }
             if (orient[s]) {
-                const double pr = __dmul_rn(p, es[r]);
 #pragma unroll
-                for (int c = 0; c < 6; ++c) acc[c] = __dadd_rn(acc[c], __dmul_rn(pr, gs[c]));
+                for (int r = 0; r < 6; ++r) {
+                    const double pr = __dmul_rn(p, es[r]);
+#pragma unroll
+                    for (int c = 0; c < 6; ++c) acc[r][c] = __dadd_rn(acc[r][c], __dmul_rn(pr, gs[c]));
+                }
             } else {
-                const double gr = gs[r];
 #pragma unroll
-                for (int c = 0; c < 6; ++c) acc[c] = __dadd_rn(acc[c], __dmul_rn(__dmul_rn(p, es[c]), gr));
+                for (int c = 0; c < 6; ++c) {
+                    const double pc = __dmul_rn(p, es[c]);
+#pragma unroll
+                    for (int r = 0; r < 6; ++r) acc[r][c] = __dadd_rn(acc[r][c], __dmul_rn(pc, gs[r]));
+                }
             }
         }
         double* B = upper + (size_t)kBlk * u;
 #pragma unroll
-        for (int c = 0; c < 6; ++c) B[tile_off(r, c)] = acc[c];
+        for (int q = 0; q < 9; ++q) {
+            const int R = q / 3, C = q % 3;
+            *reinterpret_cast<double4*>(B + 4 * q) =
+                make_double4(acc[2 * R][2 * C], acc[2 * R][2 * C + 1], acc[2 * R + 1][2 * C], acc[2 * R + 1][2 * C + 1]);
+        }
     }
 }
 
-// D_i row r (c >= r): Kd_i[r][c] then the endpoint segment in spring order; mirrored.
-__global__ void k_diag(int32_t n, const int32_t* __restrict__ dstart, const int32_t* __restrict__ dperm,
-                       const double* __restrict__ pen, const double* __restrict__ e, const double* __restrict__ g,
-                       const double* __restrict__ kdiag, double* __restrict__ diag) {
-    for (int64_t idx = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; idx < (int64_t)n * 6;
-         idx += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t i = idx / 6;
-        const int r = (int)(idx - 6 * i);
-        double acc[6];
+// D_i: Kd_i's upper triangle, then the block's endpoint records in spring order
+// (p*w[r])*w[c] for r <= c, mirrored.  One thread per block, 21 accumulators.
+__global__ void __launch_bounds__(128) k_diag(int32_t n, const int32_t* __restrict__ dstart,
+                                              const int32_t* __restrict__ dperm, const double* __restrict__ pen,
+                                              const double* __restrict__ e, const double* __restrict__ g,
+                                              const double* __restrict__ kdiag, double* __restrict__ diag) {
+    for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        double acc[6][6];
 #pragma unroll
-        for (int c = 0; c < 6; ++c) acc[c] = (c >= r) ? kdiag[36 * i + 6 * r + c] : 0.0;
+        for (int r = 0; r < 6; ++r)
+#pragma unroll
+            for (int c = 0; c < 6; ++c) acc[r][c] = (c >= r) ? kdiag[36 * i + 6 * r + c] : 0.0;
         const int32_t t1 = dstart[i + 1];
         for (int32_t t = dstart[i]; t < t1; ++t) {
             const int32_t v = dperm[t];
             const int64_t s = v >> 1;
-            const double* w = ((v & 1) ? g : e) + 6 * s;
-            const double pr = __dmul_rn(pen[s], w[r]);
+            const double* wp = ((v & 1) ? g : e) + 6 * s;
+            double w[6];
 #pragma unroll
-            for (int c = 0; c < 6; ++c)
-                if (c >= r) acc[c] = __dadd_rn(acc[c], __dmul_rn(pr, w[c]));
+            for (int k = 0; k < 3; ++k) {
+                const double2 a = *reinterpret_cast<const double2*>(wp + 2 * k);
+                w[2 * k] = a.x; w[2 * k + 1] = a.y;
+            }
+            const double p = pen[s];
+#pragma unroll
+            for (int r = 0; r < 6; ++r) {
+                const double pr = __dmul_rn(p, w[r]);
+#pragma unroll
+                for (int c = r; c < 6; ++c) acc[r][c] = __dadd_rn(acc[r][c], __dmul_rn(pr, w[c]));
+            }
         }
         double* D = diag + (size_t)kBlk * i;
 #pragma unroll
-        for (int c = 0; c < 6; ++c)
-            if (c >= r) {
-                D[tile_off(r, c)] = acc[c];
-                D[tile_off(c, r)] = acc[c];
-            }
+        for (int q = 0; q < 9; ++q) {
+            const int R = q / 3, C = q % 3;
+            double m[2][2];
+#pragma unroll
+            for (int a = 0; a < 2; ++a)
+#pragma unroll
+                for (int b = 0; b < 2; ++b) {
+                    const int r = 2 * R + a, c = 2 * C + b;
+                    m[a][b] = r <= c ? acc[r][c] : acc[c][r];
+                }
+            *reinterpret_cast<double4*>(D + 4 * q) = make_double4(m[0][0], m[0][1], m[1][0], m[1][1]);
+        }
     }
 }
 
@@ -206,10 +243,11 @@ cudaError_t dmalloc(T** p, size_t count, cudaStream_t st) {
 dda_status_t run_values(dda_matrix* K, const double* kdiag, const double* pen, const double* e, const double* g,
                         cudaStream_t st) {
     if (K->nnzb > 0) {
-        k_offdiag<<<grid_for(K->nnzb * 6), TPB, 0, st>>>(K->nnzb, K->seg, K->perm, K->orient, pen, e, g, K->upper);
+        const int gb = (int)((K->nnzb + 127) / 128);
+        k_offdiag<<<gb, 128, 0, st>>>(K->nnzb, K->seg, K->perm, K->orient, pen, e, g, K->upper);
         DDA_LAUNCHED();
     }
-    k_diag<<<grid_for((int64_t)K->n * 6), TPB, 0, st>>>(K->n, K->dstart, K->dperm, pen, e, g, kdiag, K->diag);
+    k_diag<<<(K->n + 127) / 128, 128, 0, st>>>(K->n, K->dstart, K->dperm, pen, e, g, kdiag, K->diag);
     DDA_LAUNCHED();
     K->dinv_valid = false;
     K->ilu_valid = false;
@@ -253,6 +291,7 @@ extern "C" dda_status_t dda_build_matrix(int32_t n, const double* kdiag, int64_t
     if (n <= 0 || m < 0 || !kdiag) return DDA_ERR_ARG;
     if (m > 0 && (!bi || !bj || !pen || !e || !g)) return DDA_ERR_ARG;
     if (m > (int64_t)INT_MAX / 2 || (int64_t)n > (int64_t)INT_MAX / 36) return DDA_ERR_ARG;
+    if (m > 0 && ((reinterpret_cast<uintptr_t>(e) | reinterpret_cast<uintptr_t>(g)) & 15)) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
 
     dda_matrix* K = new dda_matrix();
@@ -392,6 +431,7 @@ extern "C" dda_status_t dda_update_values(dda_matrix_t K, const double* kdiag, i
                                           const double* e, const double* g, void* stream) {
     if (!K || !kdiag || m != K->m) return DDA_ERR_ARG;
     if (m > 0 && (!pen || !e || !g)) return DDA_ERR_ARG;
+    if (m > 0 && ((reinterpret_cast<uintptr_t>(e) | reinterpret_cast<uintptr_t>(g)) & 15)) return DDA_ERR_ARG;
     return run_values(K, kdiag, pen, e, g, reinterpret_cast<cudaStream_t>(stream));
 }
 
