@@ -439,6 +439,14 @@ dda_status_t pcg_solve(dda_matrix* K, const double* F, const double* d0, double*
     }
     const size_t N = 6 * (size_t)K->n;
     int G = pcg_grid();
+    {   // fewer CTAs when the rows are few: grid barriers and partial sums scale with the CTA count
+        static int cap = -1;
+        if (cap < 0) {
+            const char* e = getenv("DDA_PCG_GRID");
+            cap = e ? atoi(e) : 0;
+        }
+        if (cap > 0 && cap < G) G = cap;
+    }
     const int need = (K->n + 3 * WPB - 1) / (3 * WPB);
     if (need < G) G = need > 0 ? need : 1;
     const size_t bytes = (7 * N + 4 * (size_t)G) * sizeof(double);

@@ -67,6 +67,14 @@ __device__ __forceinline__ void set_cond(const GArgs& a, cudaGraphConditionalHan
 
 __device__ __forceinline__ bool loop_done(const State* st) { return *reinterpret_cast<volatile const int*>(&st->done); }
 
+// Programmatic dependent launch: wait for the previous kernel of the loop body
+// (all its memory operations visible), then allow the next one to be launched
+// and staged while this one runs.  No-ops when launched without the attribute.
+__device__ __forceinline__ void pdl_enter() {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
 // Deterministic grid reduction of NV values: CTA partials -> part[k*Gmax + blockIdx.x];
 // returns true in the last CTA to finish, where tot[] then holds the fixed-order sums
 // (every thread of that CTA sees them).
@@ -140,6 +148,7 @@ struct XFusedG {
 // phase A: p^(k) (fused p-update for k > 0), q = K p^(k); last CTA: sigma = p^T q, alpha = rho / sigma
 template <int MINB>
 __global__ void __launch_bounds__(DDA_THREADS, MINB) k_g_spmv(const GArgs a, cudaGraphConditionalHandle h) {
+    pdl_enter();
     if (loop_done(a.st)) {                 // finished at setup: leave the loop
         if (blockIdx.x == 0 && threadIdx.x == 0) set_cond(a, h, 0);
         return;
@@ -205,6 +214,7 @@ __device__ __forceinline__ void finish_iteration(const GArgs& a, double rz, cuda
 // phase B: d += alpha p; r -= alpha q; z = D^{-1} r (BJ) / t = D^{-1} r (SSOR) / z = r;
 // last CTA: rr, rz -> convergence test, (BJ / none) beta and the loop condition
 __global__ void __launch_bounds__(DDA_THREADS) k_g_update(const GArgs a, cudaGraphConditionalHandle h) {
+    pdl_enter();
     if (loop_done(a.st)) return;
     const int k = a.st->k;
     const double alpha = a.st->alpha;
@@ -258,6 +268,7 @@ __global__ void __launch_bounds__(DDA_THREADS) k_g_update(const GArgs a, cudaGra
 // SSOR-AI halves (INIT: at setup, also p0 = z and rho = r^T z)
 template <bool INIT>
 __global__ void __launch_bounds__(DDA_THREADS) k_g_ssor_lower(const GArgs a) {
+    pdl_enter();
     if (!INIT && loop_done(a.st)) return;
     const int lane = threadIdx.x & 31;
     const double omega = a.ca->omega;
@@ -269,6 +280,7 @@ __global__ void __launch_bounds__(DDA_THREADS) k_g_ssor_lower(const GArgs a) {
 
 template <bool INIT>
 __global__ void __launch_bounds__(DDA_THREADS) k_g_ssor_upper(const GArgs a, cudaGraphConditionalHandle h) {
+    pdl_enter();
     if (loop_done(a.st)) return;   // at setup: done means converged / F = 0 already
     const int lane = threadIdx.x & 31;
     const double omega = a.ca->omega;
@@ -513,16 +525,31 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         cudaStream_t cs;
         DDA_CK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
         DDA_CK(cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal));
-        k_g_spmv<6><<<G->G_spmv, DDA_THREADS, 0, cs>>>(a, G->h);
-        k_g_update<<<G->G_vec, DDA_THREADS, 0, cs>>>(a, G->h);
-        if (pc == DDA_PC_SSOR_AI) {
-            k_g_ssor_lower<false><<<G->G_spmv, DDA_THREADS, 0, cs>>>(a);
-            k_g_ssor_upper<false><<<G->G_spmv, DDA_THREADS, 0, cs>>>(a, G->h);
-        } else if (pc == DDA_PC_ILU0) {
-            cudaMemsetAsync(a.ilu_flags_f, 0, 2 * (size_t)K->n * sizeof(int), cs);
-            cudaMemsetAsync(a.ilu_counters, 0, 2 * sizeof(int), cs);
-            k_g_ilu_fwd<false><<<G->g_ilu, DDA_THREADS, 0, cs>>>(a);
-            k_g_ilu_bwd<false><<<G->g_ilu, DDA_THREADS, 0, cs>>>(a, G->h);
+        // body = two PCG iterations; kernels chained with programmatic dependent launch
+        cudaLaunchAttribute pdl[1];
+        pdl[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        pdl[0].val.programmaticStreamSerializationAllowed = 1;
+        auto launch = [&](auto kern, int grid, auto... args) {
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(grid);
+            cfg.blockDim = dim3(DDA_THREADS);
+            cfg.stream = cs;
+            cfg.attrs = pdl;
+            cfg.numAttrs = 1;
+            cudaLaunchKernelEx(&cfg, kern, args...);
+        };
+        for (int rep = 0; rep < 2; ++rep) {
+            launch(k_g_spmv<6>, G->G_spmv, a, G->h);
+            launch(k_g_update, G->G_vec, a, G->h);
+            if (pc == DDA_PC_SSOR_AI) {
+                launch(k_g_ssor_lower<false>, G->G_spmv, a);
+                launch(k_g_ssor_upper<false>, G->G_spmv, a, G->h);
+            } else if (pc == DDA_PC_ILU0) {
+                cudaMemsetAsync(a.ilu_flags_f, 0, 2 * (size_t)K->n * sizeof(int), cs);
+                cudaMemsetAsync(a.ilu_counters, 0, 2 * sizeof(int), cs);
+                k_g_ilu_fwd<false><<<G->g_ilu, DDA_THREADS, 0, cs>>>(a);
+                k_g_ilu_bwd<false><<<G->g_ilu, DDA_THREADS, 0, cs>>>(a, G->h);
+            }
         }
         cudaError_t ce = cudaStreamEndCapture(cs, nullptr);
         cudaStreamDestroy(cs);
@@ -565,8 +592,9 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     DDA_CK(cudaStreamSynchronize(st));
     // loop body: k_g_spmv + k_g_update (+ 2 SSOR-AI halves or 2 ILU sweeps) per pass; the body runs
     // max(iterations, 1) times (once, as a no-op pass, when the setup already decided the result)
-    const int per_pass = (pc == DDA_PC_SSOR_AI || pc == DDA_PC_ILU0) ? 4 : 2;
-    note_launch(per_pass * (hres.it > 0 ? hres.it : 1));
+    // (the body holds two iterations: an odd count still runs the whole body once more)
+    const int per_it = (pc == DDA_PC_SSOR_AI || pc == DDA_PC_ILU0) ? 4 : 2;
+    note_launch(per_it * 2 * ((hres.it > 0 ? hres.it : 1) + 1) / 2);
     if (iters) *iters = hres.it;
     if (rel_res) *rel_res = hres.rel;
     return (dda_status_t)hres.status;
