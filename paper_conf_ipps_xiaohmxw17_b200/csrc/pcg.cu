@@ -538,22 +538,28 @@ extern "C" dda_status_t dda_solve_host(int32_t n, const double* kdiag, int64_t m
     if (m > 0 && (!bi || !bj || !pen || !e || !g)) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     const size_t N = 6 * (size_t)n;
-    const size_t bytes = sizeof(double) * ((size_t)36 * n + 3 * N + (size_t)13 * m) + sizeof(int32_t) * 2 * (size_t)m;
+    // one allocation, every sub-buffer 256-byte aligned (e, g need 16 B for the vector loads)
+    auto up = [](size_t b) { return (b + 255) & ~(size_t)255; };
+    const size_t sz[9] = {sizeof(double) * 36 * (size_t)n, sizeof(double) * N, sizeof(double) * N,
+                          sizeof(double) * N, sizeof(double) * (size_t)m, sizeof(double) * 6 * (size_t)m,
+                          sizeof(double) * 6 * (size_t)m, sizeof(int32_t) * (size_t)m, sizeof(int32_t) * (size_t)m};
+    size_t off[10] = {0};
+    for (int k = 0; k < 9; ++k) off[k + 1] = off[k] + up(sz[k] ? sz[k] : 1);
     char* buf = nullptr;
-    DDA_CK(cudaMallocAsync(reinterpret_cast<void**>(&buf), bytes, st));
+    DDA_CK(cudaMallocAsync(reinterpret_cast<void**>(&buf), off[9], st));
     struct Free {
         char* b; cudaStream_t s;
         ~Free() { cudaFreeAsync(b, s); cudaStreamSynchronize(s); }
     } fr{buf, st};
-    double* dk = reinterpret_cast<double*>(buf);
-    double* dF = dk + (size_t)36 * n;
-    double* dd0 = dF + N;
-    double* dd = dd0 + N;
-    double* dpen = dd + N;
-    double* de = dpen + m;
-    double* dg = de + 6 * (size_t)m;
-    int32_t* dbi = reinterpret_cast<int32_t*>(dg + 6 * (size_t)m);
-    int32_t* dbj = dbi + m;
+    double* dk = reinterpret_cast<double*>(buf + off[0]);
+    double* dF = reinterpret_cast<double*>(buf + off[1]);
+    double* dd0 = reinterpret_cast<double*>(buf + off[2]);
+    double* dd = reinterpret_cast<double*>(buf + off[3]);
+    double* dpen = reinterpret_cast<double*>(buf + off[4]);
+    double* de = reinterpret_cast<double*>(buf + off[5]);
+    double* dg = reinterpret_cast<double*>(buf + off[6]);
+    int32_t* dbi = reinterpret_cast<int32_t*>(buf + off[7]);
+    int32_t* dbj = reinterpret_cast<int32_t*>(buf + off[8]);
     DDA_CK(cudaMemcpyAsync(dk, kdiag, sizeof(double) * 36 * (size_t)n, cudaMemcpyHostToDevice, st));
     DDA_CK(cudaMemcpyAsync(dF, F, sizeof(double) * N, cudaMemcpyHostToDevice, st));
     if (d0) DDA_CK(cudaMemcpyAsync(dd0, d0, sizeof(double) * N, cudaMemcpyHostToDevice, st));
