@@ -21,6 +21,7 @@
 #include <cstdlib>
 
 #include "ilu_dev.cuh"
+#include "spmv_col.cuh"
 
 namespace dda {
 namespace {
@@ -158,24 +159,25 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_g_spmv(const GArgs a, cud
     const int lane = threadIdx.x & 31;
     const int w0 = blockIdx.x * WPB + (threadIdx.x >> 5), W = gridDim.x * WPB;
     double acc = 0.0;
+    // column-pair map (spmv_col.cuh): 10 rows per warp, lane C holds pair C of its group's row
     if (k == 0) {
         const XPlain xf{a.p0};
-        for_rows<SPMV_FULL>(a.A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
-            if (ok && is_out_lane(lane)) {
-                const size_t o = 6 * (size_t)i + 2 * (q_of(lane) / 3);
+        for_rows_c<SPMV_FULL>(a.A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+            if (ok) {
+                const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
                 *reinterpret_cast<double2*>(a.q + o) = make_double2(y0, y1);
-                const double2 pv = xf(i, q_of(lane) / 3);
+                const double2 pv = xf(i, ccol_of(lane));
                 acc += pv.x * y0 + pv.y * y1;
             }
         });
     } else {
         double* pnew = (k & 1) ? a.p1 : a.p0;
         const XFusedG xf{a.z, (k & 1) ? a.p0 : a.p1, beta};
-        for_rows<SPMV_FULL>(a.A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
-            if (ok && is_out_lane(lane)) {
-                const size_t o = 6 * (size_t)i + 2 * (q_of(lane) / 3);
+        for_rows_c<SPMV_FULL>(a.A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+            if (ok) {
+                const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
                 *reinterpret_cast<double2*>(a.q + o) = make_double2(y0, y1);
-                const double2 pv = xf(i, q_of(lane) / 3);
+                const double2 pv = xf(i, ccol_of(lane));
                 *reinterpret_cast<double2*>(pnew + o) = pv;
                 acc += pv.x * y0 + pv.y * y1;
             }
@@ -472,8 +474,8 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         G = nullptr;
     }
     if (!G) {
-        const int need_rows = (K->n + 3 * WPB - 1) / (3 * WPB);
-        int g_spmv = occ_grid((const void*)k_g_spmv<6>, 6);
+        const int need_rows = (K->n + 10 * WPB - 1) / (10 * WPB);
+        int g_spmv = occ_grid((const void*)k_g_spmv<4>, 4);
         if (g_spmv > need_rows) g_spmv = need_rows > 0 ? need_rows : 1;
         const int need_vec = ((K->n + 4) / 5 + WPB - 1) / WPB;
         int g_vec = occ_grid((const void*)k_g_update, 8);
@@ -539,7 +541,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
             cudaLaunchKernelEx(&cfg, kern, args...);
         };
         for (int rep = 0; rep < 2; ++rep) {
-            launch(k_g_spmv<6>, G->G_spmv, a, G->h);
+            launch(k_g_spmv<4>, G->G_spmv, a, G->h);
             launch(k_g_update, G->G_vec, a, G->h);
             if (pc == DDA_PC_SSOR_AI) {
                 launch(k_g_ssor_lower<false>, G->G_spmv, a);
@@ -627,7 +629,7 @@ extern "C" int dda__time_pcg_phases(dda_matrix_t K, const double* F, double* d, 
     for (int r = 0; r < reps; ++r) {
         cudaMemcpy(&a.st->k, &one, sizeof(int), cudaMemcpyHostToDevice);   // stay on the fused path
         cudaEventRecord(e0, st);
-        k_g_spmv<6><<<G->G_spmv, DDA_THREADS, 0, st>>>(a, 0);
+        k_g_spmv<4><<<G->G_spmv, DDA_THREADS, 0, st>>>(a, 0);
         cudaEventRecord(e1, st);
         k_g_update<<<G->G_vec, DDA_THREADS, 0, st>>>(a, 0);
         cudaEventRecord(e2, st);
