@@ -227,6 +227,18 @@ dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double *const *F, const doub
                                 void *stream);
 void dda_comm_free(dda_comm_t c);
 
+/*
+ * NEXT-2 — ordering-robust SpMV: reverse Cuthill-McKee order of the block
+ * contact graph (blocks joined by a spring), host arrays, O(n + m log d).  The
+ * symmetric SpMV re-reads each transposed block from L2 soon after its first
+ * use; a random block numbering breaks that reuse (P:180 applies both uses of
+ * every stored block).  perm[new] = old block id; renumber kdiag / springs / F
+ * with it before dda_build_matrix and map d back (partition.py's peers use the
+ * same convention).  DDA_ERR_ARG for bad ids.
+ */
+dda_status_t dda_rcm_order(int32_t n_blocks, int64_t n_springs, const int32_t *bi, const int32_t *bj,
+                           int32_t *perm);
+
 /* Number of kernel launches the library has issued in this process (for the
  * benchmark's gpu_launches count). */
 int64_t dda_launch_count(void);

@@ -27,7 +27,7 @@ ABI_SYMBOLS = ("dda_build_matrix", "dda_update_values", "dda_matrix_info", "dda_
                "dda_bj_setup", "dda_precond_apply", "dda_pcg_solve", "dda_solve_host", "dda_launch_count",
                "dda_matrix_free", "dda_status_string", "dda_last_cuda_error", "dda_comm_unique_id",
                "dda_comm_init", "dda_comm_init_loopback", "dda_dist_attach", "dda_spmv_dist",
-               "dda_pcg_solve_dist", "dda_comm_free", "dda_spmv_full")
+               "dda_pcg_solve_dist", "dda_comm_free", "dda_spmv_full", "dda_rcm_order")
 
 _lib = None
 
@@ -92,6 +92,8 @@ def lib() -> C.CDLL:
         L.dda_pcg_solve_dist.restype = st
         L.dda_comm_free.argtypes = [P]
         L.dda_comm_free.restype = None
+        L.dda_rcm_order.argtypes = [I32, I64, P, P, P]
+        L.dda_rcm_order.restype = st
         _lib = L
     return _lib
 
@@ -360,3 +362,28 @@ def build_local(lp, device="cuda") -> Matrix:
     torch = _torch()
     t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(device)
     return build_matrix(t(lp.kdiag), t(lp.bi), t(lp.bj), t(lp.pen), t(lp.e), t(lp.g))
+
+
+# ----------------------------------------------------------------------------- NEXT-2 reordering
+
+def rcm_order(n: int, bi, bj) -> np.ndarray:
+    """Reverse Cuthill-McKee block order (perm[new] = old) of the contact graph, via dda_rcm_order."""
+    bi = np.ascontiguousarray(bi, np.int32)
+    bj = np.ascontiguousarray(bj, np.int32)
+    perm = np.empty(int(n), np.int32)
+    _check(lib().dda_rcm_order(int(n), int(bi.shape[0]), bi.ctypes.data_as(C.c_void_p),
+                               bj.ctypes.data_as(C.c_void_p), perm.ctypes.data_as(C.c_void_p)), "dda_rcm_order")
+    return perm
+
+
+def renumber(perm, kdiag, bi, bj, F=None):
+    """Apply a block order perm[new] = old to host inputs; returns (kdiag, bi, bj, F) in the new numbering.
+    Map a solution back with d_old = d_new.reshape(-1, 6)[inv].ravel(), inv = argsort(perm)."""
+    perm = np.asarray(perm)
+    inv = np.empty_like(perm)
+    inv[perm] = np.arange(perm.size, dtype=perm.dtype)
+    out = (np.ascontiguousarray(np.asarray(kdiag)[perm]), inv[np.asarray(bi)].astype(np.int32),
+           inv[np.asarray(bj)].astype(np.int32))
+    if F is not None:
+        out = out + (np.ascontiguousarray(np.asarray(F).reshape(-1, 6)[perm].reshape(-1)),)
+    return out

@@ -55,15 +55,19 @@ def main():
     sizes = [int(s) for s in (sys.argv[1] if len(sys.argv) > 1 else "1000,4000,16000,64000,256000,1000000,4000000").split(",")]
     shuf = os.environ.get("SHUFFLE_AT", "16000,256000,1000000").split(",")
     flush = torch.zeros(64 * 1024 * 1024, dtype=torch.float64, device="cuda")    # 512 MB > L2
+    import numpy as np
     for t, n in enumerate(sizes):
-        for sh in ([False, True] if str(n) in shuf else [False]):
-            P = make_slope(preset(n, seed=1040 + t, shuffle=sh))
+        for sh in (["course", "shuffled", "shuffled+rcm"] if str(n) in shuf else ["course"]):
+            P = make_slope(preset(n, seed=1040 + t, shuffle=(sh != "course")))
+            if sh == "shuffled+rcm":                       # NEXT-2: dda_rcm_order renumbering
+                perm = dda.rcm_order(P.n, P.bi, P.bj)
+                P.kdiag, P.bi, P.bj, P.F = dda.renumber(perm, P.kdiag, P.bi, P.bj, P.F)
             K = dda.build_from_problem(P)
             u = K.nnzb / K.n
             x = torch.rand(6 * K.n, dtype=torch.float64, device="cuda") * 2 - 1
             y = torch.empty_like(x)
             reps = 50 if K.n <= 300_000 else 20
-            out = {"blocks": K.n, "nnzb_upper": K.nnzb, "u": round(u, 3), "shuffled": sh}
+            out = {"blocks": K.n, "nnzb_upper": K.nnzb, "u": round(u, 3), "order": sh, "shuffled": sh != "course"}
             for name, fn, bpr in (("sym", lambda: K.spmv(x, y), 392 + 300 * u),
                                   ("full", lambda: K.spmv_full(x, y), 392 + 584 * u)):
                 hot_med, hot_min = timeit(fn, reps)
