@@ -1,0 +1,91 @@
+"""Parity at BASELINE.json's full size, in the launch configuration bench.py
+times (configs[4] at N = 1: ~1M blocks, 6M DOF, the CUDA-graph PCG engine):
+
+* assembly: every index array bit-exact, and sampled value blocks bit-exact,
+  against the oracle's own 1M-block assembly (O-1);
+* SpMV: 20,000 sampled scalar rows evaluated one by one by the oracle
+  (orc_spmv_rows), componentwise <= 1e-12 (|K||x|)_i;
+* PCG-BJ to 1e-10: the TRUE residual ||F - K d|| / ||F|| recomputed by the
+  oracle over all rows; and a matched 12-iteration run vs the oracle's PCG
+  (reading Z17) <= 1e-9.
+About a minute of CPU for the oracle side."""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+
+import oracle
+from synth import make_slope, preset, random_vector
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def dda():
+    if not torch.cuda.is_available():
+        pytest.fail("GPU tests need a CUDA device")
+    import __graft_entry__
+    __graft_entry__.build()
+    import paper_conf_ipps_xiaohmxw17_b200 as m
+    return m
+
+
+@pytest.fixture(scope="module")
+def full(dda):
+    P = make_slope(preset(1_000_000, seed=1005))            # bench.py's workload
+    O = oracle.assemble(P)
+    t = dda.problem_to_device(P)
+    K = dda.build_matrix(t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+    return P, O, t, K
+
+
+def test_fullsize_assembly(dda, full):
+    P, O, t, K = full
+    assert K.n == O.n and K.nnzb == O.nnzb
+    S, ex = O.export(), K.export()
+    for k in ("row_ptr", "col_idx", "low_ptr", "low_row", "low_to_up"):
+        assert np.array_equal(ex[k], getattr(S, k)), k
+    rng = np.random.default_rng(0)
+    bi = rng.choice(K.n, 5000, replace=False)
+    bu = rng.choice(K.nnzb, 5000, replace=False)
+    assert np.array_equal(ex["diag"][bi], S.diag[bi])
+    assert np.array_equal(ex["upper"][bu], S.upper[bu])
+
+
+def test_fullsize_spmv_sampled_rows(dda, full):
+    P, O, t, K = full
+    x = random_vector(P.n, 77)
+    y = K.spmv(torch.from_numpy(x).cuda()).cpu().numpy()
+    rows = np.sort(np.random.default_rng(1).choice(6 * P.n, 20000, replace=False))
+    yo = O.spmv_rows(rows, x)
+    # (|K||x|)_r on the sampled rows, from the oracle's exported blocks
+    S = O.export()
+    bound = np.zeros(rows.size)
+    for q, r in enumerate(rows):
+        i, a = divmod(int(r), 6)
+        s = np.abs(S.diag[i][a]) @ np.abs(x[6 * i:6 * i + 6])
+        for u in range(S.row_ptr[i], S.row_ptr[i + 1]):
+            j = S.col_idx[u]
+            s += np.abs(S.upper[u][a]) @ np.abs(x[6 * j:6 * j + 6])
+        for tt in range(S.low_ptr[i], S.low_ptr[i + 1]):
+            k = S.low_row[tt]
+            s += np.abs(S.upper[S.low_to_up[tt]][:, a]) @ np.abs(x[6 * k:6 * k + 6])
+        bound[q] = s
+    assert (np.abs(y[rows] - yo) <= 1e-12 * bound).all()
+
+
+def test_fullsize_pcg(dda, full):
+    P, O, t, K = full
+    d, it, rr, st = K.pcg_solve(t["F"], tol=1e-10, precond="bj")
+    assert st == dda.OK and rr <= 1.01e-10
+    dh = d.cpu().numpy()
+    allrows = np.arange(6 * P.n, dtype=np.int64)
+    res = P.F - O.spmv_rows(allrows, dh)
+    assert np.linalg.norm(res) / np.linalg.norm(P.F) <= 1.05e-10      # oracle-computed true residual
+    assert 200 <= it <= 350                                            # calibrated scale (Table I)
+    # matched iterations (reading Z17) on a short run
+    d12, it12, _, st12 = K.pcg_solve(t["F"], tol=1e-300, maxit=12, precond="bj")
+    assert st12 == dda.ERR_NO_CONVERGENCE and it12 == 12
+    dm, itm, _, _ = O.pcg(P.F, tol=1e-300, maxit=12, precond="bj")
+    assert itm == 12
+    assert np.linalg.norm(d12.cpu().numpy() - dm) <= 1e-9 * np.linalg.norm(dm)
