@@ -81,6 +81,20 @@ def pcg_launch_bytes(n: int, u: float, iters: int) -> float:
     return n * (432.0 + (S + 528.0) + (it - 1) * (S + 96.0 + 528.0) + S + 96.0)
 
 
+def pcg_launch_bytes_scaled(n: int, nnzb: int, iters: int) -> float:
+    """Algorithmic bytes of one dda_pcg_solve on the scaled block-Jacobi engine, d0 = 0
+    (DESIGN.md §6): k_scale_upper nnzb*(288 V read + 288 written + 8 indices) + n*192 (S);
+    k_s_init 384 B/row (F, S read; r~, p, x written); iteration 0: scaled SpMV 300u + 8 + 96
+    (p read, q written) + update 480 (p, x, r~, q~, L read; x, r~ written); iterations k >= 1: the
+    SpMV also reads p_old (+48) and writes p (+48); k_s_final 288 (x, S read; d written); the
+    true-residual SpMV on K + 96 (F, q read)."""
+    u = nnzb / n
+    it = max(iters, 1)
+    sp = 300.0 * u + 8.0 + 96.0
+    return (nnzb * 584.0 + n * 192.0
+            + n * (384.0 + (sp + 480.0) + (it - 1) * (sp + 96.0 + 480.0) + 288.0 + bytes_per_row_spmv(u) + 96.0))
+
+
 class ClockSampler:
     """NVML sampler of SM clock and throttle reasons during the timed region."""
 
@@ -256,8 +270,10 @@ def main():
         if ev: ev[3].record(stream)
         return K, d, it, rr, st
 
+    engine = None
     for _ in range(args.warmup):
         K, d, it, rr, st = step()
+        engine = K.pcg_engine(args.precond)
         K.free()
     torch.cuda.synchronize()
 
@@ -291,7 +307,14 @@ def main():
     assert rel_res <= 1e-10 * 1.01, rel_res
     u = nnzb / n
     pcg_ms = statistics.mean(ph_pcg)
-    pcg_bytes = pcg_launch_bytes(n, u, iters)
+    if engine == "scaled":
+        pcg_bytes = pcg_launch_bytes_scaled(n, nnzb, iters)
+        pcg_kernel = ("dda_pcg_solve, scaled block-Jacobi engine: k_scale_upper (S_i V_ij S_j^T) + one CUDA-graph "
+                      "while loop (k_g_spmv<SC> + k_s_update per iteration) with its prelude/epilogue kernels")
+    else:
+        pcg_bytes = pcg_launch_bytes(n, u, iters)
+        pcg_kernel = ("dda_pcg_solve: one CUDA-graph while loop (k_g_spmv + k_g_update per iteration) with its "
+                      "prelude/epilogue kernels")
     ach = pcg_bytes / (pcg_ms * 1e-3) / 1e9
 
     # ---- standalone symmetric SpMV (metric's first half), back to back (hot, as PCG sees it)
@@ -355,10 +378,9 @@ def main():
                    "step": "dda_build_matrix + dda_bj_setup + dda_pcg_solve"},
         "phases_ms": {"assemble": ph_build, "bj_setup": ph_bj, "pcg": pcg_ms, "pcg_iters": iters,
                       "pcg_us_per_iter": 1000.0 * pcg_ms / max(iters, 1), "true_rel_res": rel_res},
-        "roofline": {"kernel": "dda_pcg_solve: one CUDA-graph while loop (k_g_spmv + k_g_update per "
-                               "iteration) with its prelude/epilogue kernels",
+        "roofline": {"kernel": pcg_kernel, "engine": engine,
                      "bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
-                     "traffic": traffic_for(n, "pcg"), "peak_source": peak_src,
+                     "traffic": traffic_for(n, "pcg_" + str(engine)), "peak_source": peak_src,
                      "algorithmic_bytes_per_launch": pcg_bytes},
         "spmv": {"kernel": "k_spmv<FULL,6>", "ms": spmv_ms, "traffic": traffic_for(n, "spmv"), "gbs": spmv_gbs, "frac_hbm": spmv_gbs / hbm_peak,
                  "gflops": n * (72 + 144 * u) / (spmv_ms * 1e-3) / 1e9, "bytes": spmv_bytes,

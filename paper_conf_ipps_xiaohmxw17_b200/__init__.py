@@ -94,6 +94,8 @@ def lib() -> C.CDLL:
         L.dda_comm_free.restype = None
         L.dda_rcm_order.argtypes = [I32, I64, P, P, P]
         L.dda_rcm_order.restype = st
+        L.dda__pcg_engine.argtypes = [P, C.c_int]
+        L.dda__pcg_engine.restype = C.c_int
         _lib = L
     return _lib
 
@@ -223,6 +225,10 @@ class Matrix:
         if st not in (OK, ERR_NO_CONVERGENCE, ERR_BREAKDOWN) or (raise_on_fail and st != OK):
             raise DDAError(st, "dda_pcg_solve")
         return d, int(it.value), float(rr.value), int(st)
+
+    def pcg_engine(self, precond="bj") -> str:
+        """The PCG engine dda_pcg_solve picks for this matrix (internal query, for byte accounting)."""
+        return {0: "graph", 1: "persistent", 2: "scaled"}[lib().dda__pcg_engine(self.handle, PRECOND[precond])]
 
     def update_values(self, kdiag, pen, e, g, stream=None):
         torch = _torch()

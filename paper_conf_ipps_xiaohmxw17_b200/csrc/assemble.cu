@@ -250,6 +250,7 @@ dda_status_t run_values(dda_matrix* K, const double* kdiag, const double* pen, c
     k_diag<<<(K->n + 127) / 128, 128, 0, st>>>(K->n, K->dstart, K->dperm, pen, e, g, kdiag, K->diag);
     DDA_LAUNCHED();
     K->dinv_valid = false;
+    K->scaled_valid = false;
     K->ilu_valid = false;
     if (K->full_ptr) {                 // the full-storage copy holds the old values
         cudaStreamSynchronize(st);
@@ -276,7 +277,8 @@ extern "C" void dda_matrix_free(dda_matrix_t K) {
     if (K->graph_engine) pcg_graph_free(K->graph_engine);
     void* ptrs[] = {K->row_ptr, K->col_idx, K->low_ptr, K->low_row, K->low_to_up, K->urow, K->diag, K->upper,
                     K->perm, K->seg, K->dperm, K->dstart, K->orient, K->dinv, K->ws, K->scratch,
-                    K->ilu_up, K->ilu_inv, K->ilu_flags, K->ilu_order, K->full_ptr, K->full_col, K->full_val};
+                    K->ilu_up, K->ilu_inv, K->ilu_flags, K->ilu_order, K->full_ptr, K->full_col, K->full_val,
+                    K->lfac, K->sfac, K->sc_upper};
     for (void* p : ptrs)
         if (p) dev_free(p);
     cudaSetDevice(prev);

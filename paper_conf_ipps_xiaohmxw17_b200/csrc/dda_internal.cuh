@@ -34,6 +34,9 @@ __host__ __device__ __forceinline__ int pk_off(int r, int c) {
     return r * 6 - (r * (r - 1)) / 2 + (c - r);
 }
 
+// offset of (r, c), c <= r, in the packed lower triangle (row-major): Cholesky factors L, L^{-1}
+__host__ __device__ __forceinline__ int lo_off(int r, int c) { return (r * (r + 1)) / 2 + c; }
+
 // ------------------------------------------------------------------ host-side bookkeeping
 void note_launch(int k = 1);               // counts kernel launches (dda_launch_count)
 dda_status_t cuda_fail(cudaError_t e);      // records the message, maps to a status
@@ -110,6 +113,10 @@ struct dda_matrix {
     // preconditioners
     double* dinv = nullptr;         // [n][24] packed D_i^{-1}
     bool dinv_valid = false;
+    double* lfac = nullptr;         // [n][24] packed lower Cholesky factor L_i of D_i (D_i = L_i L_i^T)
+    double* sfac = nullptr;         // [n][24] packed lower S_i = L_i^{-1}
+    double* sc_upper = nullptr;     // [nnzb][36] tiled: S_i V_ij S_j^T (scaled BJ engine)
+    bool scaled_valid = false;
     double* ilu_up = nullptr;       // [nnzb][36] tiled: U_ij of the block IC(0) = ILU(0) factor
     double* ilu_inv = nullptr;      // [n][36] tiled: U_ii^{-1}
     int* ilu_flags = nullptr;       // [3n + 8]: factor / forward / backward ready flags, counters
@@ -137,5 +144,5 @@ dda_status_t ilu_apply(dda_matrix* K, const double* r, double* z, double* y, dou
 int ilu_grid();
 dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, double* d, double tol,
                              int32_t maxit, dda_precond_t pc, double omega, int32_t* iters, double* rel_res,
-                             cudaStream_t st);
+                             cudaStream_t st, bool scaled);
 }  // namespace dda

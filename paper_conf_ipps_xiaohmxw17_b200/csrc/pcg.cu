@@ -491,29 +491,37 @@ using namespace dda;
 // Engine choice: the CUDA-graph while loop (one kernel per phase, each at its
 // own occupancy) wins when the phases are HBM-bound; the persistent cooperative
 // kernel (grid barriers instead of kernel boundaries) wins for L2-resident
-// block-Jacobi solves (10k blocks: 15.5 vs 18.6 us/iteration on B200).
-// DDA_PCG_ENGINE=graph|persistent overrides.
+// block-Jacobi solves (10k blocks: 15.5 vs 18.6 us/iteration on B200).  For
+// HBM-bound block-Jacobi solves the graph loop runs on the block-scaled matrix
+// S K S^T (pcg_graph.cu, "scaled BJ engine": same iterates, 18% fewer bytes).
+// DDA_PCG_ENGINE=graph|persistent|scaled overrides.
 static int g_forced_engine = -2;
-// Internal testing hook (not in include/dda.h): -1 = automatic, 0 = graph, 1 = persistent.
+// Internal testing hook (not in include/dda.h): -1 = automatic, 0 = graph, 1 = persistent, 2 = scaled.
 extern "C" void dda__set_pcg_engine(int e) { g_forced_engine = e; }
 
-static int pcg_engine(const dda_matrix* K, dda_precond_t pc) {   // 0 = graph, 1 = persistent
+static int pcg_engine(const dda_matrix* K, dda_precond_t pc) {   // 0 = graph, 1 = persistent, 2 = scaled
     int& forced = g_forced_engine;
     if (forced == -2) {
         const char* v = getenv("DDA_PCG_ENGINE");
-        forced = !v ? -1 : ((v[0] == 'p' || v[0] == '1') ? 1 : 0);
+        forced = !v ? -1 : ((v[0] == 'p' || v[0] == '1') ? 1 : ((v[0] == 's' || v[0] == '2') ? 2 : 0));
     }
     if (pc == DDA_PC_ILU0) return 0;   // the sync-free ILU sweeps exist in the graph engine only
+    if (forced == 2) return pc == DDA_PC_BJ ? 2 : 0;
     if (forced >= 0) return forced;
+    if (pc == DDA_PC_BJ && K->n >= 65536) return 2;
     return (pc != DDA_PC_SSOR_AI && K->n < 65536) ? 1 : 0;
 }
+
+// Internal query (not in include/dda.h): the engine dda_pcg_solve would use (bench.py's byte accounting).
+extern "C" int dda__pcg_engine(dda_matrix_t K, int pc) { return K ? pcg_engine(K, (dda_precond_t)pc) : -1; }
 
 extern "C" dda_status_t dda_pcg_solve(dda_matrix_t K, const double* F, const double* d0, double* d, double tol,
                                       int32_t maxit, dda_precond_t pc, double omega, int32_t* iters,
                                       double* rel_res, void* stream) {
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (!K) return DDA_ERR_ARG;
-    if (pcg_engine(K, pc) == 1) return pcg_solve(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, st);
+    const int engine = pcg_engine(K, pc);
+    if (engine == 1) return pcg_solve(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, st);
     if (iters) *iters = 0;
     if (rel_res) *rel_res = 0.0;
     if (!K || !F || !d || !(tol > 0.0) || maxit < 0) return DDA_ERR_ARG;
@@ -526,7 +534,7 @@ extern "C" dda_status_t dda_pcg_solve(dda_matrix_t K, const double* F, const dou
         dda_status_t s = ilu_setup(K, st, nullptr);
         if (s != DDA_OK) return s;
     }
-    return pcg_graph_solve(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, st);
+    return pcg_graph_solve(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, st, engine == 2);
 }
 
 extern "C" dda_status_t dda_solve_host(int32_t n, const double* kdiag, int64_t m, const int32_t* bi,

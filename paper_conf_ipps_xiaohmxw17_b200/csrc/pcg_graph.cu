@@ -59,6 +59,9 @@ struct GArgs {           // constant for a (matrix, preconditioner): baked into 
     int* ilu_flags_b;
     int* ilu_counters;
     const int* ilu_order;
+    const double* su;    // scaled BJ engine: S_i V_ij S_j^T (tiled, upper pattern)
+    const double* lfac;  // packed lower L_i (D_i = L_i L_i^T)
+    const double* sfac;  // packed lower S_i = L_i^{-1}
     int use_cond;        // 0 only for the internal phase-timing hook (kernels launched outside the graph)
 };
 
@@ -146,14 +149,20 @@ struct XFusedG {
 
 // ---------------------------------------------------------------- loop body
 
-// phase A: p^(k) (fused p-update for k > 0), q = K p^(k); last CTA: sigma = p^T q, alpha = rho / sigma
-template <int MINB>
+// phase A: p^(k) (fused p-update for k > 0), q = K p^(k); last CTA: sigma = p^T q, alpha = rho / sigma.
+// SC (scaled BJ engine): the matrix is S K S^T, whose diagonal blocks are the identity, so the
+// off-diagonal product (SPMV_OFFDIAG over the scaled blocks) is completed by q_i += p_i and the
+// "preconditioned residual" gathered for p is the scaled residual itself (a.z == a.r).
+template <int MINB, bool SC>
 __global__ void __launch_bounds__(DDA_THREADS, MINB) k_g_spmv(const GArgs a, cudaGraphConditionalHandle h) {
     pdl_enter();
     if (loop_done(a.st)) {                 // finished at setup: leave the loop
         if (blockIdx.x == 0 && threadIdx.x == 0) set_cond(a, h, 0);
         return;
     }
+    constexpr int MODE = SC ? SPMV_OFFDIAG : SPMV_FULL;
+    BsrView A = a.A;
+    if (SC) A.upper = a.su;
     const int k = a.st->k;
     const double beta = a.st->beta;
     const int lane = threadIdx.x & 31;
@@ -162,22 +171,24 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_g_spmv(const GArgs a, cud
     // column-pair map (spmv_col.cuh): 10 rows per warp, lane C holds pair C of its group's row
     if (k == 0) {
         const XPlain xf{a.p0};
-        for_rows_c<SPMV_FULL>(a.A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+        for_rows_c<MODE>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
             if (ok) {
                 const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
-                *reinterpret_cast<double2*>(a.q + o) = make_double2(y0, y1);
                 const double2 pv = xf(i, ccol_of(lane));
+                if (SC) { y0 += pv.x; y1 += pv.y; }
+                *reinterpret_cast<double2*>(a.q + o) = make_double2(y0, y1);
                 acc += pv.x * y0 + pv.y * y1;
             }
         });
     } else {
         double* pnew = (k & 1) ? a.p1 : a.p0;
-        const XFusedG xf{a.z, (k & 1) ? a.p0 : a.p1, beta};
-        for_rows_c<SPMV_FULL>(a.A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+        const XFusedG xf{SC ? a.r : a.z, (k & 1) ? a.p0 : a.p1, beta};
+        for_rows_c<MODE>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
             if (ok) {
                 const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
-                *reinterpret_cast<double2*>(a.q + o) = make_double2(y0, y1);
                 const double2 pv = xf(i, ccol_of(lane));
+                if (SC) { y0 += pv.x; y1 += pv.y; }
+                *reinterpret_cast<double2*>(a.q + o) = make_double2(y0, y1);
                 *reinterpret_cast<double2*>(pnew + o) = pv;
                 acc += pv.x * y0 + pv.y * y1;
             }
@@ -335,6 +346,8 @@ __global__ void __launch_bounds__(DDA_THREADS) k_g_ilu_bwd(const GArgs a, cudaGr
 
 // ---------------------------------------------------------------- prelude / epilogue
 
+__device__ __noinline__ void init_decide(const GArgs& a, const double (&tot)[3]);
+
 // d = d0 (or 0), r = F - q (or F); BJ/none: z = p0 = M^{-1} r; SSOR: t = D^{-1} r;
 // last CTA: FF, rr, rho and the setup decisions (F = 0, converged at start, breakdown, maxit = 0)
 __global__ void __launch_bounds__(DDA_THREADS) k_g_init(const GArgs a) {
@@ -369,7 +382,13 @@ __global__ void __launch_bounds__(DDA_THREADS) k_g_init(const GArgs a) {
         }
     }
     double v[3] = {FF, rr, rz}, tot[3];
-    if (grid_reduce_last<3>(a, v, tot) && threadIdx.x == 0) {
+    if (grid_reduce_last<3>(a, v, tot) && threadIdx.x == 0) init_decide(a, tot);
+}
+
+// setup decisions from (FF, rr, rho): F = 0, converged at start, breakdown, maxit = 0
+__device__ __noinline__ void init_decide(const GArgs& a, const double (&tot)[3]) {
+    const CallArgs* ca = a.ca;
+    {
         State* st = a.st;
         st->FF = tot[0];
         st->bnorm = sqrt(tot[0]);
@@ -436,6 +455,183 @@ __global__ void __launch_bounds__(DDA_THREADS) k_g_resid(const GArgs a) {
     }
 }
 
+// ---------------------------------------------------------------- scaled block-Jacobi engine
+//
+// Block-Jacobi PCG on K d = F (M = D = blockdiag(D_i), D_i = L_i L_i^T) is, in exact
+// arithmetic, plain CG on the block-scaled system  Ks x = S F,  Ks = S K S^T,  S = blockdiag(L_i^{-1}),
+// d = S^T x: every iterate maps one to one (r~ = S r, p~ = L^T p, z = S^T r~, rho = r^T z = |r~|^2,
+// sigma = p^T K p = p~^T Ks p~), so alpha, beta and the iteration count are those of BJ-PCG.
+// Ks has identity diagonal blocks, so the loop streams no D_i and no D_i^{-1} and writes no z:
+// 1916 -> 1580 algorithmic bytes per block row and iteration.  The stopping test
+// stays reading Z1 on the ORIGINAL residual, ||r|| = ||L r~||, from the packed L_i.
+
+// row a of a packed lower-triangular block (M[a][c], zero for c > a)
+__device__ __forceinline__ DinvRow tri_row(const double* __restrict__ M, const Row5& R) {
+    const double* blk = M + (size_t)kDinv * (R.valid ? R.i : 0);
+    DinvRow d;
+#pragma unroll
+    for (int c = 0; c < 6; ++c) d.v[c] = c <= R.a ? __ldg(blk + lo_off(R.a, c)) : 0.0;
+    return d;
+}
+// row a of the transpose of a packed lower-triangular block (M[c][a], zero for c < a)
+__device__ __forceinline__ DinvRow tri_col(const double* __restrict__ M, const Row5& R) {
+    const double* blk = M + (size_t)kDinv * (R.valid ? R.i : 0);
+    DinvRow d;
+#pragma unroll
+    for (int c = 0; c < 6; ++c) d.v[c] = c >= R.a ? __ldg(blk + lo_off(c, R.a)) : 0.0;
+    return d;
+}
+
+// Vs_ij = S_i V_ij S_j^T for every stored upper block (one thread per block, in registers)
+__global__ void __launch_bounds__(128) k_scale_upper(int64_t nnzb, const int32_t* __restrict__ urow,
+                                                     const int32_t* __restrict__ col,
+                                                     const double* __restrict__ upper,
+                                                     const double* __restrict__ sfac, double* __restrict__ su) {
+    for (int64_t u = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; u < nnzb;
+         u += (int64_t)gridDim.x * blockDim.x) {
+        const double* V = upper + (size_t)kBlk * u;
+        double A[6][6];
+#pragma unroll
+        for (int q = 0; q < 9; ++q) {
+            const double4 v = ld_chunk(V + 4 * q);
+            const int R = q / 3, C = q % 3;
+            A[2 * R][2 * C] = v.x; A[2 * R][2 * C + 1] = v.y;
+            A[2 * R + 1][2 * C] = v.z; A[2 * R + 1][2 * C + 1] = v.w;
+        }
+        const double* Si = sfac + (size_t)kDinv * __ldg(urow + u);
+        const double* Sj = sfac + (size_t)kDinv * __ldg(col + u);
+        double s[21];
+#pragma unroll
+        for (int k = 0; k < 21; ++k) s[k] = __ldg(Si + k);
+        // A <- S_i A, rows in decreasing order (row r needs the original rows 0..r)
+#pragma unroll
+        for (int r = 5; r >= 0; --r)
+#pragma unroll
+            for (int c = 0; c < 6; ++c) {
+                double t = 0.0;
+#pragma unroll
+                for (int k = 0; k <= r; ++k) t = fma(s[lo_off(r, k)], A[k][c], t);
+                A[r][c] = t;
+            }
+#pragma unroll
+        for (int k = 0; k < 21; ++k) s[k] = __ldg(Sj + k);
+        // A <- A S_j^T: (A S^T)[r][c] = sum_{k<=c} A[r][k] S[c][k], columns in decreasing order
+#pragma unroll
+        for (int r = 0; r < 6; ++r)
+#pragma unroll
+            for (int c = 5; c >= 0; --c) {
+                double t = 0.0;
+#pragma unroll
+                for (int k = 0; k <= c; ++k) t = fma(A[r][k], s[lo_off(c, k)], t);
+                A[r][c] = t;
+            }
+        double* out = su + (size_t)kBlk * u;
+#pragma unroll
+        for (int q = 0; q < 9; ++q) {
+            const int R = q / 3, C = q % 3;
+            reinterpret_cast<double4*>(out)[q] = make_double4(A[2 * R][2 * C], A[2 * R][2 * C + 1],
+                                                              A[2 * R + 1][2 * C], A[2 * R + 1][2 * C + 1]);
+        }
+    }
+}
+
+// prelude: r = F - K d0 (or F); r~ = S r -> r, p0; x = L^T d0 (or 0) -> d; FF, rr = |r|^2, rho = |r~|^2
+__global__ void __launch_bounds__(DDA_THREADS) k_s_init(const GArgs a) {
+    const CallArgs* ca = a.ca;
+    const double* d0 = ca->d0;
+    double* d = ca->d;
+    const int lane = threadIdx.x & 31;
+    const int n = a.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    double FF = 0.0, rr = 0.0, rz = 0.0;
+    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        double rv = 0.0, fv = 0.0, dv = 0.0;
+        if (R.valid) {
+            fv = ca->F[R.idx];
+            if (d0) dv = d0[R.idx];
+            rv = d0 ? fv - a.q[R.idx] : fv;
+        }
+        const DinvRow Srow = tri_row(a.sfac, R);
+        FF += fv * fv;
+        rr += rv * rv;
+        // (lanes without a row, e.g. 30 and 31, shuffle a neighbour's values: mask them out)
+        const double rt0 = dinv_row_apply(Srow, rv, R);
+        const double rt = R.valid ? rt0 : 0.0;
+        double xt = 0.0;
+        if (d0) {                                  // uniform branch: every lane shuffles
+            const DinvRow Lcol = tri_col(a.lfac, R);
+            xt = dinv_row_apply(Lcol, dv, R);
+        }
+        if (R.valid) {
+            a.r[R.idx] = rt;
+            a.p0[R.idx] = rt;
+            d[R.idx] = xt;
+        }
+        rz += rt * rt;
+    }
+    double v[3] = {FF, rr, rz}, tot[3];
+    if (grid_reduce_last<3>(a, v, tot) && threadIdx.x == 0) init_decide(a, tot);
+}
+
+// phase B: x += alpha p~ (in d); r~ -= alpha q~; rr = |L r~|^2 (the original residual), rz = |r~|^2
+__global__ void __launch_bounds__(DDA_THREADS) k_s_update(const GArgs a, cudaGraphConditionalHandle h) {
+    pdl_enter();
+    if (loop_done(a.st)) return;
+    const int k = a.st->k;
+    const double alpha = a.st->alpha;
+    const double* pk = (k & 1) ? a.p1 : a.p0;
+    double* d = a.ca->d;
+    const int lane = threadIdx.x & 31;
+    const int n = a.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    double rr = 0.0, rz = 0.0;
+    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += 2 * W) {
+        const Row5 RA = row5(grp, lane, n);
+        const Row5 RB = row5(grp + W, lane, n);
+        double pa = 0, da = 0, ra = 0, qa = 0, pb = 0, db = 0, rb = 0, qb = 0;
+        if (RA.valid) { pa = pk[RA.idx]; da = d[RA.idx]; ra = a.r[RA.idx]; qa = a.q[RA.idx]; }
+        if (RB.valid) { pb = pk[RB.idx]; db = d[RB.idx]; rb = a.r[RB.idx]; qb = a.q[RB.idx]; }
+        const DinvRow LA = tri_row(a.lfac, RA), LB = tri_row(a.lfac, RB);
+        const double rva = RA.valid ? ra - alpha * qa : 0.0;
+        const double rvb = RB.valid ? rb - alpha * qb : 0.0;
+        if (RA.valid) { d[RA.idx] = da + alpha * pa; a.r[RA.idx] = rva; }
+        if (RB.valid) { d[RB.idx] = db + alpha * pb; a.r[RB.idx] = rvb; }
+        rz += rva * rva + rvb * rvb;
+        const double oa0 = dinv_row_apply(LA, rva, RA);   // L r~ (invalid lanes masked below)
+        const double ob0 = dinv_row_apply(LB, rvb, RB);
+        const double oa = RA.valid ? oa0 : 0.0, ob = RB.valid ? ob0 : 0.0;
+        rr += oa * oa + ob * ob;
+    }
+    double v[2] = {rr, rz}, tot[2];
+    if (grid_reduce_last<2>(a, v, tot) && threadIdx.x == 0) {
+        State* st = a.st;
+        st->rr = tot[0];
+        st->iters = k + 1;
+        if (sqrt(tot[0]) <= a.ca->tol * st->bnorm) {
+            st->status = DDA_OK;
+            st->k = k + 1;
+            st->done = 1;
+            set_cond(a, h, 0);
+        } else {
+            finish_iteration(a, tot[1], h);
+        }
+    }
+}
+
+// epilogue: d = S^T x in place (before the true residual)
+__global__ void __launch_bounds__(DDA_THREADS) k_s_final(const GArgs a) {
+    if (a.st->zero_d) return;
+    double* d = a.ca->d;
+    const int lane = threadIdx.x & 31;
+    const int n = a.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        const double xv = R.valid ? d[R.idx] : 0.0;
+        const DinvRow Scol = tri_col(a.sfac, R);
+        const double dv = dinv_row_apply(Scol, xv, R);
+        if (R.valid) d[R.idx] = dv;
+    }
+}
+
 int occ_grid(const void* k, int minb_cap) {
     int per_sm = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, DDA_THREADS, 0);
@@ -464,18 +660,40 @@ void pcg_graph_free(void* p) {
     delete g;
 }
 
+// S_i V_ij S_j^T for the scaled BJ engine (needs the factors from bj_setup); cached until the values change
+dda_status_t scaled_setup(dda_matrix* K, cudaStream_t st) {
+    if (K->scaled_valid) return DDA_OK;
+    if (!K->sc_upper && K->nnzb > 0)
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->sc_upper), sizeof(double) * kBlk * (size_t)K->nnzb, st));
+    if (K->nnzb > 0) {
+        int g = (int)((K->nnzb + 127) / 128);
+        const int cap = device_sms() * 16;
+        if (g > cap) g = cap;
+        k_scale_upper<<<g, 128, 0, st>>>(K->nnzb, K->urow, K->col_idx, K->upper, K->sfac, K->sc_upper);
+        DDA_LAUNCHED();
+    }
+    K->scaled_valid = true;
+    return DDA_OK;
+}
+
 dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, double* d, double tol,
                              int32_t maxit, dda_precond_t pc, double omega, int32_t* iters, double* rel_res,
-                             cudaStream_t st) {
+                             cudaStream_t st, bool scaled) {
     const size_t N = 6 * (size_t)K->n;
+    if (scaled) {
+        if (pc != DDA_PC_BJ) return DDA_ERR_ARG;
+        dda_status_t s = scaled_setup(K, st);
+        if (s != DDA_OK) return s;
+    }
+    const int key = scaled ? 100 + (int)pc : (int)pc;
     PcgGraph*& G = reinterpret_cast<PcgGraph*&>(K->graph_engine);
-    if (G && G->pc != (int)pc) {
+    if (G && G->pc != key) {
         pcg_graph_free(G);
         G = nullptr;
     }
     if (!G) {
         const int need_rows = (K->n + 10 * WPB - 1) / (10 * WPB);
-        int g_spmv = occ_grid((const void*)k_g_spmv<4>, 4);
+        int g_spmv = occ_grid(scaled ? (const void*)k_g_spmv<4, true> : (const void*)k_g_spmv<4, false>, 4);
         if (g_spmv > need_rows) g_spmv = need_rows > 0 ? need_rows : 1;
         const int need_vec = ((K->n + 4) / 5 + WPB - 1) / WPB;
         int g_vec = occ_grid((const void*)k_g_update, 8);
@@ -487,7 +705,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         dda_status_t s = ensure_workspace(K, bytes, st);
         if (s != DDA_OK) return s;
         G = new PcgGraph();
-        G->pc = (int)pc;
+        G->pc = key;
         G->G_spmv = g_spmv;
         G->G_vec = g_vec;
         double* ws = K->ws;
@@ -510,6 +728,9 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         a.ilu_flags_b = K->ilu_flags ? K->ilu_flags + 2 * (size_t)K->n : nullptr;
         a.ilu_counters = K->ilu_flags ? K->ilu_flags + 3 * (size_t)K->n + 2 : nullptr;
         a.ilu_order = K->ilu_order;
+        a.su = K->sc_upper;
+        a.lfac = K->lfac;
+        a.sfac = K->sfac;
         G->g_ilu = ilu_grid();
         DDA_CK(cudaMemsetAsync(a.st, 0, sizeof(State), st));       // ticket = 0
 
@@ -541,7 +762,12 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
             cudaLaunchKernelEx(&cfg, kern, args...);
         };
         for (int rep = 0; rep < 2; ++rep) {
-            launch(k_g_spmv<4>, G->G_spmv, a, G->h);
+            if (scaled) {
+                launch(k_g_spmv<4, true>, G->G_spmv, a, G->h);
+                launch(k_s_update, G->G_vec, a, G->h);
+                continue;
+            }
+            launch(k_g_spmv<4, false>, G->G_spmv, a, G->h);
             launch(k_g_update, G->G_vec, a, G->h);
             if (pc == DDA_PC_SSOR_AI) {
                 launch(k_g_ssor_lower<false>, G->G_spmv, a);
@@ -567,7 +793,10 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         k_g_spmv_x<true><<<G->G_spmv, DDA_THREADS, 0, st>>>(a);
         DDA_LAUNCHED();
     }
-    k_g_init<<<G->G_vec, DDA_THREADS, 0, st>>>(a);
+    if (scaled)
+        k_s_init<<<G->G_vec, DDA_THREADS, 0, st>>>(a);
+    else
+        k_g_init<<<G->G_vec, DDA_THREADS, 0, st>>>(a);
     DDA_LAUNCHED();
     if (pc == DDA_PC_SSOR_AI) {
         k_g_ssor_lower<true><<<G->G_spmv, DDA_THREADS, 0, st>>>(a);
@@ -584,7 +813,11 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     }
     // ---- the device-side loop (its kernel launches are counted below from the iteration count)
     DDA_CK(cudaGraphLaunch(G->exec, st));
-    // ---- epilogue: true residual
+    // ---- epilogue: [d = S^T x], true residual
+    if (scaled) {
+        k_s_final<<<G->G_vec, DDA_THREADS, 0, st>>>(a);
+        DDA_LAUNCHED();
+    }
     k_g_spmv_x<false><<<G->G_spmv, DDA_THREADS, 0, st>>>(a);
     DDA_LAUNCHED();
     k_g_resid<<<G->G_vec, DDA_THREADS, 0, st>>>(a);
@@ -607,20 +840,23 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
 // Internal tuning hook (not part of include/dda.h): runs the setup of a BJ solve,
 // then times `reps` direct launches of each loop-body kernel (outside the graph).
 // ms[0] = k_g_spmv (fused, k >= 1), ms[1] = k_g_update.
-extern "C" int dda__time_pcg_phases(dda_matrix_t K, const double* F, double* d, int reps, float* ms) {
+extern "C" int dda__time_pcg_phases_ex(dda_matrix_t K, const double* F, double* d, int reps, float* ms, int scaled) {
     using namespace dda;
     cudaStream_t st = 0;
     int it = 0;
     double rr = 0;
     if (!K->dinv_valid && bj_setup(K, st, nullptr) != DDA_OK) return -1;
-    if (pcg_graph_solve(K, F, nullptr, d, 1e-10, 3, DDA_PC_BJ, 1.0, &it, &rr, st) < 0) return -2;
+    if (pcg_graph_solve(K, F, nullptr, d, 1e-10, 3, DDA_PC_BJ, 1.0, &it, &rr, st, scaled != 0) < 0) return -2;
     PcgGraph* G = reinterpret_cast<PcgGraph*>(K->graph_engine);
     GArgs a = G->a;
     a.use_cond = 0;
     // re-run the setup so the state is "in the loop"
     CallArgs hca{F, nullptr, d, 1e-300, 1.0, 1 << 30};
     cudaMemcpy(const_cast<CallArgs*>(a.ca), &hca, sizeof hca, cudaMemcpyHostToDevice);
-    k_g_init<<<G->G_vec, DDA_THREADS, 0, st>>>(a);
+    if (scaled)
+        k_s_init<<<G->G_vec, DDA_THREADS, 0, st>>>(a);
+    else
+        k_g_init<<<G->G_vec, DDA_THREADS, 0, st>>>(a);
     int one = 1;
     cudaMemcpy(&a.st->k, &one, sizeof(int), cudaMemcpyHostToDevice);
     cudaEvent_t e0, e1, e2;
@@ -629,9 +865,15 @@ extern "C" int dda__time_pcg_phases(dda_matrix_t K, const double* F, double* d, 
     for (int r = 0; r < reps; ++r) {
         cudaMemcpy(&a.st->k, &one, sizeof(int), cudaMemcpyHostToDevice);   // stay on the fused path
         cudaEventRecord(e0, st);
-        k_g_spmv<4><<<G->G_spmv, DDA_THREADS, 0, st>>>(a, 0);
+        if (scaled)
+            k_g_spmv<4, true><<<G->G_spmv, DDA_THREADS, 0, st>>>(a, 0);
+        else
+            k_g_spmv<4, false><<<G->G_spmv, DDA_THREADS, 0, st>>>(a, 0);
         cudaEventRecord(e1, st);
-        k_g_update<<<G->G_vec, DDA_THREADS, 0, st>>>(a, 0);
+        if (scaled)
+            k_s_update<<<G->G_vec, DDA_THREADS, 0, st>>>(a, 0);
+        else
+            k_g_update<<<G->G_vec, DDA_THREADS, 0, st>>>(a, 0);
         cudaEventRecord(e2, st);
         cudaEventSynchronize(e2);
         float x, y;
@@ -643,4 +885,22 @@ extern "C" int dda__time_pcg_phases(dda_matrix_t K, const double* F, double* d, 
     ms[1] = t_upd / reps;
     cudaEventDestroy(e0); cudaEventDestroy(e1); cudaEventDestroy(e2);
     return cudaGetLastError() == cudaSuccess ? 0 : -3;
+}
+
+extern "C" int dda__time_pcg_phases(dda_matrix_t K, const double* F, double* d, int reps, float* ms) {
+    return dda__time_pcg_phases_ex(K, F, d, reps, ms, 0);
+}
+
+// Internal debugging hook (not in include/dda.h): copies the scaled-engine arrays to host
+// buffers (any may be NULL): su [nnzb][36] tiled, lfac / sfac [n][24] packed lower.
+extern "C" int dda__scaled_export(dda_matrix_t K, double* su, double* lfac, double* sfac) {
+    using namespace dda;
+    if (!K) return -1;
+    if (!K->dinv_valid && bj_setup(K, 0, nullptr) != DDA_OK) return -2;
+    if (scaled_setup(K, 0) != DDA_OK) return -3;
+    if (cudaDeviceSynchronize() != cudaSuccess) return -4;
+    if (su && K->nnzb) cudaMemcpy(su, K->sc_upper, sizeof(double) * kBlk * K->nnzb, cudaMemcpyDeviceToHost);
+    if (lfac) cudaMemcpy(lfac, K->lfac, sizeof(double) * kDinv * K->n, cudaMemcpyDeviceToHost);
+    if (sfac) cudaMemcpy(sfac, K->sfac, sizeof(double) * kDinv * K->n, cudaMemcpyDeviceToHost);
+    return cudaGetLastError() == cudaSuccess ? 0 : -5;
 }

@@ -15,7 +15,8 @@ namespace dda {
 namespace {
 
 __global__ void __launch_bounds__(128) k_bj_inv(int32_t n, const double* __restrict__ diag, double* __restrict__ dinv,
-                                                double* __restrict__ full, int* __restrict__ bad) {
+                                                double* __restrict__ full, double* __restrict__ lfac,
+                                                double* __restrict__ sfac, int* __restrict__ bad) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const double* D = diag + (size_t)kBlk * i;
         double A[6][6];
@@ -73,6 +74,24 @@ __global__ void __launch_bounds__(128) k_bj_inv(int32_t n, const double* __restr
         P[21] = P[22] = P[23] = 0.0;
 #pragma unroll
         for (int q = 0; q < 12; ++q) reinterpret_cast<double2*>(out)[q] = make_double2(P[2 * q], P[2 * q + 1]);
+        if (lfac) {   // packed lower triangles of L and S = L^{-1} for the scaled BJ engine (pcg_graph.cu)
+            double PL[24], PS[24];
+#pragma unroll
+            for (int r = 0; r < 6; ++r)
+#pragma unroll
+                for (int c = 0; c <= r; ++c) {
+                    PL[lo_off(r, c)] = L[r][c];
+                    PS[lo_off(r, c)] = Li[r][c];
+                }
+            PL[21] = PL[22] = PL[23] = PS[21] = PS[22] = PS[23] = 0.0;
+            double* lo = lfac + (size_t)kDinv * i;
+            double* so = sfac + (size_t)kDinv * i;
+#pragma unroll
+            for (int q = 0; q < 12; ++q) {
+                reinterpret_cast<double2*>(lo)[q] = make_double2(PL[2 * q], PL[2 * q + 1]);
+                reinterpret_cast<double2*>(so)[q] = make_double2(PS[2 * q], PS[2 * q + 1]);
+            }
+        }
         if (full) {
 #pragma unroll
             for (int r = 0; r < 6; ++r)
@@ -133,7 +152,12 @@ static dda_status_t bj_setup_n(dda_matrix* K, int32_t nrows, cudaStream_t st, in
     int g = (nrows + 127) / 128;
     const int cap = device_sms() * 16;
     if (g > cap) g = cap;
-    k_bj_inv<<<g, 128, 0, st>>>(nrows, K->diag, K->dinv, full, bad);
+    if (!K->lfac) {
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->lfac), sizeof(double) * kDinv * (size_t)K->n, st));
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->sfac), sizeof(double) * kDinv * (size_t)K->n, st));
+    }
+    K->scaled_valid = false;
+    k_bj_inv<<<g, 128, 0, st>>>(nrows, K->diag, K->dinv, full, K->lfac, K->sfac, bad);
     DDA_LAUNCHED();
     int hbad = 0;
     DDA_CK(cudaMemcpyAsync(&hbad, bad, sizeof(int), cudaMemcpyDeviceToHost, st));

@@ -24,7 +24,9 @@
 
 namespace dda {
 
-enum SpmvMode { SPMV_FULL = 0, SPMV_LOWER_T = 1, SPMV_UPPER = 2 };
+// SPMV_OFFDIAG: both triangles without the diagonal block (the scaled BJ engine, whose
+// diagonal blocks are the identity and are applied by the caller)
+enum SpmvMode { SPMV_FULL = 0, SPMV_LOWER_T = 1, SPMV_UPPER = 2, SPMV_OFFDIAG = 3 };
 
 struct BsrView {
     int32_t n;

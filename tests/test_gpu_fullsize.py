@@ -74,7 +74,19 @@ def test_fullsize_spmv_sampled_rows(dda, full):
     assert (np.abs(y[rows] - yo) <= 1e-12 * bound).all()
 
 
-def test_fullsize_pcg(dda, full):
+@pytest.fixture(params=["auto", "graph"])
+def engine(request, dda):
+    """auto = the scaled block-Jacobi engine bench.py times at this size; graph = the
+    unscaled CUDA-graph loop (internal hook dda__set_pcg_engine)."""
+    import ctypes
+    f = dda.lib().dda__set_pcg_engine
+    f.argtypes = [ctypes.c_int]
+    f({"auto": -1, "graph": 0}[request.param])
+    yield request.param
+    f(-1)
+
+
+def test_fullsize_pcg(dda, full, engine):
     P, O, t, K = full
     d, it, rr, st = K.pcg_solve(t["F"], tol=1e-10, precond="bj")
     assert st == dda.OK and rr <= 1.01e-10

@@ -243,14 +243,16 @@ def _pcg_parity(dda, P, O, pc, omega=1.0, d0=None, tol=1e-10):
     return d, it
 
 
-@pytest.fixture(params=["auto", "graph", "persistent"])
+@pytest.fixture(params=["auto", "graph", "persistent", "scaled"])
 def engine(request, dda):
-    """PCG engine: the CUDA-graph while loop or the persistent cooperative kernel
-    (internal hook; 'auto' picks by size and preconditioner)."""
+    """PCG engine: the CUDA-graph while loop, the persistent cooperative kernel, or the
+    graph loop on the block-scaled matrix S K S^T (block-Jacobi only; other
+    preconditioners fall back to the graph loop) — internal hook; 'auto' picks by
+    size and preconditioner."""
     import ctypes
     f = dda.lib().dda__set_pcg_engine
     f.argtypes = [ctypes.c_int]
-    f({"auto": -1, "graph": 0, "persistent": 1}[request.param])
+    f({"auto": -1, "graph": 0, "persistent": 1, "scaled": 2}[request.param])
     yield request.param
     f(-1)
 

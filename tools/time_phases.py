@@ -9,12 +9,17 @@ P = make_slope(preset(n, seed=1005))
 t = dda.problem_to_device(P)
 K = dda.build_matrix(t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
 L = dda.lib()
-L.dda__time_pcg_phases.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_int, C.c_void_p]
+L.dda__time_pcg_phases_ex.argtypes = [C.c_void_p, C.c_void_p, C.c_void_p, C.c_int, C.c_void_p, C.c_int]
 d = torch.empty_like(t["F"])
-ms = (C.c_float * 2)()
-rc = L.dda__time_pcg_phases(K.handle, C.c_void_p(t["F"].data_ptr()), C.c_void_p(d.data_ptr()), 20, ms)
 u = K.nnzb / K.n
-spmv_bytes = K.n * (392 + 300 * u + 96)
-upd_bytes = K.n * 528
-print(json.dumps({"rc": rc, "n": K.n, "spmv_fused_ms": ms[0], "spmv_fused_gbs": spmv_bytes / ms[0] / 1e6,
-                  "update_ms": ms[1], "update_gbs": upd_bytes / ms[1] / 1e6}))
+for scaled in (0, 1):
+    ms = (C.c_float * 2)()
+    rc = L.dda__time_pcg_phases_ex(K.handle, C.c_void_p(t["F"].data_ptr()), C.c_void_p(d.data_ptr()), 20, ms,
+                                   scaled)
+    # algorithmic bytes per row: unscaled SpMV + 96 / update 528; scaled SpMV
+    # without D (300u + 8 + 192) / update 480 (p, x, r~, q~, L read; x, r~ written)
+    spmv_bytes = K.n * ((300 * u + 200) if scaled else (392 + 300 * u + 96))
+    upd_bytes = K.n * (480 if scaled else 528)
+    print(json.dumps({"scaled": scaled, "rc": rc, "n": K.n, "spmv_fused_ms": ms[0],
+                      "spmv_fused_gbs": spmv_bytes / ms[0] / 1e6,
+                      "update_ms": ms[1], "update_gbs": upd_bytes / ms[1] / 1e6}))
