@@ -632,6 +632,24 @@ __global__ void __launch_bounds__(DDA_THREADS) k_s_final(const GArgs a) {
     }
 }
 
+// loop-body SpMV kernel variants (tuning aid, DDA_GSPMV_VARIANT): occupancy / register budget
+typedef void (*GSpmvKernel)(const GArgs, cudaGraphConditionalHandle);
+struct GSpmvVariant { GSpmvKernel plain, scaled; int minb; };
+const GSpmvVariant kGSpmv[] = {
+    {k_g_spmv<4, false>, k_g_spmv<4, true>, 4},
+    {k_g_spmv<3, false>, k_g_spmv<3, true>, 3},
+    {k_g_spmv<5, false>, k_g_spmv<5, true>, 5},
+};
+const GSpmvVariant& gspmv_variant() {
+    static int v = -1;
+    if (v < 0) {
+        const char* e = getenv("DDA_GSPMV_VARIANT");
+        v = e ? atoi(e) : 0;
+        if (v < 0 || v >= (int)(sizeof(kGSpmv) / sizeof(kGSpmv[0]))) v = 0;
+    }
+    return kGSpmv[v];
+}
+
 int occ_grid(const void* k, int minb_cap) {
     int per_sm = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, DDA_THREADS, 0);
@@ -693,7 +711,8 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     }
     if (!G) {
         const int need_rows = (K->n + 10 * WPB - 1) / (10 * WPB);
-        int g_spmv = occ_grid(scaled ? (const void*)k_g_spmv<4, true> : (const void*)k_g_spmv<4, false>, 4);
+        const GSpmvVariant& gv = gspmv_variant();
+        int g_spmv = occ_grid(scaled ? (const void*)gv.scaled : (const void*)gv.plain, gv.minb);
         if (g_spmv > need_rows) g_spmv = need_rows > 0 ? need_rows : 1;
         const int need_vec = ((K->n + 4) / 5 + WPB - 1) / WPB;
         int g_vec = occ_grid((const void*)k_g_update, 8);
@@ -763,11 +782,11 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         };
         for (int rep = 0; rep < 2; ++rep) {
             if (scaled) {
-                launch(k_g_spmv<4, true>, G->G_spmv, a, G->h);
+                launch(gspmv_variant().scaled, G->G_spmv, a, G->h);
                 launch(k_s_update, G->G_vec, a, G->h);
                 continue;
             }
-            launch(k_g_spmv<4, false>, G->G_spmv, a, G->h);
+            launch(gspmv_variant().plain, G->G_spmv, a, G->h);
             launch(k_g_update, G->G_vec, a, G->h);
             if (pc == DDA_PC_SSOR_AI) {
                 launch(k_g_ssor_lower<false>, G->G_spmv, a);
@@ -866,9 +885,9 @@ extern "C" int dda__time_pcg_phases_ex(dda_matrix_t K, const double* F, double* 
         cudaMemcpy(&a.st->k, &one, sizeof(int), cudaMemcpyHostToDevice);   // stay on the fused path
         cudaEventRecord(e0, st);
         if (scaled)
-            k_g_spmv<4, true><<<G->G_spmv, DDA_THREADS, 0, st>>>(a, 0);
+            gspmv_variant().scaled<<<G->G_spmv, DDA_THREADS, 0, st>>>(a, 0);
         else
-            k_g_spmv<4, false><<<G->G_spmv, DDA_THREADS, 0, st>>>(a, 0);
+            gspmv_variant().plain<<<G->G_spmv, DDA_THREADS, 0, st>>>(a, 0);
         cudaEventRecord(e1, st);
         if (scaled)
             k_s_update<<<G->G_vec, DDA_THREADS, 0, st>>>(a, 0);
