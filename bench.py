@@ -228,6 +228,7 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--cpu-sample-blocks", type=int, default=65_536)
     ap.add_argument("--ref-sample-blocks", type=int, default=16_384)
+    ap.add_argument("--clock-period", type=float, default=0.05, help="NVML clock sampling period (s)")
     args = ap.parse_args()
     if args.warmup < 3:
         print("warning: --warmup < 3 violates the timing rules; using 3", file=sys.stderr)
@@ -284,7 +285,7 @@ def main():
     if world > 1:
         torch.distributed.barrier()
     torch.cuda.synchronize()
-    with ClockSampler(local) as clk:
+    with ClockSampler(local, args.clock_period) as clk:
         start.record(stream)
         for k in range(args.steps):
             K, d, it, rr, st = step(evs[k])
@@ -431,7 +432,7 @@ def run_dist(args, P, world, rank, local):
     dist.barrier()
     torch.cuda.synchronize()
     res = []
-    with ClockSampler(local) as clk:
+    with ClockSampler(local, args.clock_period) as clk:
         start.record(stream)
         for k in range(args.steps):
             res.append(step(evs[k]))

@@ -243,6 +243,16 @@ dda_status_t dda_rcm_order(int32_t n_blocks, int64_t n_springs, const int32_t *b
  * benchmark's gpu_launches count). */
 int64_t dda_launch_count(void);
 
+/* Device memory.  The library allocates its own arrays (matrix, preconditioners,
+ * PCG workspace, assembly temporaries) from a caching allocator: blocks freed by
+ * dda_matrix_free stay cached and are handed back, stream-ordered, to the next
+ * build of a similar size (the open-close loop rebuilds K every loop).
+ * dda_memory_release returns every cached block to the driver (it synchronises
+ * each device that holds some); dda_memory_cached reports the cached bytes.
+ * Caller-owned buffers are never touched by either. */
+void dda_memory_release(void);
+int64_t dda_memory_cached(void);
+
 void dda_matrix_free(dda_matrix_t K);
 const char *dda_status_string(dda_status_t s);
 /* Text of the last CUDA error seen by this thread ("" if none). */

@@ -27,7 +27,8 @@ ABI_SYMBOLS = ("dda_build_matrix", "dda_update_values", "dda_matrix_info", "dda_
                "dda_bj_setup", "dda_precond_apply", "dda_pcg_solve", "dda_solve_host", "dda_launch_count",
                "dda_matrix_free", "dda_status_string", "dda_last_cuda_error", "dda_comm_unique_id",
                "dda_comm_init", "dda_comm_init_loopback", "dda_dist_attach", "dda_spmv_dist",
-               "dda_pcg_solve_dist", "dda_comm_free", "dda_spmv_full", "dda_rcm_order")
+               "dda_pcg_solve_dist", "dda_comm_free", "dda_spmv_full", "dda_rcm_order",
+               "dda_memory_release", "dda_memory_cached")
 
 _lib = None
 
@@ -94,6 +95,10 @@ def lib() -> C.CDLL:
         L.dda_comm_free.restype = None
         L.dda_rcm_order.argtypes = [I32, I64, P, P, P]
         L.dda_rcm_order.restype = st
+        L.dda_memory_release.argtypes = []
+        L.dda_memory_release.restype = None
+        L.dda_memory_cached.argtypes = []
+        L.dda_memory_cached.restype = I64
         L.dda__pcg_engine.argtypes = [P, C.c_int]
         L.dda__pcg_engine.restype = C.c_int
         _lib = L
@@ -127,6 +132,16 @@ def _dev(t, dtype, shape=None, name="tensor"):
 def _check(st: int, what: str):
     if st != OK:
         raise DDAError(st, what)
+
+
+def memory_release() -> None:
+    """Return the library's cached device blocks to the driver (dda_memory_release)."""
+    lib().dda_memory_release()
+
+
+def memory_cached() -> int:
+    """Bytes the library's caching allocator holds for reuse (dda_memory_cached)."""
+    return int(lib().dda_memory_cached())
 
 
 def launch_count() -> int:

@@ -225,13 +225,13 @@ struct Tmp {
     template <class T>
     cudaError_t get(T** p, size_t count) {
         void* q = nullptr;
-        cudaError_t e = cudaMallocAsync(&q, count ? count * sizeof(T) : 16, s);
+        cudaError_t e = dev_alloc(&q, count ? count * sizeof(T) : 16, s);
         if (e == cudaSuccess) ptrs.push_back(q);
         *p = reinterpret_cast<T*>(q);
         return e;
     }
     ~Tmp() {
-        for (void* p : ptrs) cudaFreeAsync(p, s);
+        for (void* p : ptrs) dev_free_on(p, s);
     }
 };
 
@@ -273,8 +273,11 @@ extern "C" void dda_matrix_free(dda_matrix_t K) {
     int prev = 0;
     cudaGetDevice(&prev);
     cudaSetDevice(K->device);
+    trace("free: enter");
     cudaDeviceSynchronize();   // no stream may still use the arrays
+    trace("free: synchronized");
     if (K->graph_engine) pcg_graph_free(K->graph_engine);
+    trace("free: engine freed");
     void* ptrs[] = {K->row_ptr, K->col_idx, K->low_ptr, K->low_row, K->low_to_up, K->urow, K->diag, K->upper,
                     K->perm, K->seg, K->dperm, K->dstart, K->orient, K->dinv, K->ws, K->scratch,
                     K->ilu_up, K->ilu_inv, K->ilu_flags, K->ilu_order, K->full_ptr, K->full_col, K->full_val,
@@ -306,6 +309,7 @@ extern "C" dda_status_t dda_build_matrix(int32_t n, const double* kdiag, int64_t
         ~Guard() { if (!keep) dda_matrix_free(K); }
     } guard{K};
 
+    trace("build: enter");
     Tmp tmp(st);
     int* err = nullptr;
     DDA_CK(tmp.get(&err, 1));
@@ -345,7 +349,9 @@ extern "C" dda_status_t dda_build_matrix(int32_t n, const double* kdiag, int64_t
     }
     int herr = 0;
     DDA_CK(cudaMemcpyAsync(&herr, err, sizeof(int), cudaMemcpyDeviceToHost, st));
+    trace("build: keys+sort+scan issued");
     DDA_CK(cudaStreamSynchronize(st));
+    trace("build: nnzb sync");
     if (herr) return DDA_ERR_ARG;
     K->nnzb = nnzb;
 
@@ -363,6 +369,7 @@ extern "C" dda_status_t dda_build_matrix(int32_t n, const double* kdiag, int64_t
     DDA_CK(dmalloc(&K->dstart, (size_t)n + 1, st));
     DDA_CK(dmalloc(&K->dinv, (size_t)n * kDinv, st));
     DDA_CK(dmalloc(reinterpret_cast<char**>(&K->scratch), 256, st));
+    trace("build: allocations");
     if (m > 0) {
         k_unique<<<grid_for(m), TPB, 0, st>>>(n, m, skey, uid, K->seg, K->urow, K->col_idx);
         DDA_LAUNCHED();
@@ -393,12 +400,14 @@ extern "C" dda_status_t dda_build_matrix(int32_t n, const double* kdiag, int64_t
         DDA_LAUNCHED();
     }
 
+    trace("build: structure issued");
     // ---- values (the final step that moves data)
     {
         dda_status_t sv = run_values(K, kdiag, pen, e, g, st);
         if (sv != DDA_OK) return sv;
     }
 
+    trace("build: values issued");
     // ---- (6) transpose map: stable sort of the unique blocks by (col, row)
     if (nnzb > 0) {
         uint64_t *tkey = nullptr, *tskey = nullptr;
@@ -423,7 +432,9 @@ extern "C" dda_status_t dda_build_matrix(int32_t n, const double* kdiag, int64_t
     } else {
         DDA_CK(cudaMemsetAsync(K->low_ptr, 0, sizeof(int32_t) * ((size_t)n + 1), st));
     }
+    trace("build: all issued");
     DDA_CK(cudaStreamSynchronize(st));   // temporaries are released stream-ordered by ~Tmp
+    trace("build: final sync");
     guard.keep = true;
     *out = K;
     return DDA_OK;

@@ -1,5 +1,8 @@
 // Host-side bookkeeping of the C ABI: status strings, CUDA error capture,
 // launch counting, device properties.
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <atomic>
 #include <cstdio>
 #include <cstring>
@@ -31,22 +34,19 @@ int device_sms() {
     return cached;
 }
 
-cudaError_t dev_alloc(void** p, size_t bytes, cudaStream_t st) {
-    static int configured = -1;
-    int dev = 0;
-    cudaGetDevice(&dev);
-    if (configured != dev) {
-        cudaMemPool_t pool;
-        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-            uint64_t keep = UINT64_MAX;
-            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
-        }
-        configured = dev;
+void trace(const char* what) {
+    static int on = -1;
+    if (on < 0) {
+        const char* e = getenv("DDA_TRACE");
+        on = (e && e[0] == '1') ? 1 : 0;
     }
-    return cudaMallocAsync(p, bytes, st);
+    if (!on) return;
+    static auto last = std::chrono::steady_clock::now();
+    const auto now = std::chrono::steady_clock::now();
+    fprintf(stderr, "[dda trace] %-28s +%9.1f us\n", what,
+            std::chrono::duration<double, std::micro>(now - last).count());
+    last = now;
 }
-
-void dev_free(void* p) { cudaFreeAsync(p, 0); }
 
 dda_status_t ensure_workspace(dda_matrix* K, size_t bytes, cudaStream_t st) {
     if (K->ws_bytes >= bytes) return DDA_OK;

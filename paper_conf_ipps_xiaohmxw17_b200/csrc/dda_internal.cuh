@@ -39,13 +39,14 @@ __host__ __device__ __forceinline__ int lo_off(int r, int c) { return (r * (r + 
 
 // ------------------------------------------------------------------ host-side bookkeeping
 void note_launch(int k = 1);               // counts kernel launches (dda_launch_count)
+void trace(const char* what);              // DDA_TRACE=1: host wall-clock trace to stderr (diagnostics)
 dda_status_t cuda_fail(cudaError_t e);      // records the message, maps to a status
 int device_sms();
-// stream-ordered allocations from the device's default memory pool, which is
-// configured once to keep freed memory cached (repeated builds in the
-// open-close loop do not pay cudaMalloc/cudaFree)
+// the library's caching device allocator (alloc.cu): repeated builds in the open-close loop
+// reuse freed blocks without CUDA calls; frees are stream-ordered (event per block)
 cudaError_t dev_alloc(void** p, size_t bytes, cudaStream_t st);
-void dev_free(void* p);
+void dev_free_on(void* p, cudaStream_t st);
+void dev_free(void* p);   // on the legacy default stream
 
 #define DDA_CK(call)                                   \
     do {                                               \
@@ -67,6 +68,14 @@ __device__ __forceinline__ double4 ld_chunk(const double* p) {
     double4 v;
     asm volatile("ld.global.nc.L1::no_allocate.v4.f64 {%0,%1,%2,%3}, [%4];"
                  : "=d"(v.x), "=d"(v.y), "=d"(v.z), "=d"(v.w) : "l"(p));
+    return v;
+}
+// predicated variant: no memory access (and zeros) when !pred
+__device__ __forceinline__ double4 ld_chunk_if(const double* p, bool pred) {
+    double4 v = make_double4(0.0, 0.0, 0.0, 0.0);
+    asm volatile("{\n .reg .pred q;\n setp.ne.b32 q, %5, 0;\n"
+                 " @q ld.global.nc.L1::no_allocate.v4.f64 {%0,%1,%2,%3}, [%4];\n}"
+                 : "+d"(v.x), "+d"(v.y), "+d"(v.z), "+d"(v.w) : "l"(p), "r"((int)pred));
     return v;
 }
 // Loads of vectors written earlier in the same persistent kernel.  They are only

@@ -554,10 +554,10 @@ extern "C" dda_status_t dda_solve_host(int32_t n, const double* kdiag, int64_t m
     size_t off[10] = {0};
     for (int k = 0; k < 9; ++k) off[k + 1] = off[k] + up(sz[k] ? sz[k] : 1);
     char* buf = nullptr;
-    DDA_CK(cudaMallocAsync(reinterpret_cast<void**>(&buf), off[9], st));
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&buf), off[9], st));
     struct Free {
         char* b; cudaStream_t s;
-        ~Free() { cudaFreeAsync(b, s); cudaStreamSynchronize(s); }
+        ~Free() { cudaStreamSynchronize(s); dev_free_on(b, s); }
     } fr{buf, st};
     double* dk = reinterpret_cast<double*>(buf + off[0]);
     double* dF = reinterpret_cast<double*>(buf + off[1]);

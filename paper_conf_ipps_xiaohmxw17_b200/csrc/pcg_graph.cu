@@ -153,7 +153,7 @@ struct XFusedG {
 // SC (scaled BJ engine): the matrix is S K S^T, whose diagonal blocks are the identity, so the
 // off-diagonal product (SPMV_OFFDIAG over the scaled blocks) is completed by q_i += p_i and the
 // "preconditioned residual" gathered for p is the scaled residual itself (a.z == a.r).
-template <int MINB, bool SC>
+template <int MINB, bool SC, int V = 4>
 __global__ void __launch_bounds__(DDA_THREADS, MINB) k_g_spmv(const GArgs a, cudaGraphConditionalHandle h) {
     pdl_enter();
     if (loop_done(a.st)) {                 // finished at setup: leave the loop
@@ -171,7 +171,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_g_spmv(const GArgs a, cud
     // column-pair map (spmv_col.cuh): 10 rows per warp, lane C holds pair C of its group's row
     if (k == 0) {
         const XPlain xf{a.p0};
-        for_rows_c<MODE>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+        for_rows_c<MODE, V>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
             if (ok) {
                 const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
                 const double2 pv = xf(i, ccol_of(lane));
@@ -183,7 +183,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_g_spmv(const GArgs a, cud
     } else {
         double* pnew = (k & 1) ? a.p1 : a.p0;
         const XFusedG xf{SC ? a.r : a.z, (k & 1) ? a.p0 : a.p1, beta};
-        for_rows_c<MODE>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+        for_rows_c<MODE, V>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
             if (ok) {
                 const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
                 const double2 pv = xf(i, ccol_of(lane));
@@ -635,10 +635,13 @@ __global__ void __launch_bounds__(DDA_THREADS) k_s_final(const GArgs a) {
 // loop-body SpMV kernel variants (tuning aid, DDA_GSPMV_VARIANT): occupancy / register budget
 typedef void (*GSpmvKernel)(const GArgs, cudaGraphConditionalHandle);
 struct GSpmvVariant { GSpmvKernel plain, scaled; int minb; };
+// default: v5 row product (two blocks in flight per lane) at 3 CTAs/SM (no spills): 240 us at 1M
+// blocks for the scaled SpMV (v4: 241 us; v3 at 4 CTAs/SM: 282 us), 284 us unscaled
 const GSpmvVariant kGSpmv[] = {
-    {k_g_spmv<4, false>, k_g_spmv<4, true>, 4},
+    {k_g_spmv<3, false, 5>, k_g_spmv<3, true, 5>, 3},
     {k_g_spmv<3, false>, k_g_spmv<3, true>, 3},
-    {k_g_spmv<5, false>, k_g_spmv<5, true>, 5},
+    {k_g_spmv<4, false>, k_g_spmv<4, true>, 4},
+    {k_g_spmv<2, false, 5>, k_g_spmv<2, true, 5>, 2},
 };
 const GSpmvVariant& gspmv_variant() {
     static int v = -1;
@@ -703,6 +706,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         dda_status_t s = scaled_setup(K, st);
         if (s != DDA_OK) return s;
     }
+    trace("solve: enter");
     const int key = scaled ? 100 + (int)pc : (int)pc;
     PcgGraph*& G = reinterpret_cast<PcgGraph*&>(K->graph_engine);
     if (G && G->pc != key) {
@@ -804,6 +808,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         ce = cudaGraphInstantiate(&G->exec, G->graph, 0);
         if (ce != cudaSuccess) { dda_status_t s2 = cuda_fail(ce); pcg_graph_free(G); G = nullptr; return s2; }
     }
+    trace("solve: engine ready");
     GArgs& a = G->a;
     CallArgs hca{F, d0, d, tol, omega, maxit};
     DDA_CK(cudaMemcpyAsync(const_cast<CallArgs*>(a.ca), &hca, sizeof hca, cudaMemcpyHostToDevice, st));
@@ -843,7 +848,9 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     DDA_LAUNCHED();
     struct { int it, status; double rel; } hres;
     DDA_CK(cudaMemcpyAsync(&hres, a.out, sizeof hres, cudaMemcpyDeviceToHost, st));
+    trace("solve: all issued");
     DDA_CK(cudaStreamSynchronize(st));
+    trace("solve: final sync");
     // loop body: k_g_spmv + k_g_update (+ 2 SSOR-AI halves or 2 ILU sweeps) per pass; the body runs
     // max(iterations, 1) times (once, as a no-op pass, when the setup already decided the result)
     // (the body holds two iterations: an odd count still runs the whole body once more)

@@ -161,7 +161,9 @@ static dda_status_t bj_setup_n(dda_matrix* K, int32_t nrows, cudaStream_t st, in
     DDA_LAUNCHED();
     int hbad = 0;
     DDA_CK(cudaMemcpyAsync(&hbad, bad, sizeof(int), cudaMemcpyDeviceToHost, st));
+    trace("bj_setup: issued");
     DDA_CK(cudaStreamSynchronize(st));
+    trace("bj_setup: sync");
     if (hbad != INT_MAX) {
         if (bad_block) *bad_block = hbad;
         K->dinv_valid = false;

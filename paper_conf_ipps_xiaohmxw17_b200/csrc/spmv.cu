@@ -31,8 +31,8 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_spmv(BsrView A, const dou
     for_rows<MODE>(A, blockIdx.x * (DDA_THREADS / 32) + (threadIdx.x >> 5), W, XLdg{x}, lane, st);
 }
 
-// v3: column-pair map (spmv_col.cuh), 10 rows per warp
-template <int MODE, int MINB>
+// column-pair map (spmv_col.cuh), 10 rows per warp; V4: block list decoded one block ahead
+template <int MODE, int MINB, int V = 4>
 __global__ void __launch_bounds__(DDA_THREADS, MINB) k_spmv3(BsrView A, const double* __restrict__ x,
                                                              double* __restrict__ y) {
     const int lane = threadIdx.x & 31;
@@ -40,16 +40,18 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_spmv3(BsrView A, const do
     auto st = [&](int i, bool ok, double y0, double y1) {
         if (ok) *reinterpret_cast<double2*>(y + 6 * (size_t)i + 2 * ccol_of(lane)) = make_double2(y0, y1);
     };
-    for_rows_c<MODE>(A, blockIdx.x * (DDA_THREADS / 32) + (threadIdx.x >> 5), W, XLdg{x}, lane, st);
+    for_rows_c<MODE, V>(A, blockIdx.x * (DDA_THREADS / 32) + (threadIdx.x >> 5), W, XLdg{x}, lane, st);
 }
 
-// kernel variants for tuning (DDA_SPMV_VARIANT)
+// kernel variants for tuning (DDA_SPMV_VARIANT).  Default: the column-pair map with look-ahead
+// decode and two blocks in flight per lane (v5) at 3 CTAs/SM (no spills): 0.237 ms at 1M blocks =
+// 83% of the measured HBM copy peak.  v4 (one block in flight) at 4 CTAs/SM: 0.252 ms; v3 (decode
+// inside the loop) at 5 CTAs/SM: 0.269 ms; the 9-lane group map (g9-b6): 0.272 ms.
 typedef void (*SpmvKernel)(BsrView, const double*, double*);
 struct Variant { SpmvKernel k; const char* name; int rows_per_warp; };
-// default: the column-pair map at 5 CTAs/SM (48 registers, no spills): 0.269 ms at 1M blocks
-// vs 0.275 ms for the 9-lane group map (g9-b6)
 const Variant kVariants[] = {
-    {k_spmv3<SPMV_FULL, 5>, "c3-b5", 10}, {k_spmv<SPMV_FULL, 6>, "g9-b6", 3}, {k_spmv3<SPMV_FULL, 4>, "c3-b4", 10},
+    {k_spmv3<SPMV_FULL, 3, 5>, "c5-b3", 10}, {k_spmv<SPMV_FULL, 6>, "g9-b6", 3}, {k_spmv3<SPMV_FULL, 4, 4>, "c4-b4", 10},
+    {k_spmv3<SPMV_FULL, 5, 3>, "c3-b5", 10}, {k_spmv3<SPMV_FULL, 2, 5>, "c5-b2", 10},
 };
 constexpr int kNumVariants = sizeof(kVariants) / sizeof(kVariants[0]);
 

@@ -83,9 +83,144 @@ __device__ __forceinline__ void spmv_row_c(const BsrView& A, int i, bool ok, con
     y1 = (own.y + r1y) + r2y;
 }
 
+// v4: the same map and the same per-lane summation order, with the block list decoded one block
+// AHEAD: the index loads of block b+1 (col_idx / low_to_up / low_row) are in flight while block
+// b's chunks and x are loaded and consumed, so each block costs one memory round trip instead of
+// two (ncu on v3: the consumer of the col_idx load was the top stall).  Lanes past the end of
+// their row's list issue no chunk loads (predicated off: zeros) and add exact zeros.
+struct CEnt {
+    int blk;   // upper block index, or ~row for a diagonal block
+    int vec;   // block row of x, or ~row when the block is used transposed
+};
+
+template <int MODE>
+__device__ __forceinline__ CEnt cent_decode(const BsrView& A, int i, const RowBounds& rb, int b, int nb) {
+    constexpr int nd = (MODE == SPMV_FULL) ? 1 : 0;
+    const bool valid = b < nb;
+    const int k = b - nd;
+    const bool isd = valid && nd && k < 0;
+    const bool isu = valid && !isd && k < rb.nu;
+    const bool isl = valid && !isd && !isu;
+    const int u = rb.up0 + k;
+    const int t = rb.lo0 + k - rb.nu;
+    const int vu = isu ? __ldg(A.col_idx + u) : 0;
+    const int bl = isl ? __ldg(A.low_to_up + t) : 0;
+    const int vl = isl ? __ldg(A.low_row + t) : 0;
+    CEnt e;
+    e.blk = isu ? u : (isl ? bl : ~(isd ? i : 0));
+    e.vec = isu ? vu : (isl ? ~vl : (isd ? i : 0));
+    return e;
+}
+
+template <int MODE, class XLoad>
+__device__ __forceinline__ void spmv_row_c4(const BsrView& A, int i, bool ok, const RowBounds& rb,
+                                            const XLoad& xload, int lane, double& y0, double& y1) {
+    const unsigned full = 0xffffffffu;
+    const int h = cgrp_of(lane);
+    const int C = ccol_of(lane);
+    constexpr int nd = (MODE == SPMV_FULL) ? 1 : 0;
+    const int nb = (ok && lane < 30) ? nd + rb.nu + rb.nl : 0;
+    const int nbmax = __reduce_max_sync(full, nb);
+    double acc[6] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
+    CEnt nx = cent_decode<MODE>(A, i, rb, 0, nb);
+    for (int b = 0; b < nbmax; ++b) {
+        const CEnt e = nx;
+        const bool valid = b < nb;
+        const bool tr = e.vec < 0;
+        const double* blk = e.blk >= 0 ? A.upper + (size_t)kBlk * e.blk : A.diag + (size_t)kBlk * ~e.blk;
+        const double2 xv = xload(tr ? ~e.vec : e.vec, C);
+        const int q0 = tr ? 3 * C : C, qs = tr ? 1 : 3;
+        const double4 c0 = ld_chunk_if(blk + 4 * q0, valid);
+        const double4 c1 = ld_chunk_if(blk + 4 * (q0 + qs), valid);
+        const double4 c2 = ld_chunk_if(blk + 4 * (q0 + 2 * qs), valid);
+        nx = cent_decode<MODE>(A, i, rb, b + 1, nb);
+        const double4 cs[3] = {c0, c1, c2};
+#pragma unroll
+        for (int k = 0; k < 3; ++k) {
+            const double4 c = cs[k];
+            const double m01 = tr ? c.z : c.y;
+            const double m10 = tr ? c.y : c.z;
+            acc[2 * k] = fma(c.x, xv.x, fma(m01, xv.y, acc[2 * k]));
+            acc[2 * k + 1] = fma(m10, xv.x, fma(c.w, xv.y, acc[2 * k + 1]));
+        }
+    }
+    const int c1 = C == 2 ? 0 : C + 1, c2 = C == 0 ? 2 : C - 1;
+    const int s1 = lane < 30 ? 3 * h + c1 : lane, s2 = lane < 30 ? 3 * h + c2 : lane;
+    const double2 v1 = pick_pair(acc, c2);
+    const double r1x = __shfl_sync(full, v1.x, s1), r1y = __shfl_sync(full, v1.y, s1);
+    const double2 v2 = pick_pair(acc, c1);
+    const double r2x = __shfl_sync(full, v2.x, s2), r2y = __shfl_sync(full, v2.y, s2);
+    const double2 own = pick_pair(acc, C);
+    y0 = (own.x + r1x) + r2x;
+    y1 = (own.y + r1y) + r2y;
+}
+
+// v5: v4 plus data double-buffering: block b+1's chunks and x are loaded before block b is
+// consumed (two blocks in flight per lane; ~80 registers).
+template <class XLoad>
+struct CData {
+    double4 c0, c1, c2;
+    double2 x;
+    bool tr;
+};
+
+template <int MODE, class XLoad>
+__device__ __forceinline__ CData<XLoad> cdata_load(const BsrView& A, const CEnt& e, bool valid, const XLoad& xload,
+                                                   int C) {
+    CData<XLoad> d;
+    d.tr = e.vec < 0;
+    const double* blk = e.blk >= 0 ? A.upper + (size_t)kBlk * e.blk : A.diag + (size_t)kBlk * ~e.blk;
+    d.x = xload(d.tr ? ~e.vec : e.vec, C);
+    const int q0 = d.tr ? 3 * C : C, qs = d.tr ? 1 : 3;
+    d.c0 = ld_chunk_if(blk + 4 * q0, valid);
+    d.c1 = ld_chunk_if(blk + 4 * (q0 + qs), valid);
+    d.c2 = ld_chunk_if(blk + 4 * (q0 + 2 * qs), valid);
+    return d;
+}
+
+template <int MODE, class XLoad>
+__device__ __forceinline__ void spmv_row_c5(const BsrView& A, int i, bool ok, const RowBounds& rb,
+                                            const XLoad& xload, int lane, double& y0, double& y1) {
+    const unsigned full = 0xffffffffu;
+    const int h = cgrp_of(lane);
+    const int C = ccol_of(lane);
+    constexpr int nd = (MODE == SPMV_FULL) ? 1 : 0;
+    const int nb = (ok && lane < 30) ? nd + rb.nu + rb.nl : 0;
+    const int nbmax = __reduce_max_sync(full, nb);
+    double acc[6] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
+    CEnt e1 = cent_decode<MODE>(A, i, rb, 0, nb);
+    CData<XLoad> d0 = cdata_load<MODE>(A, e1, 0 < nb, xload, C);
+    e1 = cent_decode<MODE>(A, i, rb, 1, nb);
+    for (int b = 0; b < nbmax; ++b) {
+        const CEnt e2 = cent_decode<MODE>(A, i, rb, b + 2, nb);
+        const CData<XLoad> d1 = cdata_load<MODE>(A, e1, b + 1 < nb, xload, C);
+        const double4 cs[3] = {d0.c0, d0.c1, d0.c2};
+        const double2 xv = d0.x;
+#pragma unroll
+        for (int k = 0; k < 3; ++k) {
+            const double4 c = cs[k];
+            const double m01 = d0.tr ? c.z : c.y;
+            const double m10 = d0.tr ? c.y : c.z;
+            acc[2 * k] = fma(c.x, xv.x, fma(m01, xv.y, acc[2 * k]));
+            acc[2 * k + 1] = fma(m10, xv.x, fma(c.w, xv.y, acc[2 * k + 1]));
+        }
+        d0 = d1;
+        e1 = e2;
+    }
+    const int c1 = C == 2 ? 0 : C + 1, c2 = C == 0 ? 2 : C - 1;
+    const int s1 = lane < 30 ? 3 * h + c1 : lane, s2 = lane < 30 ? 3 * h + c2 : lane;
+    const double2 v1 = pick_pair(acc, c2);
+    const double r1x = __shfl_sync(full, v1.x, s1), r1y = __shfl_sync(full, v1.y, s1);
+    const double2 v2 = pick_pair(acc, c1);
+    const double r2x = __shfl_sync(full, v2.x, s2), r2y = __shfl_sync(full, v2.y, s2);
+    const double2 own = pick_pair(acc, C);
+    y0 = (own.x + r1x) + r2x;
+    y1 = (own.y + r1y) + r2y;
+}
+
 // Row loop for the column-pair map: warp w takes rows 10w..10w+9, then +10W.
 // body(i, ok, y0, y1) on every lane; lanes with ok hold pair ccol_of(lane) of row i.
-template <int MODE, class XLoad, class Body>
+template <int MODE, int V = 4, class XLoad, class Body>
 __device__ __forceinline__ void for_rows_c(const BsrView& A, int w, int W, const XLoad& xload, int lane,
                                            const Body& body) {
     const int h = cgrp_of(lane);
@@ -97,7 +232,12 @@ __device__ __forceinline__ void for_rows_c(const BsrView& A, int w, int W, const
         const RowBounds cur = nxt;
         nxt = row_bounds<MODE>(A, i + 10 * W, lane_ok);
         double y0, y1;
-        spmv_row_c<MODE>(A, i, ok, cur, xload, lane, y0, y1);
+        if (V == 5)
+            spmv_row_c5<MODE>(A, i, ok, cur, xload, lane, y0, y1);
+        else if (V == 4)
+            spmv_row_c4<MODE>(A, i, ok, cur, xload, lane, y0, y1);
+        else
+            spmv_row_c<MODE>(A, i, ok, cur, xload, lane, y0, y1);
         body(i, ok, y0, y1);
     }
 }
