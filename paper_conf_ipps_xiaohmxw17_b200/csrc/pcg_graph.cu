@@ -131,20 +131,29 @@ __device__ __forceinline__ bool grid_reduce_last(const GArgs& a, double (&v)[NV]
 
 struct XPlain {
     const double* __restrict__ x;
-    __device__ __forceinline__ double2 operator()(int vec, int pair) const {
+    using Raw = double2;
+    __device__ __forceinline__ Raw raw(int vec, int pair) const {
         return __ldg(reinterpret_cast<const double2*>(x + 6 * (size_t)vec + 2 * pair));
     }
+    __device__ __forceinline__ double2 cook(const Raw& r) const { return r; }
+    __device__ __forceinline__ double2 operator()(int vec, int pair) const { return raw(vec, pair); }
 };
+// x = z + beta p_old, formed on the fly for every gathered neighbour (the fused p-update).  Formed
+// at load time (Raw = the combined pair): keeping z and p raw until the block is consumed costs 8
+// registers and measured slower (250 vs 240 us at 1M blocks, scaled engine).
 struct XFusedG {
     const double* __restrict__ z;
     const double* __restrict__ p;
     double beta;
-    __device__ __forceinline__ double2 operator()(int vec, int pair) const {
+    using Raw = double2;
+    __device__ __forceinline__ Raw raw(int vec, int pair) const {
         const size_t o = 6 * (size_t)vec + 2 * pair;
         const double2 zz = __ldg(reinterpret_cast<const double2*>(z + o));
         const double2 pp = __ldg(reinterpret_cast<const double2*>(p + o));
         return make_double2(fma(beta, pp.x, zz.x), fma(beta, pp.y, zz.y));
     }
+    __device__ __forceinline__ double2 cook(const Raw& r) const { return r; }
+    __device__ __forceinline__ double2 operator()(int vec, int pair) const { return raw(vec, pair); }
 };
 
 // ---------------------------------------------------------------- loop body
@@ -574,7 +583,7 @@ __global__ void __launch_bounds__(DDA_THREADS) k_s_init(const GArgs a) {
 }
 
 // phase B: x += alpha p~ (in d); r~ -= alpha q~; rr = |L r~|^2 (the original residual), rz = |r~|^2
-__global__ void __launch_bounds__(DDA_THREADS) k_s_update(const GArgs a, cudaGraphConditionalHandle h) {
+__global__ void __launch_bounds__(DDA_THREADS, 4) k_s_update(const GArgs a, cudaGraphConditionalHandle h) {
     pdl_enter();
     if (loop_done(a.st)) return;
     const int k = a.st->k;
@@ -653,6 +662,11 @@ const GSpmvVariant& gspmv_variant() {
     return kGSpmv[v];
 }
 
+int env_int(const char* name, int dflt) {
+    const char* e = getenv(name);
+    return e ? atoi(e) : dflt;
+}
+
 int occ_grid(const void* k, int minb_cap) {
     int per_sm = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, DDA_THREADS, 0);
@@ -671,6 +685,7 @@ struct PcgGraph {
     cudaGraph_t graph = nullptr;
     cudaGraphConditionalHandle h = 0;
     int G_spmv = 0, G_vec = 0, g_ilu = 0;
+    int body_iters = 2;
 };
 
 void pcg_graph_free(void* p) {
@@ -719,7 +734,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         int g_spmv = occ_grid(scaled ? (const void*)gv.scaled : (const void*)gv.plain, gv.minb);
         if (g_spmv > need_rows) g_spmv = need_rows > 0 ? need_rows : 1;
         const int need_vec = ((K->n + 4) / 5 + WPB - 1) / WPB;
-        int g_vec = occ_grid((const void*)k_g_update, 8);
+        int g_vec = occ_grid(scaled ? (const void*)k_s_update : (const void*)k_g_update, 8);
         if (g_vec > need_vec) g_vec = need_vec > 0 ? need_vec : 1;
         int Gmax = g_spmv > g_vec ? g_spmv : g_vec;
         if (ilu_grid() > Gmax) Gmax = ilu_grid();
@@ -774,7 +789,11 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         // body = two PCG iterations; kernels chained with programmatic dependent launch
         cudaLaunchAttribute pdl[1];
         pdl[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-        pdl[0].val.programmaticStreamSerializationAllowed = 1;
+        pdl[0].val.programmaticStreamSerializationAllowed = env_int("DDA_PDL", 1) ? 1 : 0;
+        // iterations per while-loop pass (tuning aid); the kernels exit early once the loop is done
+        int body_iters = env_int("DDA_BODY_ITERS", 2);
+        if (body_iters < 1 || body_iters > 16) body_iters = 2;
+        G->body_iters = body_iters;
         auto launch = [&](auto kern, int grid, auto... args) {
             cudaLaunchConfig_t cfg = {};
             cfg.gridDim = dim3(grid);
@@ -784,7 +803,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
             cfg.numAttrs = 1;
             cudaLaunchKernelEx(&cfg, kern, args...);
         };
-        for (int rep = 0; rep < 2; ++rep) {
+        for (int rep = 0; rep < body_iters; ++rep) {
             if (scaled) {
                 launch(gspmv_variant().scaled, G->G_spmv, a, G->h);
                 launch(k_s_update, G->G_vec, a, G->h);
@@ -851,11 +870,12 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     trace("solve: all issued");
     DDA_CK(cudaStreamSynchronize(st));
     trace("solve: final sync");
-    // loop body: k_g_spmv + k_g_update (+ 2 SSOR-AI halves or 2 ILU sweeps) per pass; the body runs
-    // max(iterations, 1) times (once, as a no-op pass, when the setup already decided the result)
-    // (the body holds two iterations: an odd count still runs the whole body once more)
+    // loop body: k_g_spmv + k_g_update (+ 2 SSOR-AI halves or 2 ILU sweeps) per iteration, body_iters
+    // iterations per pass; the body runs ceil(max(iterations, 1) / body_iters) times (once, as a no-op
+    // pass, when the setup already decided the result); every kernel of a pass is launched
     const int per_it = (pc == DDA_PC_SSOR_AI || pc == DDA_PC_ILU0) ? 4 : 2;
-    note_launch(per_it * 2 * ((hres.it > 0 ? hres.it : 1) + 1) / 2);
+    const int its = hres.it > 0 ? hres.it : 1;
+    note_launch(per_it * G->body_iters * ((its + G->body_iters - 1) / G->body_iters));
     if (iters) *iters = hres.it;
     if (rel_res) *rel_res = hres.rel;
     return (dda_status_t)hres.status;

@@ -14,9 +14,12 @@ namespace {
 
 struct XLdg {
     const double* __restrict__ x;
-    __device__ __forceinline__ double2 operator()(int vec, int pair) const {
+    using Raw = double2;
+    __device__ __forceinline__ Raw raw(int vec, int pair) const {
         return __ldg(reinterpret_cast<const double2*>(x + 6 * (size_t)vec + 2 * pair));
     }
+    __device__ __forceinline__ double2 cook(const Raw& r) const { return r; }
+    __device__ __forceinline__ double2 operator()(int vec, int pair) const { return raw(vec, pair); }
 };
 
 template <int MODE, int MINB>

@@ -156,11 +156,13 @@ __device__ __forceinline__ void spmv_row_c4(const BsrView& A, int i, bool ok, co
 }
 
 // v5: v4 plus data double-buffering: block b+1's chunks and x are loaded before block b is
-// consumed (two blocks in flight per lane; ~80 registers).
+// consumed (two blocks in flight per lane; ~80 registers).  XLoad::raw loads the x operand and
+// XLoad::cook finishes it when the block is consumed (the functor decides how much work is
+// deferred; see XFusedG in pcg_graph.cu).
 template <class XLoad>
 struct CData {
     double4 c0, c1, c2;
-    double2 x;
+    typename XLoad::Raw x;
     bool tr;
 };
 
@@ -170,7 +172,7 @@ __device__ __forceinline__ CData<XLoad> cdata_load(const BsrView& A, const CEnt&
     CData<XLoad> d;
     d.tr = e.vec < 0;
     const double* blk = e.blk >= 0 ? A.upper + (size_t)kBlk * e.blk : A.diag + (size_t)kBlk * ~e.blk;
-    d.x = xload(d.tr ? ~e.vec : e.vec, C);
+    d.x = xload.raw(d.tr ? ~e.vec : e.vec, C);
     const int q0 = d.tr ? 3 * C : C, qs = d.tr ? 1 : 3;
     d.c0 = ld_chunk_if(blk + 4 * q0, valid);
     d.c1 = ld_chunk_if(blk + 4 * (q0 + qs), valid);
@@ -195,7 +197,7 @@ __device__ __forceinline__ void spmv_row_c5(const BsrView& A, int i, bool ok, co
         const CEnt e2 = cent_decode<MODE>(A, i, rb, b + 2, nb);
         const CData<XLoad> d1 = cdata_load<MODE>(A, e1, b + 1 < nb, xload, C);
         const double4 cs[3] = {d0.c0, d0.c1, d0.c2};
-        const double2 xv = d0.x;
+        const double2 xv = xload.cook(d0.x);
 #pragma unroll
         for (int k = 0; k < 3; ++k) {
             const double4 c = cs[k];
