@@ -81,18 +81,22 @@ def pcg_launch_bytes(n: int, u: float, iters: int) -> float:
     return n * (432.0 + (S + 528.0) + (it - 1) * (S + 96.0 + 528.0) + S + 96.0)
 
 
-def pcg_launch_bytes_scaled(n: int, nnzb: int, iters: int) -> float:
+def pcg_launch_bytes_scaled(n: int, nnzb: int, iters: int, checks: int) -> float:
     """Algorithmic bytes of one dda_pcg_solve on the scaled block-Jacobi engine, d0 = 0
-    (DESIGN.md §6): k_scale_upper nnzb*(288 V read + 288 written + 8 indices) + n*192 (S);
-    k_s_init 384 B/row (F, S read; r~, p, x written); iteration 0: scaled SpMV 300u + 8 + 96
-    (p read, q written) + update 480 (p, x, r~, q~, L read; x, r~ written); iterations k >= 1: the
-    SpMV also reads p_old (+48) and writes p (+48); k_s_final 288 (x, S read; d written); the
-    true-residual SpMV on K + 96 (F, q read)."""
+    (DESIGN.md §6), per block row unless noted:
+    k_scale_upper: nnzb*(288 V read + 288 written + 8 indices) + n*192 (S);
+    k_s_init 384 (F, S read; r~, p, x written);
+    iteration 0: scaled SpMV 300u + 8 + 96 (p read, q written) + k_s_update 144 (r~, q read; r~ written);
+    iterations k >= 1: the SpMV also reads p_old (+48), writes p (+48) and applies the deferred
+    x += alpha p_old (x read + written, +96) + k_s_update 144;
+    each exact stopping test (k_s_check, `checks` of them) 240 (r~ + L read);
+    k_s_final 336 (x, p, S read; d written); the true-residual SpMV on K + 96 (F, q read)."""
     u = nnzb / n
     it = max(iters, 1)
     sp = 300.0 * u + 8.0 + 96.0
     return (nnzb * 584.0 + n * 192.0
-            + n * (384.0 + (sp + 480.0) + (it - 1) * (sp + 96.0 + 480.0) + 288.0 + bytes_per_row_spmv(u) + 96.0))
+            + n * (384.0 + (sp + 144.0) + (it - 1) * (sp + 192.0 + 144.0) + 240.0 * checks + 336.0
+                   + bytes_per_row_spmv(u) + 96.0))
 
 
 class ClockSampler:
@@ -275,6 +279,7 @@ def main():
     for _ in range(args.warmup):
         K, d, it, rr, st = step()
         engine = K.pcg_engine(args.precond)
+        checks = K.last_checks()
         K.free()
     torch.cuda.synchronize()
 
@@ -309,9 +314,10 @@ def main():
     u = nnzb / n
     pcg_ms = statistics.mean(ph_pcg)
     if engine == "scaled":
-        pcg_bytes = pcg_launch_bytes_scaled(n, nnzb, iters)
+        pcg_bytes = pcg_launch_bytes_scaled(n, nnzb, iters, checks)
         pcg_kernel = ("dda_pcg_solve, scaled block-Jacobi engine: k_scale_upper (S_i V_ij S_j^T) + one CUDA-graph "
-                      "while loop (k_g_spmv<SC> + k_s_update per iteration) with its prelude/epilogue kernels")
+                      "while loop (k_g_spmv<SC> + k_s_update + k_s_check per iteration) with its prelude/epilogue "
+                      f"kernels; {checks} exact stopping tests")
     else:
         pcg_bytes = pcg_launch_bytes(n, u, iters)
         pcg_kernel = ("dda_pcg_solve: one CUDA-graph while loop (k_g_spmv + k_g_update per iteration) with its "

@@ -99,6 +99,8 @@ def lib() -> C.CDLL:
         L.dda_memory_release.restype = None
         L.dda_memory_cached.argtypes = []
         L.dda_memory_cached.restype = I64
+        L.dda__last_checks.argtypes = [P]
+        L.dda__last_checks.restype = C.c_int
         L.dda__pcg_engine.argtypes = [P, C.c_int]
         L.dda__pcg_engine.restype = C.c_int
         _lib = L
@@ -244,6 +246,10 @@ class Matrix:
     def pcg_engine(self, precond="bj") -> str:
         """The PCG engine dda_pcg_solve picks for this matrix (internal query, for byte accounting)."""
         return {0: "graph", 1: "persistent", 2: "scaled"}[lib().dda__pcg_engine(self.handle, PRECOND[precond])]
+
+    def last_checks(self) -> int:
+        """Exact stopping tests the last scaled-engine solve evaluated (internal query, byte accounting)."""
+        return int(lib().dda__last_checks(self.handle))
 
     def update_values(self, kdiag, pen, e, g, stream=None):
         torch = _torch()

@@ -141,6 +141,7 @@ struct dda_matrix {
     int32_t* full_col = nullptr;
     double* full_val = nullptr;
     int64_t graph_iters = 0;        // loop-body launches issued inside graphs (launch accounting)
+    int last_checks = 0;            // scaled engine: exact stopping tests in the last solve
 };
 
 namespace dda {

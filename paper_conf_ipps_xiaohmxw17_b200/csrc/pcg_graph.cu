@@ -41,6 +41,12 @@ struct State {
     double rho, beta, alpha, FF, bnorm, rr, rel;
     int k, done, status, iters, zero_d;
     unsigned ticket;
+    // scaled engine: lam = a lower bound of min_i lambda_min(D_i); maybe = the exact stopping test
+    // is due (k_s_check); pend_rz = the new rho waiting for it
+    double lam, pend_rz;
+    int maybe;
+    int checks;   // exact stopping tests evaluated (k_s_check passes that did work)
+    int pend;   // scaled engine: x += alpha p of the last k_s_update still to apply (k_s_final)
 };
 
 struct GArgs {           // constant for a (matrix, preconditioner): baked into the graph
@@ -62,6 +68,7 @@ struct GArgs {           // constant for a (matrix, preconditioner): baked into 
     const double* su;    // scaled BJ engine: S_i V_ij S_j^T (tiled, upper pattern)
     const double* lfac;  // packed lower L_i (D_i = L_i L_i^T)
     const double* sfac;  // packed lower S_i = L_i^{-1}
+    const unsigned long long* dinv_fmax;   // bits of max_i ||D_i^{-1}||_F (bj_setup)
     int use_cond;        // 0 only for the internal phase-timing hook (kernels launched outside the graph)
 };
 
@@ -191,12 +198,24 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_g_spmv(const GArgs a, cud
         });
     } else {
         double* pnew = (k & 1) ? a.p1 : a.p0;
-        const XFusedG xf{SC ? a.r : a.z, (k & 1) ? a.p0 : a.p1, beta};
+        const double* pold = (k & 1) ? a.p0 : a.p1;
+        const XFusedG xf{SC ? a.r : a.z, pold, beta};
+        // scaled engine: the solution update of the previous iteration, x += alpha_{k-1} p_{k-1}, is
+        // applied here for the own rows (p_{k-1} is read here anyway), not in k_s_update
+        const double alpha_prev = a.st->alpha;
+        double* x = a.ca->d;
         for_rows_c<MODE, V>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
             if (ok) {
                 const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
                 const double2 pv = xf(i, ccol_of(lane));
-                if (SC) { y0 += pv.x; y1 += pv.y; }
+                if (SC) {
+                    y0 += pv.x;
+                    y1 += pv.y;
+                    const double2 po = __ldg(reinterpret_cast<const double2*>(pold + o));
+                    const double2 xo = *reinterpret_cast<const double2*>(x + o);
+                    *reinterpret_cast<double2*>(x + o) = make_double2(xo.x + alpha_prev * po.x,
+                                                                      xo.y + alpha_prev * po.y);
+                }
                 *reinterpret_cast<double2*>(a.q + o) = make_double2(y0, y1);
                 *reinterpret_cast<double2*>(pnew + o) = pv;
                 acc += pv.x * y0 + pv.y * y1;
@@ -206,6 +225,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_g_spmv(const GArgs a, cud
     double v[1] = {acc}, tot[1];
     if (grid_reduce_last<1>(a, v, tot) && threadIdx.x == 0) {
         State* st = a.st;
+        st->pend = 0;                                      // the pending solution update is applied
         const double sigma = tot[0];
         if (!(sigma > 0.0) || !isfinite(sigma)) {          // reading Z19: d stays the last iterate
             st->status = DDA_ERR_BREAKDOWN;
@@ -410,6 +430,10 @@ __device__ __noinline__ void init_decide(const GArgs& a, const double (&tot)[3])
         st->rel = 0.0;
         st->zero_d = 0;
         st->done = 0;
+        st->maybe = 0;
+        st->checks = 0;
+        st->pend = 0;
+        st->pend_rz = 0.0;
         st->status = DDA_ERR_NO_CONVERGENCE;
         if (tot[0] == 0.0) {                                   // reading Z2
             st->zero_d = 1; st->status = DDA_OK; st->done = 1;
@@ -461,6 +485,7 @@ __global__ void __launch_bounds__(DDA_THREADS) k_g_resid(const GArgs a) {
         a.out[0] = st->iters;
         a.out[1] = st->status;
         *reinterpret_cast<double*>(a.out + 2) = st->rel;
+        a.out[4] = st->checks;
     }
 }
 
@@ -579,62 +604,107 @@ __global__ void __launch_bounds__(DDA_THREADS) k_s_init(const GArgs a) {
         rz += rt * rt;
     }
     double v[3] = {FF, rr, rz}, tot[3];
-    if (grid_reduce_last<3>(a, v, tot) && threadIdx.x == 0) init_decide(a, tot);
+    if (grid_reduce_last<3>(a, v, tot) && threadIdx.x == 0) {
+        init_decide(a, tot);
+        const double lam = 1.0 / __longlong_as_double((long long)*a.dinv_fmax);
+        a.st->lam = (isfinite(lam) && lam > 0.0) ? lam : 0.0;   // 0: the exact test in every iteration
+    }
 }
 
-// phase B: x += alpha p~ (in d); r~ -= alpha q~; rr = |L r~|^2 (the original residual), rz = |r~|^2
+// phase B: r~ -= alpha q~; rho' = |r~|^2 (x += alpha p~ is applied by the next SpMV or k_s_final).
+// The stopping test (reading Z1) is on the ORIGINAL residual r = L r~, whose norm costs the packed
+// L_i (192 B per row).  It is evaluated only when it can succeed: |L r~|^2 >= lam |r~|^2 with
+// lam = min_i lambda_min(D_i) >= 1 / max_i ||D_i^{-1}||_F, so while 0.999 lam rho' > tol^2 ||F||^2
+// the iteration cannot have converged and L is not read.  Otherwise k_s_check evaluates |L r~|
+// exactly (the decision, the iteration count and the solution are those of the plain test).
 __global__ void __launch_bounds__(DDA_THREADS, 4) k_s_update(const GArgs a, cudaGraphConditionalHandle h) {
     pdl_enter();
     if (loop_done(a.st)) return;
     const int k = a.st->k;
     const double alpha = a.st->alpha;
-    const double* pk = (k & 1) ? a.p1 : a.p0;
-    double* d = a.ca->d;
     const int lane = threadIdx.x & 31;
     const int n = a.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
-    double rr = 0.0, rz = 0.0;
+    double rz = 0.0;
     for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += 2 * W) {
         const Row5 RA = row5(grp, lane, n);
         const Row5 RB = row5(grp + W, lane, n);
-        double pa = 0, da = 0, ra = 0, qa = 0, pb = 0, db = 0, rb = 0, qb = 0;
-        if (RA.valid) { pa = pk[RA.idx]; da = d[RA.idx]; ra = a.r[RA.idx]; qa = a.q[RA.idx]; }
-        if (RB.valid) { pb = pk[RB.idx]; db = d[RB.idx]; rb = a.r[RB.idx]; qb = a.q[RB.idx]; }
-        const DinvRow LA = tri_row(a.lfac, RA), LB = tri_row(a.lfac, RB);
+        double ra = 0, qa = 0, rb = 0, qb = 0;
+        if (RA.valid) { ra = a.r[RA.idx]; qa = a.q[RA.idx]; }
+        if (RB.valid) { rb = a.r[RB.idx]; qb = a.q[RB.idx]; }
         const double rva = RA.valid ? ra - alpha * qa : 0.0;
         const double rvb = RB.valid ? rb - alpha * qb : 0.0;
-        if (RA.valid) { d[RA.idx] = da + alpha * pa; a.r[RA.idx] = rva; }
-        if (RB.valid) { d[RB.idx] = db + alpha * pb; a.r[RB.idx] = rvb; }
+        if (RA.valid) a.r[RA.idx] = rva;
+        if (RB.valid) a.r[RB.idx] = rvb;
         rz += rva * rva + rvb * rvb;
-        const double oa0 = dinv_row_apply(LA, rva, RA);   // L r~ (invalid lanes masked below)
-        const double ob0 = dinv_row_apply(LB, rvb, RB);
-        const double oa = RA.valid ? oa0 : 0.0, ob = RB.valid ? ob0 : 0.0;
-        rr += oa * oa + ob * ob;
     }
-    double v[2] = {rr, rz}, tot[2];
-    if (grid_reduce_last<2>(a, v, tot) && threadIdx.x == 0) {
+    double v[1] = {rz}, tot[1];
+    if (grid_reduce_last<1>(a, v, tot) && threadIdx.x == 0) {
         State* st = a.st;
-        st->rr = tot[0];
+        st->pend = 1;                                       // x += alpha p_k: next SpMV or k_s_final
+        const double rho1 = tot[0];
         st->iters = k + 1;
-        if (sqrt(tot[0]) <= a.ca->tol * st->bnorm) {
+        const double thr = a.ca->tol * st->bnorm;
+        if (rho1 == 0.0) {                                  // r~ = 0 exactly: r = L r~ = 0
+            st->rr = 0.0;
             st->status = DDA_OK;
             st->k = k + 1;
             st->done = 1;
             set_cond(a, h, 0);
+        } else if (isfinite(rho1) && 0.999 * st->lam * rho1 <= thr * thr) {
+            st->maybe = 1;                                  // k_s_check decides
+            st->pend_rz = rho1;
         } else {
-            finish_iteration(a, tot[1], h);
+            finish_iteration(a, rho1, h);                   // cannot have converged (or breakdown)
         }
     }
 }
 
-// epilogue: d = S^T x in place (before the true residual)
+// the exact stopping test |L r~| <= tol ||F|| when k_s_update flagged it; then beta / the loop
+// condition as k_s_update would have set them
+__global__ void __launch_bounds__(DDA_THREADS, 4) k_s_check(const GArgs a, cudaGraphConditionalHandle h) {
+    pdl_enter();
+    if (loop_done(a.st) || !*reinterpret_cast<volatile const int*>(&a.st->maybe)) return;
+    const int lane = threadIdx.x & 31;
+    const int n = a.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    double rr = 0.0;
+    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        const double rv = R.valid ? a.r[R.idx] : 0.0;
+        const DinvRow Lrow = tri_row(a.lfac, R);
+        const double o0 = dinv_row_apply(Lrow, rv, R);
+        const double o = R.valid ? o0 : 0.0;
+        rr += o * o;
+    }
+    double v[1] = {rr}, tot[1];
+    if (grid_reduce_last<1>(a, v, tot) && threadIdx.x == 0) {
+        State* st = a.st;
+        st->maybe = 0;
+        st->checks += 1;
+        st->rr = tot[0];
+        if (sqrt(tot[0]) <= a.ca->tol * st->bnorm) {
+            st->status = DDA_OK;
+            st->k = st->k + 1;
+            st->done = 1;
+            set_cond(a, h, 0);
+        } else {
+            finish_iteration(a, st->pend_rz, h);
+        }
+    }
+}
+
+// epilogue: the pending x += alpha p of the last iteration, then d = S^T x in place (before the
+// true residual)
 __global__ void __launch_bounds__(DDA_THREADS) k_s_final(const GArgs a) {
     if (a.st->zero_d) return;
     double* d = a.ca->d;
+    const bool pend = a.st->pend;
+    const double alpha = a.st->alpha;
+    const double* pk = ((a.st->k - 1) & 1) ? a.p1 : a.p0;   // p of the last k_s_update (iteration k-1)
     const int lane = threadIdx.x & 31;
     const int n = a.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
     for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
         const Row5 R = row5(grp, lane, n);
-        const double xv = R.valid ? d[R.idx] : 0.0;
+        const double xv = R.valid ? (pend ? d[R.idx] + alpha * pk[R.idx] : d[R.idx]) : 0.0;
         const DinvRow Scol = tri_col(a.sfac, R);
         const double dv = dinv_row_apply(Scol, xv, R);
         if (R.valid) d[R.idx] = dv;
@@ -644,8 +714,9 @@ __global__ void __launch_bounds__(DDA_THREADS) k_s_final(const GArgs a) {
 // loop-body SpMV kernel variants (tuning aid, DDA_GSPMV_VARIANT): occupancy / register budget
 typedef void (*GSpmvKernel)(const GArgs, cudaGraphConditionalHandle);
 struct GSpmvVariant { GSpmvKernel plain, scaled; int minb; };
-// default: v5 row product (two blocks in flight per lane) at 3 CTAs/SM (no spills): 240 us at 1M
-// blocks for the scaled SpMV (v4: 241 us; v3 at 4 CTAs/SM: 282 us), 284 us unscaled
+// default: v5 row product (look-ahead decode, two blocks in flight) at 3 CTAs/SM (no spills): 317.6
+// us per whole scaled-engine iteration at 1M blocks vs 330.8 with v4 (one block in flight) since the
+// SpMV also applies the deferred x += alpha p; v3 at 4 CTAs/SM: 282 us for the SpMV alone (v4: 240).
 const GSpmvVariant kGSpmv[] = {
     {k_g_spmv<3, false, 5>, k_g_spmv<3, true, 5>, 3},
     {k_g_spmv<3, false>, k_g_spmv<3, true>, 3},
@@ -769,6 +840,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         a.su = K->sc_upper;
         a.lfac = K->lfac;
         a.sfac = K->sfac;
+        a.dinv_fmax = reinterpret_cast<const unsigned long long*>(reinterpret_cast<char*>(K->scratch) + 192);
         G->g_ilu = ilu_grid();
         DDA_CK(cudaMemsetAsync(a.st, 0, sizeof(State), st));       // ticket = 0
 
@@ -807,6 +879,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
             if (scaled) {
                 launch(gspmv_variant().scaled, G->G_spmv, a, G->h);
                 launch(k_s_update, G->G_vec, a, G->h);
+                launch(k_s_check, G->G_vec, a, G->h);
                 continue;
             }
             launch(gspmv_variant().plain, G->G_spmv, a, G->h);
@@ -865,7 +938,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     DDA_LAUNCHED();
     k_g_resid<<<G->G_vec, DDA_THREADS, 0, st>>>(a);
     DDA_LAUNCHED();
-    struct { int it, status; double rel; } hres;
+    struct { int it, status; double rel; int checks, pad; } hres;
     DDA_CK(cudaMemcpyAsync(&hres, a.out, sizeof hres, cudaMemcpyDeviceToHost, st));
     trace("solve: all issued");
     DDA_CK(cudaStreamSynchronize(st));
@@ -873,9 +946,10 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     // loop body: k_g_spmv + k_g_update (+ 2 SSOR-AI halves or 2 ILU sweeps) per iteration, body_iters
     // iterations per pass; the body runs ceil(max(iterations, 1) / body_iters) times (once, as a no-op
     // pass, when the setup already decided the result); every kernel of a pass is launched
-    const int per_it = (pc == DDA_PC_SSOR_AI || pc == DDA_PC_ILU0) ? 4 : 2;
+    const int per_it = (pc == DDA_PC_SSOR_AI || pc == DDA_PC_ILU0) ? 4 : (scaled ? 3 : 2);
     const int its = hres.it > 0 ? hres.it : 1;
     note_launch(per_it * G->body_iters * ((its + G->body_iters - 1) / G->body_iters));
+    K->last_checks = scaled ? hres.checks : 0;
     if (iters) *iters = hres.it;
     if (rel_res) *rel_res = hres.rel;
     return (dda_status_t)hres.status;
@@ -936,6 +1010,10 @@ extern "C" int dda__time_pcg_phases_ex(dda_matrix_t K, const double* F, double* 
 extern "C" int dda__time_pcg_phases(dda_matrix_t K, const double* F, double* d, int reps, float* ms) {
     return dda__time_pcg_phases_ex(K, F, d, reps, ms, 0);
 }
+
+// Internal query (not in include/dda.h): exact stopping tests (k_s_check passes) of the last
+// scaled-engine solve on K (bench.py's algorithmic byte count).
+extern "C" int dda__last_checks(dda_matrix_t K) { return K ? K->last_checks : -1; }
 
 // Internal debugging hook (not in include/dda.h): copies the scaled-engine arrays to host
 // buffers (any may be NULL): su [nnzb][36] tiled, lfac / sfac [n][24] packed lower.

@@ -16,7 +16,8 @@ namespace {
 
 __global__ void __launch_bounds__(128) k_bj_inv(int32_t n, const double* __restrict__ diag, double* __restrict__ dinv,
                                                 double* __restrict__ full, double* __restrict__ lfac,
-                                                double* __restrict__ sfac, int* __restrict__ bad) {
+                                                double* __restrict__ sfac, int* __restrict__ bad,
+                                                unsigned long long* __restrict__ fmax) {
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const double* D = diag + (size_t)kBlk * i;
         double A[6][6];
@@ -72,6 +73,14 @@ __global__ void __launch_bounds__(128) k_bj_inv(int32_t n, const double* __restr
                 P[pk_off(r, c)] = s;
             }
         P[21] = P[22] = P[23] = 0.0;
+        if (fmax) {   // ||D_i^{-1}||_F >= 1 / lambda_min(D_i): the scaled engine's stopping-test bound
+            double f2 = 0.0;
+#pragma unroll
+            for (int r = 0; r < 6; ++r)
+#pragma unroll
+                for (int c = r; c < 6; ++c) f2 += (r == c ? 1.0 : 2.0) * P[pk_off(r, c)] * P[pk_off(r, c)];
+            if (ok) atomicMax(fmax, (unsigned long long)__double_as_longlong(sqrt(f2)));   // positive: bits order
+        }
 #pragma unroll
         for (int q = 0; q < 12; ++q) reinterpret_cast<double2*>(out)[q] = make_double2(P[2 * q], P[2 * q + 1]);
         if (lfac) {   // packed lower triangles of L and S = L^{-1} for the scaled BJ engine (pcg_graph.cu)
@@ -157,7 +166,9 @@ static dda_status_t bj_setup_n(dda_matrix* K, int32_t nrows, cudaStream_t st, in
         DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->sfac), sizeof(double) * kDinv * (size_t)K->n, st));
     }
     K->scaled_valid = false;
-    k_bj_inv<<<g, 128, 0, st>>>(nrows, K->diag, K->dinv, full, K->lfac, K->sfac, bad);
+    unsigned long long* fmax = reinterpret_cast<unsigned long long*>(reinterpret_cast<char*>(K->scratch) + 192);
+    DDA_CK(cudaMemsetAsync(fmax, 0, sizeof(unsigned long long), st));
+    k_bj_inv<<<g, 128, 0, st>>>(nrows, K->diag, K->dinv, full, K->lfac, K->sfac, bad, fmax);
     DDA_LAUNCHED();
     int hbad = 0;
     DDA_CK(cudaMemcpyAsync(&hbad, bad, sizeof(int), cudaMemcpyDeviceToHost, st));

@@ -327,6 +327,30 @@ def test_pcg_warm_start_and_edge_cases(dda, engine):
     assert st5 == dda.ERR_NO_CONVERGENCE and it5 == 200 and rr5 > 1e-10
 
 
+def test_scaled_engine_stopping_test(dda):
+    """The scaled engine evaluates the exact stopping test |L r~| only when lam |r~|^2 allows it to
+    pass: it must stop at the same iteration as the unscaled loop with far fewer
+    exact tests than iterations."""
+    import ctypes
+    f = dda.lib().dda__set_pcg_engine
+    f.argtypes = [ctypes.c_int]
+    P, O = case("paper")
+    K = dda.build_from_problem(P)
+    F = torch.from_numpy(P.F).cuda()
+    try:
+        f(0)
+        d0, it0, rr0, st0 = K.pcg_solve(F)
+        f(2)
+        d2, it2, rr2, st2 = K.pcg_solve(F)
+    finally:
+        f(-1)
+    assert st0 == st2 == dda.OK
+    assert abs(it0 - it2) <= 1, (it0, it2)
+    checks = K.last_checks()
+    assert 1 <= checks < it2 // 2, (checks, it2)
+    assert np.linalg.norm(d2.cpu().numpy() - d0.cpu().numpy()) <= 1e-8 * np.linalg.norm(d0.cpu().numpy())
+
+
 def test_pcg_deterministic(dda):
     P, O = case("paper")
     K = dda.build_from_problem(P)

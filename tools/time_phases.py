@@ -17,9 +17,9 @@ for scaled in (0, 1):
     rc = L.dda__time_pcg_phases_ex(K.handle, C.c_void_p(t["F"].data_ptr()), C.c_void_p(d.data_ptr()), 20, ms,
                                    scaled)
     # algorithmic bytes per row: unscaled SpMV + 96 / update 528; scaled SpMV
-    # without D (300u + 8 + 192) / update 480 (p, x, r~, q~, L read; x, r~ written)
-    spmv_bytes = K.n * ((300 * u + 200) if scaled else (392 + 300 * u + 96))
-    upd_bytes = K.n * (480 if scaled else 528)
+    # without D (300u + 8 + 192) + deferred x update (96) / update 144 (r~, q~ read; r~ written)
+    spmv_bytes = K.n * ((300 * u + 296) if scaled else (392 + 300 * u + 96))
+    upd_bytes = K.n * (144 if scaled else 528)
     print(json.dumps({"scaled": scaled, "rc": rc, "n": K.n, "spmv_fused_ms": ms[0],
                       "spmv_fused_gbs": spmv_bytes / ms[0] / 1e6,
                       "update_ms": ms[1], "update_gbs": upd_bytes / ms[1] / 1e6}))
