@@ -17,7 +17,8 @@ namespace {
 __global__ void __launch_bounds__(128) k_bj_inv(int32_t n, const double* __restrict__ diag, double* __restrict__ dinv,
                                                 double* __restrict__ full, double* __restrict__ lfac,
                                                 double* __restrict__ sfac, int* __restrict__ bad,
-                                                unsigned long long* __restrict__ fmax) {
+                                                unsigned long long* __restrict__ fnorm_max) {
+    double fmax_local = 0.0;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const double* D = diag + (size_t)kBlk * i;
         double A[6][6];
@@ -73,13 +74,13 @@ __global__ void __launch_bounds__(128) k_bj_inv(int32_t n, const double* __restr
                 P[pk_off(r, c)] = s;
             }
         P[21] = P[22] = P[23] = 0.0;
-        if (fmax) {   // ||D_i^{-1}||_F >= 1 / lambda_min(D_i): the scaled engine's stopping-test bound
+        if (fnorm_max) {   // ||D_i^{-1}||_F >= 1 / lambda_min(D_i): the scaled engine's stopping-test bound
             double f2 = 0.0;
 #pragma unroll
             for (int r = 0; r < 6; ++r)
 #pragma unroll
                 for (int c = r; c < 6; ++c) f2 += (r == c ? 1.0 : 2.0) * P[pk_off(r, c)] * P[pk_off(r, c)];
-            if (ok) atomicMax(fmax, (unsigned long long)__double_as_longlong(sqrt(f2)));   // positive: bits order
+            fmax_local = fmax(fmax_local, ok ? sqrt(f2) : 0.0);
         }
 #pragma unroll
         for (int q = 0; q < 12; ++q) reinterpret_cast<double2*>(out)[q] = make_double2(P[2 * q], P[2 * q + 1]);
@@ -107,6 +108,12 @@ __global__ void __launch_bounds__(128) k_bj_inv(int32_t n, const double* __restr
 #pragma unroll
                 for (int c = 0; c < 6; ++c) full[36 * i + 6 * r + c] = P[r <= c ? pk_off(r, c) : pk_off(c, r)];
         }
+    }
+    if (fnorm_max) {   // one atomic per warp (positive doubles order like their bit patterns)
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) fmax_local = fmax(fmax_local, __shfl_xor_sync(0xffffffffu, fmax_local, o));
+        if ((threadIdx.x & 31) == 0 && fmax_local > 0.0)
+            atomicMax(fnorm_max, (unsigned long long)__double_as_longlong(fmax_local));
     }
 }
 
