@@ -313,7 +313,14 @@ def main():
     assert rel_res <= 1e-10 * 1.01, rel_res
     u = nnzb / n
     pcg_ms = statistics.mean(ph_pcg)
-    if engine == "scaled":
+    if engine == "scaled" and dda.lib().dda__get_scaled_loop() == 1:
+        engine = "scaled_persistent"
+        pcg_bytes = pcg_launch_bytes_scaled(n, nnzb, iters, checks)
+        pcg_kernel = ("dda_pcg_solve, scaled block-Jacobi engine: k_scale_upper (S_i V_ij S_j^T) + k_s_init + ONE "
+                      "persistent cooperative kernel k_sp_loop running every iteration (phase A fused p-update + "
+                      "SpMV + x update, phase B r~ update, rare phase C exact stopping test; grid barriers) + "
+                      f"k_s_final + true-residual SpMV; {checks} exact stopping tests")
+    elif engine == "scaled":
         pcg_bytes = pcg_launch_bytes_scaled(n, nnzb, iters, checks)
         pcg_kernel = ("dda_pcg_solve, scaled block-Jacobi engine: k_scale_upper (S_i V_ij S_j^T) + one CUDA-graph "
                       "while loop (k_g_spmv<SC> + k_s_update + k_s_check per iteration) with its prelude/epilogue "

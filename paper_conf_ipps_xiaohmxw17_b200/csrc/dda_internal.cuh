@@ -124,6 +124,7 @@ struct dda_matrix {
     bool dinv_valid = false;
     double* lfac = nullptr;         // [n][24] packed lower Cholesky factor L_i of D_i (D_i = L_i L_i^T)
     double* sfac = nullptr;         // [n][24] packed lower S_i = L_i^{-1}
+    double* bj_w = nullptr;         // [n] w_i <= lambda_min(D_i): 1 / min(||D_i^{-1}||_F, ||D_i^{-1}||_inf)
     double* sc_upper = nullptr;     // [nnzb][36] tiled: S_i V_ij S_j^T (scaled BJ engine)
     bool scaled_valid = false;
     double* ilu_up = nullptr;       // [nnzb][36] tiled: U_ij of the block IC(0) = ILU(0) factor

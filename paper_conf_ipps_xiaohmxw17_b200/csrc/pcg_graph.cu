@@ -17,11 +17,15 @@
 // re-summing.  Per-call pointers (F, d0, d) and tol / maxit / omega travel
 // in a device CallArgs block, so one instantiated graph per (matrix, precond)
 // is reused across solves.
+#include <cooperative_groups.h>
+
 #include <cmath>
 #include <cstdlib>
 
 #include "ilu_dev.cuh"
 #include "spmv_col.cuh"
+
+namespace cg = cooperative_groups;
 
 namespace dda {
 namespace {
@@ -69,8 +73,17 @@ struct GArgs {           // constant for a (matrix, preconditioner): baked into 
     const double* lfac;  // packed lower L_i (D_i = L_i L_i^T)
     const double* sfac;  // packed lower S_i = L_i^{-1}
     const unsigned long long* dinv_fmax;   // bits of max_i ||D_i^{-1}||_F (bj_setup)
+    const double* bj_w;  // [n] w_i <= lambda_min(D_i) (bj_setup): sum_i w_i |r~_i|^2 <= |L r~|^2
     int use_cond;        // 0 only for the internal phase-timing hook (kernels launched outside the graph)
+    unsigned long long* trace;   // k_sp_loop timeline [iter][cta][4] (%globaltimer), null = off (internal hook)
+    int trace_iters;
 };
+
+__device__ __forceinline__ unsigned long long gtimer() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
 
 __device__ __forceinline__ void set_cond(const GArgs& a, cudaGraphConditionalHandle h, unsigned v) {
     if (a.use_cond) cudaGraphSetConditional(h, v);
@@ -613,10 +626,11 @@ __global__ void __launch_bounds__(DDA_THREADS) k_s_init(const GArgs a) {
 
 // phase B: r~ -= alpha q~; rho' = |r~|^2 (x += alpha p~ is applied by the next SpMV or k_s_final).
 // The stopping test (reading Z1) is on the ORIGINAL residual r = L r~, whose norm costs the packed
-// L_i (192 B per row).  It is evaluated only when it can succeed: |L r~|^2 >= lam |r~|^2 with
-// lam = min_i lambda_min(D_i) >= 1 / max_i ||D_i^{-1}||_F, so while 0.999 lam rho' > tol^2 ||F||^2
-// the iteration cannot have converged and L is not read.  Otherwise k_s_check evaluates |L r~|
-// exactly (the decision, the iteration count and the solution are those of the plain test).
+// L_i (192 B per row).  It is evaluated only when it can succeed: |L_i r~_i|^2 >= lambda_min(D_i)
+// |r~_i|^2 >= w_i |r~_i|^2 (w_i = 1 / min(||D_i^{-1}||_F, ||D_i^{-1}||_inf), bj_setup), so while
+// 0.999 sum_i w_i |r~_i|^2 > tol^2 ||F||^2 the iteration cannot have converged and L is not read
+// (8 B of w per row instead of 192 B of L).  Otherwise k_s_check evaluates |L r~| exactly (the
+// decision, the iteration count and the solution are those of the plain test).
 __global__ void __launch_bounds__(DDA_THREADS, 4) k_s_update(const GArgs a, cudaGraphConditionalHandle h) {
     pdl_enter();
     if (loop_done(a.st)) return;
@@ -624,21 +638,22 @@ __global__ void __launch_bounds__(DDA_THREADS, 4) k_s_update(const GArgs a, cuda
     const double alpha = a.st->alpha;
     const int lane = threadIdx.x & 31;
     const int n = a.A.n, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
-    double rz = 0.0;
+    double rz = 0.0, lb = 0.0;
     for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += 2 * W) {
         const Row5 RA = row5(grp, lane, n);
         const Row5 RB = row5(grp + W, lane, n);
-        double ra = 0, qa = 0, rb = 0, qb = 0;
-        if (RA.valid) { ra = a.r[RA.idx]; qa = a.q[RA.idx]; }
-        if (RB.valid) { rb = a.r[RB.idx]; qb = a.q[RB.idx]; }
+        double ra = 0, qa = 0, rb = 0, qb = 0, wa = 0, wb = 0;
+        if (RA.valid) { ra = a.r[RA.idx]; qa = a.q[RA.idx]; wa = __ldg(a.bj_w + RA.i); }
+        if (RB.valid) { rb = a.r[RB.idx]; qb = a.q[RB.idx]; wb = __ldg(a.bj_w + RB.i); }
         const double rva = RA.valid ? ra - alpha * qa : 0.0;
         const double rvb = RB.valid ? rb - alpha * qb : 0.0;
         if (RA.valid) a.r[RA.idx] = rva;
         if (RB.valid) a.r[RB.idx] = rvb;
         rz += rva * rva + rvb * rvb;
+        lb += wa * (rva * rva) + wb * (rvb * rvb);
     }
-    double v[1] = {rz}, tot[1];
-    if (grid_reduce_last<1>(a, v, tot) && threadIdx.x == 0) {
+    double v[2] = {rz, lb}, tot[2];
+    if (grid_reduce_last<2>(a, v, tot) && threadIdx.x == 0) {
         State* st = a.st;
         st->pend = 1;                                       // x += alpha p_k: next SpMV or k_s_final
         const double rho1 = tot[0];
@@ -650,7 +665,7 @@ __global__ void __launch_bounds__(DDA_THREADS, 4) k_s_update(const GArgs a, cuda
             st->k = k + 1;
             st->done = 1;
             set_cond(a, h, 0);
-        } else if (isfinite(rho1) && 0.999 * st->lam * rho1 <= thr * thr) {
+        } else if (isfinite(rho1) && !(0.999 * tot[1] > thr * thr)) {
             st->maybe = 1;                                  // k_s_check decides
             st->pend_rz = rho1;
         } else {
@@ -711,6 +726,190 @@ __global__ void __launch_bounds__(DDA_THREADS) k_s_final(const GArgs a) {
     }
 }
 
+// ---------------------------------------------------------------- scaled engine, persistent loop
+//
+// The same iteration as the graph loop above (k_g_spmv<SC> -> k_s_update -> [k_s_check]) with the
+// kernel boundaries replaced by grid barriers: ONE cooperative launch runs every iteration.  At 1M
+// blocks the graph loop spends ~45 us per iteration (of 323) between its kernels (drain / fill of
+// three grids, the while-loop back edge); a grid barrier costs a few us.  Every CTA sums the CTA
+// partials itself in one fixed order, so all CTAs take the same branches.  Vectors written in
+// this launch (p, q, r~, x) are read with weak loads after the barrier (grid.sync is a gpu-scope
+// fence), never through the read-only path; the matrix is read-only and keeps its .nc loads.
+
+// x = r~ + beta p_old with coherent loads (k = 0: p = r~, beta = 0 gives r~ exactly)
+struct XFusedW {
+    const double* z;
+    const double* p;
+    double beta;
+    using Raw = double2;
+    __device__ __forceinline__ Raw raw(int vec, int pair) const {
+        const size_t o = 6 * (size_t)vec + 2 * pair;
+        const double2 zz = ld_cg2(z + o), pp = ld_cg2(p + o);
+        return make_double2(fma(beta, pp.x, zz.x), fma(beta, pp.y, zz.y));
+    }
+    __device__ __forceinline__ double2 cook(const Raw& r) const { return r; }
+    __device__ __forceinline__ double2 operator()(int vec, int pair) const { return raw(vec, pair); }
+};
+
+// Fixed-order grid sums of NV values per thread: CTA partials -> part[(slot+k)*Gmax + cta], grid
+// barrier, then every CTA sums the G partials in the order grid_reduce_last uses.  Slots: 0 (phase
+// A), 1-2 (phase B), 0 (phase C); a slot is rewritten only after at least one further barrier, so
+// no CTA can still be reading it.
+template <int NV>
+__device__ __forceinline__ void grid_allsum(const GArgs& a, cg::grid_group& grid, int slot, double (&v)[NV],
+                                            double (&tot)[NV]) {
+    __shared__ double red[NV][DDA_THREADS];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+#pragma unroll
+    for (int k = 0; k < NV; ++k) v[k] = warp_sum(v[k]);
+    if (lane == 0) {
+#pragma unroll
+        for (int k = 0; k < NV; ++k) red[k][wib] = v[k];
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+#pragma unroll
+        for (int k = 0; k < NV; ++k) {
+            double s = 0.0;
+            for (int w = 0; w < WPB; ++w) s += red[k][w];
+            a.part[(size_t)(slot + k) * a.Gmax + blockIdx.x] = s;
+        }
+    }
+    grid.sync();
+    const int G = gridDim.x;
+#pragma unroll
+    for (int k = 0; k < NV; ++k) {
+        const double* part = a.part + (size_t)(slot + k) * a.Gmax;
+        double s = 0.0;
+        for (int j = threadIdx.x; j < G; j += DDA_THREADS) s += ld_cg(part + j);
+        red[k][threadIdx.x] = s;
+    }
+    __syncthreads();
+    for (int h = DDA_THREADS / 2; h > 0; h >>= 1) {
+        if (threadIdx.x < h) {
+#pragma unroll
+            for (int k = 0; k < NV; ++k) red[k][threadIdx.x] += red[k][threadIdx.x + h];
+        }
+        __syncthreads();
+    }
+#pragma unroll
+    for (int k = 0; k < NV; ++k) tot[k] = red[k][0];
+    __syncthreads();
+}
+
+template <int MINB>
+__global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_loop(const GArgs a) {
+    cg::grid_group grid = cg::this_grid();
+    State* st = a.st;
+    unsigned long long* tr_k = (a.trace && blockIdx.x == 0 && threadIdx.x == 0)
+                                   ? a.trace + 4 * (size_t)a.trace_iters * gridDim.x : nullptr;
+    if (tr_k) tr_k[0] = gtimer();                           // kernel entry / exit stamps (after the rows)
+    if (st->done) return;                                   // decided at setup (uniform: no barrier reached)
+    double rho = st->rho, alpha = 0.0, beta = 0.0, rr_last = st->rr;
+    const double thr = a.ca->tol * st->bnorm;
+    const int maxit = a.ca->maxit;
+    BsrView A = a.A;
+    A.upper = a.su;
+    const int lane = threadIdx.x & 31;
+    const int w0 = blockIdx.x * WPB + (threadIdx.x >> 5), W = gridDim.x * WPB;
+    const int n = A.n, ngrp = (n + 4) / 5;
+    double* x = a.ca->d;
+    int k = 0, status = DDA_ERR_NO_CONVERGENCE, iters = 0, checks = 0, pend = 0;
+    unsigned long long* tr = nullptr;
+    for (;;) {
+        tr = (a.trace && k < a.trace_iters && threadIdx.x == 0)
+                 ? a.trace + 4 * ((size_t)k * gridDim.x + blockIdx.x) : nullptr;
+        if (tr) tr[0] = gtimer();
+        // phase A: p_k = r~ + beta p_{k-1} (own rows written), q = Ks p_k, x += alpha_{k-1} p_{k-1}
+        double* pnew = (k & 1) ? a.p1 : a.p0;
+        const double* pold = k == 0 ? a.r : ((k & 1) ? a.p0 : a.p1);
+        const XFusedW xf{a.r, pold, beta};
+        const double ap = alpha;
+        double acc = 0.0;
+        for_rows_c<SPMV_OFFDIAG, 5>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+            if (ok) {
+                const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
+                const double2 pv = xf(i, ccol_of(lane));
+                y0 += pv.x;
+                y1 += pv.y;
+                const double2 po = ld_cg2(pold + o);
+                const double2 xo = ld_cg2(x + o);
+                *reinterpret_cast<double2*>(x + o) = make_double2(xo.x + ap * po.x, xo.y + ap * po.y);
+                *reinterpret_cast<double2*>(a.q + o) = make_double2(y0, y1);
+                *reinterpret_cast<double2*>(pnew + o) = pv;
+                acc += pv.x * y0 + pv.y * y1;
+            }
+        });
+        if (tr) tr[1] = gtimer();
+        double sv[1] = {acc}, stot[1];
+        grid_allsum<1>(a, grid, 0, sv, stot);
+        const double sigma = stot[0];
+        if (tr) tr[2] = gtimer();
+        pend = 0;
+        if (!(sigma > 0.0) || !isfinite(sigma)) { status = DDA_ERR_BREAKDOWN; break; }   // reading Z19
+        alpha = rho / sigma;
+        // phase B: r~ -= alpha q; rho' = |r~|^2 and the lower bound sum_i w_i |r~_i|^2 of |L r~|^2
+        double rz = 0.0, lb = 0.0;
+        for (int grp = w0; grp < ngrp; grp += 2 * W) {
+            const Row5 RA = row5(grp, lane, n);
+            const Row5 RB = row5(grp + W, lane, n);
+            double ra = 0, qa = 0, rb = 0, qb = 0, wa = 0, wb = 0;
+            if (RA.valid) { ra = ld_cg(a.r + RA.idx); qa = ld_cg(a.q + RA.idx); wa = __ldg(a.bj_w + RA.i); }
+            if (RB.valid) { rb = ld_cg(a.r + RB.idx); qb = ld_cg(a.q + RB.idx); wb = __ldg(a.bj_w + RB.i); }
+            const double rva = RA.valid ? ra - alpha * qa : 0.0;
+            const double rvb = RB.valid ? rb - alpha * qb : 0.0;
+            if (RA.valid) a.r[RA.idx] = rva;
+            if (RB.valid) a.r[RB.idx] = rvb;
+            rz += rva * rva + rvb * rvb;
+            lb += wa * (rva * rva) + wb * (rvb * rvb);
+        }
+        if (tr) tr[3] = gtimer();
+        double bv[2] = {rz, lb}, btot[2];
+        grid_allsum<2>(a, grid, 1, bv, btot);
+        const double rho1 = btot[0];
+        pend = 1;                                           // x += alpha p_k: next phase A or k_s_final
+        iters = k + 1;
+        if (rho1 == 0.0) { status = DDA_OK; rr_last = 0.0; k = k + 1; break; }
+        if (isfinite(rho1) && !(0.999 * btot[1] > thr * thr)) {
+            // phase C (rare): the exact stopping test |L r~| <= tol ||F|| (reading Z1; see k_s_update)
+            double rl = 0.0;
+            for (int grp = w0; grp < ngrp; grp += W) {
+                const Row5 R = row5(grp, lane, n);
+                const double rv = R.valid ? ld_cg(a.r + R.idx) : 0.0;
+                const DinvRow Lrow = tri_row(a.lfac, R);
+                const double o0 = dinv_row_apply(Lrow, rv, R);
+                const double o = R.valid ? o0 : 0.0;
+                rl += o * o;
+            }
+            double cv[1] = {rl}, ctot[1];
+            grid_allsum<1>(a, grid, 0, cv, ctot);
+            const double rr = ctot[0];
+            checks += 1;
+            rr_last = rr;
+            if (sqrt(rr) <= thr) { status = DDA_OK; k = k + 1; break; }
+        }
+        // finish_iteration
+        k = k + 1;
+        if (!(rho1 > 0.0) || !isfinite(rho1)) { status = DDA_ERR_BREAKDOWN; break; }
+        beta = rho1 / rho;
+        rho = rho1;
+        if (k >= maxit) { status = DDA_ERR_NO_CONVERGENCE; break; }
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {              // the State k_s_final / k_g_resid read
+        st->k = k;
+        st->iters = iters;
+        st->status = status;
+        st->done = 1;
+        st->alpha = alpha;
+        st->beta = beta;
+        st->rho = rho;
+        st->rr = rr_last;
+        st->pend = pend;
+        st->checks = checks;
+    }
+    if (tr_k) tr_k[1] = gtimer();
+}
+
 // loop-body SpMV kernel variants (tuning aid, DDA_GSPMV_VARIANT): occupancy / register budget
 typedef void (*GSpmvKernel)(const GArgs, cudaGraphConditionalHandle);
 struct GSpmvVariant { GSpmvKernel plain, scaled; int minb; };
@@ -748,6 +947,12 @@ int occ_grid(const void* k, int minb_cap) {
 
 }  // namespace
 
+// scaled-engine loop: 1 = persistent cooperative kernel, 0 = CUDA-graph while loop, -1 = from
+// DDA_SCALED_LOOP (default persistent); set by the internal hook dda__set_scaled_loop
+int g_scaled_loop = -1;
+unsigned long long* g_trace = nullptr;   // k_sp_loop timeline (internal hook dda__set_loop_trace)
+int g_trace_iters = 0;
+
 // Per-handle cached graph engine
 struct PcgGraph {
     int pc = -1;
@@ -756,6 +961,7 @@ struct PcgGraph {
     cudaGraph_t graph = nullptr;
     cudaGraphConditionalHandle h = 0;
     int G_spmv = 0, G_vec = 0, g_ilu = 0;
+    int G_persist = 0;   // scaled engine, persistent loop: cooperative grid (0: graph loop)
     int body_iters = 2;
 };
 
@@ -793,7 +999,14 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         if (s != DDA_OK) return s;
     }
     trace("solve: enter");
-    const int key = scaled ? 100 + (int)pc : (int)pc;
+    // scaled engine loop: one persistent cooperative kernel (default) or the CUDA-graph while loop
+    // (DDA_SCALED_LOOP=graph)
+    if (g_scaled_loop < 0) {
+        const char* e = getenv("DDA_SCALED_LOOP");
+        g_scaled_loop = (e && (e[0] == 'g' || e[0] == '0')) ? 0 : 1;
+    }
+    const bool persist = scaled && g_scaled_loop == 1;
+    const int key = scaled ? (persist ? 200 : 100) + (int)pc : (int)pc;
     PcgGraph*& G = reinterpret_cast<PcgGraph*&>(K->graph_engine);
     if (G && G->pc != key) {
         pcg_graph_free(G);
@@ -809,6 +1022,15 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         if (g_vec > need_vec) g_vec = need_vec > 0 ? need_vec : 1;
         int Gmax = g_spmv > g_vec ? g_spmv : g_vec;
         if (ilu_grid() > Gmax) Gmax = ilu_grid();
+        int g_persist = 0;
+        if (persist) {   // every CTA must be co-resident (cooperative launch)
+            int per_sm = 0;
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_sp_loop<3>, DDA_THREADS, 0);
+            if (per_sm > 3) per_sm = 3;
+            if (per_sm < 1) return DDA_ERR_CUDA;
+            g_persist = device_sms() * per_sm;
+            if (g_persist > Gmax) Gmax = g_persist;
+        }
         const size_t bytes = (7 * N + 3 * (size_t)Gmax) * sizeof(double) + sizeof(CallArgs) + sizeof(State) + 64;
         // may reallocate the workspace (and drop any engine holding the old pointers): do it first
         dda_status_t s = ensure_workspace(K, bytes, st);
@@ -817,6 +1039,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         G->pc = key;
         G->G_spmv = g_spmv;
         G->G_vec = g_vec;
+        G->G_persist = g_persist;
         double* ws = K->ws;
         GArgs& a = G->a;
         a.A = view_of(K);
@@ -840,65 +1063,68 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         a.su = K->sc_upper;
         a.lfac = K->lfac;
         a.sfac = K->sfac;
+        a.bj_w = K->bj_w;
         a.dinv_fmax = reinterpret_cast<const unsigned long long*>(reinterpret_cast<char*>(K->scratch) + 192);
         G->g_ilu = ilu_grid();
         DDA_CK(cudaMemsetAsync(a.st, 0, sizeof(State), st));       // ticket = 0
 
-        // ---- the loop: a while conditional node whose body is captured from a stream
-        DDA_CK(cudaGraphCreate(&G->graph, 0));
-        DDA_CK(cudaGraphConditionalHandleCreate(&G->h, G->graph, 1, cudaGraphCondAssignDefault));
-        cudaGraphNodeParams cp = {};
-        cp.type = cudaGraphNodeTypeConditional;
-        cp.conditional.handle = G->h;
-        cp.conditional.type = cudaGraphCondTypeWhile;
-        cp.conditional.size = 1;
-        cudaGraphNode_t cnode;
-        DDA_CK(cudaGraphAddNode(&cnode, G->graph, nullptr, 0, &cp));
-        cudaGraph_t body = cp.conditional.phGraph_out[0];
-        cudaStream_t cs;
-        DDA_CK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
-        DDA_CK(cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal));
-        // body = two PCG iterations; kernels chained with programmatic dependent launch
-        cudaLaunchAttribute pdl[1];
-        pdl[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-        pdl[0].val.programmaticStreamSerializationAllowed = env_int("DDA_PDL", 1) ? 1 : 0;
-        // iterations per while-loop pass (tuning aid); the kernels exit early once the loop is done
-        int body_iters = env_int("DDA_BODY_ITERS", 2);
-        if (body_iters < 1 || body_iters > 16) body_iters = 2;
-        G->body_iters = body_iters;
-        auto launch = [&](auto kern, int grid, auto... args) {
-            cudaLaunchConfig_t cfg = {};
-            cfg.gridDim = dim3(grid);
-            cfg.blockDim = dim3(DDA_THREADS);
-            cfg.stream = cs;
-            cfg.attrs = pdl;
-            cfg.numAttrs = 1;
-            cudaLaunchKernelEx(&cfg, kern, args...);
-        };
-        for (int rep = 0; rep < body_iters; ++rep) {
-            if (scaled) {
-                launch(gspmv_variant().scaled, G->G_spmv, a, G->h);
-                launch(k_s_update, G->G_vec, a, G->h);
-                launch(k_s_check, G->G_vec, a, G->h);
-                continue;
+        if (!persist) {   // persistent: no graph, k_sp_loop runs the whole loop
+            // ---- the loop: a while conditional node whose body is captured from a stream
+            DDA_CK(cudaGraphCreate(&G->graph, 0));
+            DDA_CK(cudaGraphConditionalHandleCreate(&G->h, G->graph, 1, cudaGraphCondAssignDefault));
+            cudaGraphNodeParams cp = {};
+            cp.type = cudaGraphNodeTypeConditional;
+            cp.conditional.handle = G->h;
+            cp.conditional.type = cudaGraphCondTypeWhile;
+            cp.conditional.size = 1;
+            cudaGraphNode_t cnode;
+            DDA_CK(cudaGraphAddNode(&cnode, G->graph, nullptr, 0, &cp));
+            cudaGraph_t body = cp.conditional.phGraph_out[0];
+            cudaStream_t cs;
+            DDA_CK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+            DDA_CK(cudaStreamBeginCaptureToGraph(cs, body, nullptr, nullptr, 0, cudaStreamCaptureModeThreadLocal));
+            // body = two PCG iterations; kernels chained with programmatic dependent launch
+            cudaLaunchAttribute pdl[1];
+            pdl[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+            pdl[0].val.programmaticStreamSerializationAllowed = env_int("DDA_PDL", 1) ? 1 : 0;
+            // iterations per while-loop pass (tuning aid); the kernels exit early once the loop is done
+            int body_iters = env_int("DDA_BODY_ITERS", 2);
+            if (body_iters < 1 || body_iters > 16) body_iters = 2;
+            G->body_iters = body_iters;
+            auto launch = [&](auto kern, int grid, auto... args) {
+                cudaLaunchConfig_t cfg = {};
+                cfg.gridDim = dim3(grid);
+                cfg.blockDim = dim3(DDA_THREADS);
+                cfg.stream = cs;
+                cfg.attrs = pdl;
+                cfg.numAttrs = 1;
+                cudaLaunchKernelEx(&cfg, kern, args...);
+            };
+            for (int rep = 0; rep < body_iters; ++rep) {
+                if (scaled) {
+                    launch(gspmv_variant().scaled, G->G_spmv, a, G->h);
+                    launch(k_s_update, G->G_vec, a, G->h);
+                    launch(k_s_check, G->G_vec, a, G->h);
+                    continue;
+                }
+                launch(gspmv_variant().plain, G->G_spmv, a, G->h);
+                launch(k_g_update, G->G_vec, a, G->h);
+                if (pc == DDA_PC_SSOR_AI) {
+                    launch(k_g_ssor_lower<false>, G->G_spmv, a);
+                    launch(k_g_ssor_upper<false>, G->G_spmv, a, G->h);
+                } else if (pc == DDA_PC_ILU0) {
+                    cudaMemsetAsync(a.ilu_flags_f, 0, 2 * (size_t)K->n * sizeof(int), cs);
+                    cudaMemsetAsync(a.ilu_counters, 0, 2 * sizeof(int), cs);
+                    k_g_ilu_fwd<false><<<G->g_ilu, DDA_THREADS, 0, cs>>>(a);
+                    k_g_ilu_bwd<false><<<G->g_ilu, DDA_THREADS, 0, cs>>>(a, G->h);
+                }
             }
-            launch(gspmv_variant().plain, G->G_spmv, a, G->h);
-            launch(k_g_update, G->G_vec, a, G->h);
-            if (pc == DDA_PC_SSOR_AI) {
-                launch(k_g_ssor_lower<false>, G->G_spmv, a);
-                launch(k_g_ssor_upper<false>, G->G_spmv, a, G->h);
-            } else if (pc == DDA_PC_ILU0) {
-                cudaMemsetAsync(a.ilu_flags_f, 0, 2 * (size_t)K->n * sizeof(int), cs);
-                cudaMemsetAsync(a.ilu_counters, 0, 2 * sizeof(int), cs);
-                k_g_ilu_fwd<false><<<G->g_ilu, DDA_THREADS, 0, cs>>>(a);
-                k_g_ilu_bwd<false><<<G->g_ilu, DDA_THREADS, 0, cs>>>(a, G->h);
-            }
+            cudaError_t ce = cudaStreamEndCapture(cs, nullptr);
+            cudaStreamDestroy(cs);
+            if (ce != cudaSuccess) { dda_status_t s2 = cuda_fail(ce); pcg_graph_free(G); G = nullptr; return s2; }
+            ce = cudaGraphInstantiate(&G->exec, G->graph, 0);
+            if (ce != cudaSuccess) { dda_status_t s2 = cuda_fail(ce); pcg_graph_free(G); G = nullptr; return s2; }
         }
-        cudaError_t ce = cudaStreamEndCapture(cs, nullptr);
-        cudaStreamDestroy(cs);
-        if (ce != cudaSuccess) { dda_status_t s2 = cuda_fail(ce); pcg_graph_free(G); G = nullptr; return s2; }
-        ce = cudaGraphInstantiate(&G->exec, G->graph, 0);
-        if (ce != cudaSuccess) { dda_status_t s2 = cuda_fail(ce); pcg_graph_free(G); G = nullptr; return s2; }
     }
     trace("solve: engine ready");
     GArgs& a = G->a;
@@ -928,7 +1154,16 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         DDA_LAUNCHED();
     }
     // ---- the device-side loop (its kernel launches are counted below from the iteration count)
-    DDA_CK(cudaGraphLaunch(G->exec, st));
+    if (G->G_persist) {
+        a.trace = g_trace;
+        a.trace_iters = g_trace_iters;
+        void* kargs[] = {reinterpret_cast<void*>(&a)};
+        DDA_CK(cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_sp_loop<3>), dim3(G->G_persist),
+                                           dim3(DDA_THREADS), kargs, 0, st));
+        DDA_LAUNCHED();
+    } else {
+        DDA_CK(cudaGraphLaunch(G->exec, st));
+    }
     // ---- epilogue: [d = S^T x], true residual
     if (scaled) {
         k_s_final<<<G->G_vec, DDA_THREADS, 0, st>>>(a);
@@ -948,7 +1183,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     // pass, when the setup already decided the result); every kernel of a pass is launched
     const int per_it = (pc == DDA_PC_SSOR_AI || pc == DDA_PC_ILU0) ? 4 : (scaled ? 3 : 2);
     const int its = hres.it > 0 ? hres.it : 1;
-    note_launch(per_it * G->body_iters * ((its + G->body_iters - 1) / G->body_iters));
+    if (!G->G_persist) note_launch(per_it * G->body_iters * ((its + G->body_iters - 1) / G->body_iters));
     K->last_checks = scaled ? hres.checks : 0;
     if (iters) *iters = hres.it;
     if (rel_res) *rel_res = hres.rel;
@@ -1027,4 +1262,27 @@ extern "C" int dda__scaled_export(dda_matrix_t K, double* su, double* lfac, doub
     if (lfac) cudaMemcpy(lfac, K->lfac, sizeof(double) * kDinv * K->n, cudaMemcpyDeviceToHost);
     if (sfac) cudaMemcpy(sfac, K->sfac, sizeof(double) * kDinv * K->n, cudaMemcpyDeviceToHost);
     return cudaGetLastError() == cudaSuccess ? 0 : -5;
+}
+
+// Internal testing hook (not in include/dda.h): the scaled engine's loop, 1 = persistent cooperative
+// kernel, 0 = CUDA-graph while loop, -1 = DDA_SCALED_LOOP / default.  Engines cached on a matrix
+// are keyed by the loop kind, so the next solve rebuilds as needed.
+extern "C" void dda__set_scaled_loop(int v) { dda::g_scaled_loop = v; }
+// Internal hook: k_sp_loop timeline buffer (device, [iters][G][4] u64: phase A start, phase A end,
+// sigma known, phase B end), null = off.  Returns the persistent grid size of the cached engine
+// (0 if none yet).
+extern "C" int dda__set_loop_trace(dda_matrix_t K, unsigned long long* buf, int iters) {
+    dda::g_trace = buf;
+    dda::g_trace_iters = iters;
+    dda::PcgGraph* G = K ? reinterpret_cast<dda::PcgGraph*>(K->graph_engine) : nullptr;
+    return G ? G->G_persist : 0;
+}
+
+// Internal query: the scaled engine's loop driver the next solve uses (1 persistent, 0 graph).
+extern "C" int dda__get_scaled_loop() {
+    if (dda::g_scaled_loop < 0) {
+        const char* e = getenv("DDA_SCALED_LOOP");
+        return (e && (e[0] == 'g' || e[0] == '0')) ? 0 : 1;
+    }
+    return dda::g_scaled_loop;
 }

@@ -16,8 +16,8 @@ namespace {
 
 __global__ void __launch_bounds__(128) k_bj_inv(int32_t n, const double* __restrict__ diag, double* __restrict__ dinv,
                                                 double* __restrict__ full, double* __restrict__ lfac,
-                                                double* __restrict__ sfac, int* __restrict__ bad,
-                                                unsigned long long* __restrict__ fnorm_max) {
+                                                double* __restrict__ sfac, double* __restrict__ wlow,
+                                                int* __restrict__ bad, unsigned long long* __restrict__ fnorm_max) {
     double fmax_local = 0.0;
     for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const double* D = diag + (size_t)kBlk * i;
@@ -81,6 +81,18 @@ __global__ void __launch_bounds__(128) k_bj_inv(int32_t n, const double* __restr
 #pragma unroll
                 for (int c = r; c < 6; ++c) f2 += (r == c ? 1.0 : 2.0) * P[pk_off(r, c)] * P[pk_off(r, c)];
             fmax_local = fmax(fmax_local, ok ? sqrt(f2) : 0.0);
+            if (wlow) {   // per-block lower bound of lambda_min(D_i) = 1 / ||D_i^{-1}||_2 (scaled engine)
+                double ninf = 0.0;
+#pragma unroll
+                for (int r = 0; r < 6; ++r) {
+                    double s = 0.0;
+#pragma unroll
+                    for (int c = 0; c < 6; ++c) s += fabs(P[r <= c ? pk_off(r, c) : pk_off(c, r)]);
+                    ninf = fmax(ninf, s);
+                }
+                const double nb = fmin(sqrt(f2), ninf);
+                wlow[i] = (ok && nb > 0.0 && isfinite(nb)) ? 1.0 / nb : 0.0;
+            }
         }
 #pragma unroll
         for (int q = 0; q < 12; ++q) reinterpret_cast<double2*>(out)[q] = make_double2(P[2 * q], P[2 * q + 1]);
@@ -171,11 +183,12 @@ static dda_status_t bj_setup_n(dda_matrix* K, int32_t nrows, cudaStream_t st, in
     if (!K->lfac) {
         DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->lfac), sizeof(double) * kDinv * (size_t)K->n, st));
         DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->sfac), sizeof(double) * kDinv * (size_t)K->n, st));
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->bj_w), sizeof(double) * (size_t)K->n, st));
     }
     K->scaled_valid = false;
     unsigned long long* fmax = reinterpret_cast<unsigned long long*>(reinterpret_cast<char*>(K->scratch) + 192);
     DDA_CK(cudaMemsetAsync(fmax, 0, sizeof(unsigned long long), st));
-    k_bj_inv<<<g, 128, 0, st>>>(nrows, K->diag, K->dinv, full, K->lfac, K->sfac, bad, fmax);
+    k_bj_inv<<<g, 128, 0, st>>>(nrows, K->diag, K->dinv, full, K->lfac, K->sfac, K->bj_w, bad, fmax);
     DDA_LAUNCHED();
     int hbad = 0;
     DDA_CK(cudaMemcpyAsync(&hbad, bad, sizeof(int), cudaMemcpyDeviceToHost, st));

@@ -243,18 +243,27 @@ def _pcg_parity(dda, P, O, pc, omega=1.0, d0=None, tol=1e-10):
     return d, it
 
 
-@pytest.fixture(params=["auto", "graph", "persistent", "scaled"])
-def engine(request, dda):
-    """PCG engine: the CUDA-graph while loop, the persistent cooperative kernel, or the
-    graph loop on the block-scaled matrix S K S^T (block-Jacobi only; other
-    preconditioners fall back to the graph loop) — internal hook; 'auto' picks by
-    size and preconditioner."""
+def _set_engine(dda, engine, loop=-1):
     import ctypes
     f = dda.lib().dda__set_pcg_engine
     f.argtypes = [ctypes.c_int]
-    f({"auto": -1, "graph": 0, "persistent": 1, "scaled": 2}[request.param])
+    f(engine)
+    g = dda.lib().dda__set_scaled_loop
+    g.argtypes = [ctypes.c_int]
+    g(loop)
+
+
+@pytest.fixture(params=["auto", "graph", "persistent", "scaled", "scaled_graph"])
+def engine(request, dda):
+    """PCG engine: the CUDA-graph while loop, the persistent cooperative kernel, or the
+    block-scaled matrix S K S^T (block-Jacobi only; other preconditioners fall back to
+    the graph loop) run by one persistent cooperative kernel ('scaled') or by the
+    CUDA-graph while loop ('scaled_graph') — internal hooks; 'auto' picks by size and
+    preconditioner."""
+    _set_engine(dda, *{"auto": (-1, -1), "graph": (0, -1), "persistent": (1, -1), "scaled": (2, 1),
+                       "scaled_graph": (2, 0)}[request.param])
     yield request.param
-    f(-1)
+    _set_engine(dda, -1, -1)
 
 
 @pytest.mark.parametrize("name", ["tiny", "tiny_shuffled", "ragged_1k", "paper"])
@@ -327,23 +336,21 @@ def test_pcg_warm_start_and_edge_cases(dda, engine):
     assert st5 == dda.ERR_NO_CONVERGENCE and it5 == 200 and rr5 > 1e-10
 
 
-def test_scaled_engine_stopping_test(dda):
+@pytest.mark.parametrize("loop", [1, 0], ids=["persistent", "graph"])
+def test_scaled_engine_stopping_test(dda, loop):
     """The scaled engine evaluates the exact stopping test |L r~| only when lam |r~|^2 allows it to
     pass: it must stop at the same iteration as the unscaled loop with far fewer
-    exact tests than iterations."""
-    import ctypes
-    f = dda.lib().dda__set_pcg_engine
-    f.argtypes = [ctypes.c_int]
+    exact tests than iterations — with either loop driver."""
     P, O = case("paper")
     K = dda.build_from_problem(P)
     F = torch.from_numpy(P.F).cuda()
     try:
-        f(0)
+        _set_engine(dda, 0)
         d0, it0, rr0, st0 = K.pcg_solve(F)
-        f(2)
+        _set_engine(dda, 2, loop)
         d2, it2, rr2, st2 = K.pcg_solve(F)
     finally:
-        f(-1)
+        _set_engine(dda, -1, -1)
     assert st0 == st2 == dda.OK
     assert abs(it0 - it2) <= 1, (it0, it2)
     checks = K.last_checks()
@@ -351,13 +358,37 @@ def test_scaled_engine_stopping_test(dda):
     assert np.linalg.norm(d2.cpu().numpy() - d0.cpu().numpy()) <= 1e-8 * np.linalg.norm(d0.cpu().numpy())
 
 
-def test_pcg_deterministic(dda):
+@pytest.mark.parametrize("eng", [(-1, -1), (2, 1), (2, 0)], ids=["auto", "scaled", "scaled_graph"])
+def test_pcg_deterministic(dda, eng):
     P, O = case("paper")
     K = dda.build_from_problem(P)
     F = torch.from_numpy(P.F).cuda()
-    a = K.pcg_solve(F)[0].cpu().numpy()
-    b = K.pcg_solve(F)[0].cpu().numpy()
+    try:
+        _set_engine(dda, *eng)
+        a = K.pcg_solve(F)[0].cpu().numpy()
+        b = K.pcg_solve(F)[0].cpu().numpy()
+    finally:
+        _set_engine(dda, -1, -1)
     assert np.array_equal(a, b)
+
+
+def test_scaled_loops_agree(dda):
+    """The persistent and the CUDA-graph drivers of the scaled engine run the same iteration; only
+    the CTA count of the r~ update (hence the rounding of one dot product) differs."""
+    P, O = case("paper")
+    K = dda.build_from_problem(P)
+    F = torch.from_numpy(P.F).cuda()
+    out = {}
+    try:
+        for loop in (1, 0):
+            _set_engine(dda, 2, loop)
+            d, it, rr, st = K.pcg_solve(F)
+            out[loop] = (d.cpu().numpy(), it, rr, st, K.last_checks())
+    finally:
+        _set_engine(dda, -1, -1)
+    (dp, itp, rrp, stp, cp), (dg, itg, rrg, stg, cg) = out[1], out[0]
+    assert stp == stg == dda.OK and abs(itp - itg) <= 1 and rrp <= 1e-10 and rrg <= 1e-10
+    assert np.linalg.norm(dp - dg) <= 1e-9 * np.linalg.norm(dg)
 
 
 def test_solve_host_e2e(dda):
