@@ -86,16 +86,17 @@ def pcg_launch_bytes_scaled(n: int, nnzb: int, iters: int, checks: int) -> float
     (DESIGN.md §6), per block row unless noted:
     k_scale_upper: nnzb*(288 V read + 288 written + 8 indices) + n*192 (S);
     k_s_init 384 (F, S read; r~, p, x written);
-    iteration 0: scaled SpMV 300u + 8 + 96 (p read, q written) + k_s_update 144 (r~, q read; r~ written);
+    iteration 0: scaled SpMV 300u + 8 + 96 (p read, q written) + phase B 152 (r~, q read; r~ written;
+    the stopping-test weight w_i, 8 B);
     iterations k >= 1: the SpMV also reads p_old (+48), writes p (+48) and applies the deferred
-    x += alpha p_old (x read + written, +96) + k_s_update 144;
+    x += alpha p_old (x read + written, +96) + phase B 152;
     each exact stopping test (k_s_check, `checks` of them) 240 (r~ + L read);
     k_s_final 336 (x, p, S read; d written); the true-residual SpMV on K + 96 (F, q read)."""
     u = nnzb / n
     it = max(iters, 1)
     sp = 300.0 * u + 8.0 + 96.0
     return (nnzb * 584.0 + n * 192.0
-            + n * (384.0 + (sp + 144.0) + (it - 1) * (sp + 192.0 + 144.0) + 240.0 * checks + 336.0
+            + n * (384.0 + (sp + 152.0) + (it - 1) * (sp + 192.0 + 152.0) + 240.0 * checks + 336.0
                    + bytes_per_row_spmv(u) + 96.0))
 
 
