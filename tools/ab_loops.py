@@ -15,10 +15,11 @@ L = dda.lib()
 L.dda__set_pcg_engine.argtypes = [C.c_int]
 L.dda__set_scaled_loop.argtypes = [C.c_int]
 L.dda__set_pcg_engine(2)
-res = {0: [], 1: []}
+loops = [int(v) for v in (sys.argv[3].split(",") if len(sys.argv) > 3 else ["0", "1"])]
+res = {l: [] for l in loops}
 its = {}
 for r in range(reps + 1):
-    for loop in (0, 1):
+    for loop in loops:
         L.dda__set_scaled_loop(loop)
         K.pcg_solve(t["F"])          # (re)build the engine for this loop kind
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -28,5 +29,6 @@ for r in range(reps + 1):
         its[loop] = (it, rr, K.last_checks())
         if r:
             res[loop].append(a.elapsed_time(b))
-print(json.dumps({"n": K.n, "graph_ms": statistics.median(res[0]), "persistent_ms": statistics.median(res[1]),
-                  "graph_all": res[0], "persistent_all": res[1], "iters_rel_checks": its}), flush=True)
+names = {0: "graph", 1: "persistent"}
+print(json.dumps({"n": K.n, **{names[l] + "_ms": statistics.median(res[l]) for l in loops},
+                  **{names[l] + "_all": res[l] for l in loops}, "iters_rel_checks": its}), flush=True)
