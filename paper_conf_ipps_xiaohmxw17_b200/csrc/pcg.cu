@@ -506,9 +506,9 @@ static int pcg_engine(const dda_matrix* K, dda_precond_t pc) {   // 0 = graph, 1
         forced = !v ? -1 : ((v[0] == 'p' || v[0] == '1') ? 1 : ((v[0] == 's' || v[0] == '2') ? 2 : 0));
     }
     if (pc == DDA_PC_ILU0) return 0;   // the sync-free ILU sweeps exist in the graph engine only
-    if (forced == 2) return pc == DDA_PC_BJ ? 2 : 0;
+    if (forced == 2) return (pc == DDA_PC_BJ || pc == DDA_PC_SSOR_AI) ? 2 : 0;
     if (forced >= 0) return forced;
-    if (pc == DDA_PC_BJ && K->n >= 65536) return 2;
+    if ((pc == DDA_PC_BJ || pc == DDA_PC_SSOR_AI) && K->n >= 65536) return 2;
     return (pc != DDA_PC_SSOR_AI && K->n < 65536) ? 1 : 0;
 }
 

@@ -57,7 +57,7 @@ struct GArgs {           // constant for a (matrix, preconditioner): baked into 
     BsrView A;
     const double* dinv;
     double *r, *z, *p0, *p1, *q, *t, *w;
-    double* part;        // [3][Gmax] CTA partials
+    double* part;        // [4][Gmax] CTA partials
     int Gmax;
     int pc;
     State* st;
@@ -910,6 +910,195 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_loop(const GArgs a) {
     if (tr_k) tr_k[1] = gtimer();
 }
 
+// ---- scaled SSOR-AI (A7) in one persistent kernel
+//
+// The SSOR approximate inverse of reading Z14, M^{-1} = (I - w D^{-1} U) D^{-1} (I - w U^T D^{-1}),
+// is, with D^{-1} = S^T S (S = L^{-1}) and Us = S U S^T (the scaled upper blocks, sc_upper),
+//   M^{-1} = S^T (I - w Us)(I - w Us^T) S,
+// so SSOR-AI PCG on K d = F is PCG on Ks x = S F with M~^{-1} = (I - w Us)(I - w Us^T): the same
+// iterates under r~ = S r, z = S^T z~ (exact arithmetic), and the apply streams no D^{-1}.
+// Per iteration (three grid barriers, three passes over the upper storage):
+//   A  p = z~ + beta p_old (on the fly), q = Ks p, x += alpha_prev p_old; sigma      | barrier
+//   L  r~' = r~ - alpha q (on the fly for gathered lower neighbours, ping-pong r~),
+//      t = r~' - w Us^T r~' (transposed half pass); |r~'|^2 and the w-bound          | barrier
+//      [C: the exact stopping test |L r~'| when the bound allows it                  | barrier]
+//   U  z~ = t - w Us t (upper half pass); rho' = r~' . z~ -> beta                    | barrier
+// Before the loop the same L and U passes with alpha = 0 give z~0 = M~^{-1} r~0.
+
+// x = r - alpha q formed on the fly (the residual update fused into the lower half pass)
+struct XUpdW {
+    const double* r;
+    const double* q;
+    double alpha;
+    using Raw = double2;
+    __device__ __forceinline__ Raw raw(int vec, int pair) const {
+        const size_t o = 6 * (size_t)vec + 2 * pair;
+        const double2 rr = ld_cg2(r + o), qq = ld_cg2(q + o);
+        return make_double2(fma(-alpha, qq.x, rr.x), fma(-alpha, qq.y, rr.y));
+    }
+    __device__ __forceinline__ double2 cook(const Raw& v) const { return v; }
+    __device__ __forceinline__ double2 operator()(int vec, int pair) const { return raw(vec, pair); }
+};
+struct XPlainW {   // coherent loads of a vector written in this launch
+    const double* x;
+    using Raw = double2;
+    __device__ __forceinline__ Raw raw(int vec, int pair) const { return ld_cg2(x + 6 * (size_t)vec + 2 * pair); }
+    __device__ __forceinline__ double2 cook(const Raw& v) const { return v; }
+    __device__ __forceinline__ double2 operator()(int vec, int pair) const { return raw(vec, pair); }
+};
+
+// L pass: r~' (written to rn), t = r~' - w Us^T r~'; returns (|r~'|^2, sum w_i |r~'_i|^2) partials
+__device__ __forceinline__ double2 ssor_lower_pass(const GArgs& a, const BsrView& A, const double* rc, double* rn,
+                                                   const double* qv, double alpha, double omega, int w0, int W) {
+    const int lane = threadIdx.x & 31;
+    const XUpdW xf{rc, qv, alpha};
+    double rr = 0.0, lb = 0.0;
+    for_rows_c<SPMV_LOWER_T, 5>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+        if (ok) {
+            const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
+            const double2 rv = xf(i, ccol_of(lane));
+            *reinterpret_cast<double2*>(rn + o) = rv;
+            *reinterpret_cast<double2*>(a.t + o) = make_double2(fma(-omega, y0, rv.x), fma(-omega, y1, rv.y));
+            const double s = rv.x * rv.x + rv.y * rv.y;
+            rr += s;
+            lb += __ldg(a.bj_w + i) * s;
+        }
+    });
+    return make_double2(rr, lb);
+}
+
+// U pass: z~ = t - w Us t (written to z); returns this lane's share of r~' . z~
+__device__ __forceinline__ double ssor_upper_pass(const GArgs& a, const BsrView& A, const double* rn, double omega,
+                                               int w0, int W) {
+    const int lane = threadIdx.x & 31;
+    const XPlainW xf{a.t};
+    double rz = 0.0;
+    for_rows_c<SPMV_UPPER, 5>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+        if (ok) {
+            const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
+            const double2 tv = xf(i, ccol_of(lane));
+            const double2 zv = make_double2(fma(-omega, y0, tv.x), fma(-omega, y1, tv.y));
+            *reinterpret_cast<double2*>(a.z + o) = zv;
+            const double2 rv = ld_cg2(rn + o);
+            rz += rv.x * zv.x + rv.y * zv.y;
+        }
+    });
+    return rz;
+}
+
+// A pass: p = z~ + beta p_old (own rows written), q = Ks p, x += alpha_prev p_old; returns sigma share
+__device__ __forceinline__ double ssor_spmv_pass(const GArgs& a, const BsrView& A, const double* pold, double* pnew,
+                                              double beta, double alpha_prev, int w0, int W) {
+    const int lane = threadIdx.x & 31;
+    const XFusedW xf{a.z, pold, beta};
+    double* x = a.ca->d;
+    double acc = 0.0;
+    for_rows_c<SPMV_OFFDIAG, 5>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+        if (ok) {
+            const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
+            const double2 pv = xf(i, ccol_of(lane));
+            y0 += pv.x;
+            y1 += pv.y;
+            const double2 po = ld_cg2(pold + o);
+            const double2 xo = ld_cg2(x + o);
+            *reinterpret_cast<double2*>(x + o) = make_double2(xo.x + alpha_prev * po.x, xo.y + alpha_prev * po.y);
+            *reinterpret_cast<double2*>(a.q + o) = make_double2(y0, y1);
+            *reinterpret_cast<double2*>(pnew + o) = pv;
+            acc += pv.x * y0 + pv.y * y1;
+        }
+    });
+    return acc;
+}
+
+// exact stopping test share: |L r~|^2 over this thread's rows
+__device__ __forceinline__ double exact_rr_pass(const GArgs& a, const double* rn, int w0, int W) {
+    const int lane = threadIdx.x & 31;
+    const int n = a.A.n, ngrp = (n + 4) / 5;
+    double rl = 0.0;
+    for (int grp = w0; grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        const double rv = R.valid ? ld_cg(rn + R.idx) : 0.0;
+        const DinvRow Lrow = tri_row(a.lfac, R);
+        const double o0 = dinv_row_apply(Lrow, rv, R);
+        const double o = R.valid ? o0 : 0.0;
+        rl += o * o;
+    }
+    return rl;
+}
+
+__global__ void __launch_bounds__(DDA_THREADS, 3) k_sp_ssor(const GArgs a) {
+    cg::grid_group grid = cg::this_grid();
+    State* st = a.st;
+    if (st->done) return;                                   // decided at setup (uniform: no barrier reached)
+    const double thr = a.ca->tol * st->bnorm, omega = a.ca->omega;
+    const int maxit = a.ca->maxit;
+    BsrView A = a.A;
+    A.upper = a.su;
+    const int w0 = blockIdx.x * WPB + (threadIdx.x >> 5), W = gridDim.x * WPB;
+    double* rb[2] = {a.r, a.w};                             // r~ ping-pong (a.w is free in this engine)
+    int ri = 0;
+    double rho, alpha = 0.0, beta = 0.0, rr_last = st->rr;
+    int k = 0, status = DDA_ERR_NO_CONVERGENCE, iters = 0, checks = 0, pend = 0;
+    {   // z~0 = M~^{-1} r~0, rho0 = r~0 . z~0
+        const double2 lr = ssor_lower_pass(a, A, rb[ri], rb[ri ^ 1], rb[ri], 0.0, omega, w0, W);   // q = r: no NaN
+        (void)lr;
+        ri ^= 1;
+        grid.sync();
+        const double rz0 = ssor_upper_pass(a, A, rb[ri], omega, w0, W);
+        double v[1] = {rz0}, t[1];
+        grid_allsum<1>(a, grid, 3, v, t);
+        rho = t[0];
+        if (!(rho > 0.0) || !isfinite(rho)) status = DDA_ERR_BREAKDOWN;
+    }
+    while (status != DDA_ERR_BREAKDOWN) {
+        double* pnew = (k & 1) ? a.p1 : a.p0;
+        const double* pold = k == 0 ? a.z : ((k & 1) ? a.p0 : a.p1);
+        const double sg = ssor_spmv_pass(a, A, pold, pnew, beta, alpha, w0, W);
+        double sv[1] = {sg}, stt[1];
+        grid_allsum<1>(a, grid, 0, sv, stt);
+        pend = 0;
+        const double sigma = stt[0];
+        if (!(sigma > 0.0) || !isfinite(sigma)) { status = DDA_ERR_BREAKDOWN; break; }   // reading Z19
+        alpha = rho / sigma;
+        const double2 lr = ssor_lower_pass(a, A, rb[ri], rb[ri ^ 1], a.q, alpha, omega, w0, W);
+        ri ^= 1;
+        double lv[2] = {lr.x, lr.y}, lt[2];
+        grid_allsum<2>(a, grid, 1, lv, lt);
+        pend = 1;                                           // x += alpha p_k: next A pass or k_s_final
+        iters = k + 1;
+        const double rr1 = lt[0];
+        if (rr1 == 0.0) { status = DDA_OK; rr_last = 0.0; k = k + 1; break; }
+        if (isfinite(rr1) && !(0.999 * lt[1] > thr * thr)) {
+            const double rl = exact_rr_pass(a, rb[ri], w0, W);
+            double cv[1] = {rl}, ct[1];
+            grid_allsum<1>(a, grid, 0, cv, ct);
+            checks += 1;
+            rr_last = ct[0];
+            if (sqrt(ct[0]) <= thr) { status = DDA_OK; k = k + 1; break; }
+        }
+        const double rz = ssor_upper_pass(a, A, rb[ri], omega, w0, W);
+        double uv[1] = {rz}, ut[1];
+        grid_allsum<1>(a, grid, 3, uv, ut);
+        const double rho1 = ut[0];
+        k = k + 1;
+        if (!(rho1 > 0.0) || !isfinite(rho1)) { status = DDA_ERR_BREAKDOWN; break; }
+        beta = rho1 / rho;
+        rho = rho1;
+        if (k >= maxit) { status = DDA_ERR_NO_CONVERGENCE; break; }
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {              // the State k_s_final / k_g_resid read
+        st->k = k;
+        st->iters = iters;
+        st->status = status;
+        st->done = 1;
+        st->alpha = alpha;
+        st->beta = beta;
+        st->rr = rr_last;
+        st->pend = pend;
+        st->checks = checks;
+    }
+}
+
 // loop-body SpMV kernel variants (tuning aid, DDA_GSPMV_VARIANT): occupancy / register budget
 typedef void (*GSpmvKernel)(const GArgs, cudaGraphConditionalHandle);
 struct GSpmvVariant { GSpmvKernel plain, scaled; int minb; };
@@ -994,7 +1183,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
                              cudaStream_t st, bool scaled) {
     const size_t N = 6 * (size_t)K->n;
     if (scaled) {
-        if (pc != DDA_PC_BJ) return DDA_ERR_ARG;
+        if (pc != DDA_PC_BJ && pc != DDA_PC_SSOR_AI) return DDA_ERR_ARG;
         dda_status_t s = scaled_setup(K, st);
         if (s != DDA_OK) return s;
     }
@@ -1005,7 +1194,10 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         const char* e = getenv("DDA_SCALED_LOOP");
         g_scaled_loop = (e && (e[0] == 'g' || e[0] == '0')) ? 0 : 1;
     }
-    const bool persist = scaled && g_scaled_loop == 1;
+    // scaled SSOR-AI exists as a persistent kernel only (k_sp_ssor)
+    const bool persist = scaled && (g_scaled_loop == 1 || pc == DDA_PC_SSOR_AI);
+    const void* persist_kernel = pc == DDA_PC_SSOR_AI ? reinterpret_cast<const void*>(k_sp_ssor)
+                                                      : reinterpret_cast<const void*>(k_sp_loop<3>);
     const int key = scaled ? (persist ? 200 : 100) + (int)pc : (int)pc;
     PcgGraph*& G = reinterpret_cast<PcgGraph*&>(K->graph_engine);
     if (G && G->pc != key) {
@@ -1025,13 +1217,13 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         int g_persist = 0;
         if (persist) {   // every CTA must be co-resident (cooperative launch)
             int per_sm = 0;
-            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_sp_loop<3>, DDA_THREADS, 0);
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, persist_kernel, DDA_THREADS, 0);
             if (per_sm > 3) per_sm = 3;
             if (per_sm < 1) return DDA_ERR_CUDA;
             g_persist = device_sms() * per_sm;
             if (g_persist > Gmax) Gmax = g_persist;
         }
-        const size_t bytes = (7 * N + 3 * (size_t)Gmax) * sizeof(double) + sizeof(CallArgs) + sizeof(State) + 64;
+        const size_t bytes = (7 * N + 4 * (size_t)Gmax) * sizeof(double) + sizeof(CallArgs) + sizeof(State) + 64;
         // may reallocate the workspace (and drop any engine holding the old pointers): do it first
         dda_status_t s = ensure_workspace(K, bytes, st);
         if (s != DDA_OK) return s;
@@ -1048,7 +1240,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         a.w = ws + 6 * N;
         a.part = ws + 7 * N;
         a.Gmax = Gmax;
-        char* tail = reinterpret_cast<char*>(a.part + 3 * (size_t)Gmax);
+        char* tail = reinterpret_cast<char*>(a.part + 4 * (size_t)Gmax);
         a.ca = reinterpret_cast<CallArgs*>(tail);
         a.st = reinterpret_cast<State*>(tail + ((sizeof(CallArgs) + 15) / 16) * 16);
         a.pc = (int)pc;
@@ -1140,7 +1332,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     else
         k_g_init<<<G->G_vec, DDA_THREADS, 0, st>>>(a);
     DDA_LAUNCHED();
-    if (pc == DDA_PC_SSOR_AI) {
+    if (pc == DDA_PC_SSOR_AI && !scaled) {
         k_g_ssor_lower<true><<<G->G_spmv, DDA_THREADS, 0, st>>>(a);
         DDA_LAUNCHED();
         k_g_ssor_upper<true><<<G->G_spmv, DDA_THREADS, 0, st>>>(a, G->h);
@@ -1158,7 +1350,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         a.trace = g_trace;
         a.trace_iters = g_trace_iters;
         void* kargs[] = {reinterpret_cast<void*>(&a)};
-        DDA_CK(cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_sp_loop<3>), dim3(G->G_persist),
+        DDA_CK(cudaLaunchCooperativeKernel(persist_kernel, dim3(G->G_persist),
                                            dim3(DDA_THREADS), kargs, 0, st));
         DDA_LAUNCHED();
     } else {

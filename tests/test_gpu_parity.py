@@ -398,3 +398,21 @@ def test_solve_host_e2e(dda):
     d2, it2, rr2, st2 = K.pcg_solve(torch.from_numpy(P.F).cuda())
     assert st == st2 == dda.OK and it == it2
     assert np.array_equal(d, d2.cpu().numpy())
+
+
+@pytest.mark.parametrize("name", ["tiny", "paper"])
+def test_scaled_ssor_omega0_is_bj(dda, name):
+    """SSOR-AI with omega = 0 is M^{-1} = D^{-1} (reading Z14): the scaled SSOR-AI kernel must take the
+    iterations of block-Jacobi and reach the same solution."""
+    P, O = case(name)
+    K = dda.build_from_problem(P)
+    F = torch.from_numpy(P.F).cuda()
+    try:
+        _set_engine(dda, 2, 1)
+        db, itb, rrb, stb = K.pcg_solve(F, precond="bj")
+        ds, its, rrs, sts = K.pcg_solve(F, precond="ssor_ai", omega=0.0)
+    finally:
+        _set_engine(dda, -1, -1)
+    assert stb == sts == dda.OK and itb == its, (itb, its)
+    db, ds = db.cpu().numpy(), ds.cpu().numpy()
+    assert np.linalg.norm(ds - db) <= 1e-12 * np.linalg.norm(db)
