@@ -488,12 +488,12 @@ dda_status_t pcg_solve(dda_matrix* K, const double* F, const double* d0, double*
 
 using namespace dda;
 
-// Engine choice: the CUDA-graph while loop (one kernel per phase, each at its
-// own occupancy) wins when the phases are HBM-bound; the persistent cooperative
-// kernel (grid barriers instead of kernel boundaries) wins for L2-resident
-// block-Jacobi solves (10k blocks: 15.5 vs 18.6 us/iteration on B200).  For
-// HBM-bound block-Jacobi solves the graph loop runs on the block-scaled matrix
-// S K S^T (pcg_graph.cu, "scaled BJ engine": same iterates, 18% fewer bytes).
+// Engine choice: block-Jacobi and SSOR-AI run the scaled engine (pcg_graph.cu: PCG on S K S^T,
+// same iterates, no D / D^{-1} in the loop) in one persistent cooperative kernel at every size: at
+// 10k blocks (L2-resident, barrier-latency bound, grid capped to the rows) 9.8 us per iteration vs
+// 15.0 for the unscaled persistent kernel; at 30k 15.8 vs 28.4; at 1M 304 vs 456.  ILU(0) and the
+// unpreconditioned solve run the unscaled engines: the CUDA-graph while loop (ILU, and "none" from
+// 64k blocks) or the persistent kernel on K ("none" below 64k).
 // DDA_PCG_ENGINE=graph|persistent|scaled overrides.
 static int g_forced_engine = -2;
 // Internal testing hook (not in include/dda.h): -1 = automatic, 0 = graph, 1 = persistent, 2 = scaled.
@@ -508,7 +508,7 @@ static int pcg_engine(const dda_matrix* K, dda_precond_t pc) {   // 0 = graph, 1
     if (pc == DDA_PC_ILU0) return 0;   // the sync-free ILU sweeps exist in the graph engine only
     if (forced == 2) return (pc == DDA_PC_BJ || pc == DDA_PC_SSOR_AI) ? 2 : 0;
     if (forced >= 0) return forced;
-    if ((pc == DDA_PC_BJ || pc == DDA_PC_SSOR_AI) && K->n >= 65536) return 2;
+    if (pc == DDA_PC_BJ || pc == DDA_PC_SSOR_AI) return 2;   // scaled engine at every size
     return (pc != DDA_PC_SSOR_AI && K->n < 65536) ? 1 : 0;
 }
 

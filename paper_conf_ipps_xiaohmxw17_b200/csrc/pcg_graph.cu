@@ -1221,6 +1221,10 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
             if (per_sm > 3) per_sm = 3;
             if (per_sm < 1) return DDA_ERR_CUDA;
             g_persist = device_sms() * per_sm;
+            // small (L2-resident) systems are barrier-latency bound: no more CTAs than ten-row groups
+            // need (DDA_PERSIST_CTAS overrides, tuning aid)
+            const int cap = env_int("DDA_PERSIST_CTAS", need_rows > 0 ? need_rows : 1);
+            if (cap > 0 && g_persist > cap) g_persist = cap;
             if (g_persist > Gmax) Gmax = g_persist;
         }
         const size_t bytes = (7 * N + 4 * (size_t)Gmax) * sizeof(double) + sizeof(CallArgs) + sizeof(State) + 64;
