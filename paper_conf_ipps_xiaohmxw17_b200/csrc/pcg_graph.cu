@@ -1099,6 +1099,31 @@ __global__ void __launch_bounds__(DDA_THREADS, 3) k_sp_ssor(const GArgs a) {
     }
 }
 
+// Experiment kernels (internal timing hook dda__time_ks_variants): the bare off-diagonal Ks product
+// q = Ks p with sigma, gathering ONE vector, through the read-only path (LDG) or coherent loads.
+template <bool LDG, int MINB>
+__global__ void __launch_bounds__(DDA_THREADS, MINB) k_x_ks(const GArgs a) {
+    BsrView A = a.A;
+    A.upper = a.su;
+    const int lane = threadIdx.x & 31;
+    const int w0 = blockIdx.x * WPB + (threadIdx.x >> 5), W = gridDim.x * WPB;
+    double acc = 0.0;
+    auto body = [&](const auto& xf) {
+        for_rows_c<SPMV_OFFDIAG, 5>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+            if (ok) {
+                const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
+                const double2 pv = xf(i, ccol_of(lane));
+                y0 += pv.x;
+                y1 += pv.y;
+                *reinterpret_cast<double2*>(a.q + o) = make_double2(y0, y1);
+                acc += pv.x * y0 + pv.y * y1;
+            }
+        });
+    };
+    if (LDG) body(XPlain{a.p0}); else body(XPlainW{a.p0});
+    if (acc == 12345.678) a.part[0] = acc;   // keep the dot product live
+}
+
 // loop-body SpMV kernel variants (tuning aid, DDA_GSPMV_VARIANT): occupancy / register budget
 typedef void (*GSpmvKernel)(const GArgs, cudaGraphConditionalHandle);
 struct GSpmvVariant { GSpmvKernel plain, scaled; int minb; };
@@ -1481,4 +1506,38 @@ extern "C" int dda__get_scaled_loop() {
         return (e && (e[0] == 'g' || e[0] == '0')) ? 0 : 1;
     }
     return dda::g_scaled_loop;
+}
+
+// Internal timing hook (experiment): ms[0..3] = k_x_ks<LDG=1,3>, k_x_ks<0,3>, k_x_ks<1,4>, k_x_ks<0,4>
+// (bare Ks products at 3 and 4 CTAs/SM) and ms[4] = the fused scaled k_g_spmv, averaged over reps.
+extern "C" int dda__time_ks_variants(dda_matrix_t K, const double* F, double* d, int reps, float* ms) {
+    using namespace dda;
+    cudaStream_t st = 0;
+    float dummy[2];
+    if (dda__time_pcg_phases_ex(K, F, d, 1, dummy, 1) != 0) return -1;
+    PcgGraph* G = reinterpret_cast<PcgGraph*>(K->graph_engine);
+    GArgs a = G->a;
+    a.use_cond = 0;
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0); cudaEventCreate(&e1);
+    const int g3 = device_sms() * 3, g4 = device_sms() * 4;
+    for (int v = 0; v < 5; ++v) {
+        float tot = 0;
+        for (int r = 0; r < reps + 1; ++r) {
+            cudaEventRecord(e0, st);
+            if (v == 0) k_x_ks<true, 3><<<g3, DDA_THREADS, 0, st>>>(a);
+            if (v == 1) k_x_ks<false, 3><<<g3, DDA_THREADS, 0, st>>>(a);
+            if (v == 2) k_x_ks<true, 4><<<g4, DDA_THREADS, 0, st>>>(a);
+            if (v == 3) k_x_ks<false, 4><<<g4, DDA_THREADS, 0, st>>>(a);
+            if (v == 4) gspmv_variant().scaled<<<G->G_spmv, DDA_THREADS, 0, st>>>(a, 0);
+            cudaEventRecord(e1, st);
+            cudaEventSynchronize(e1);
+            float x;
+            cudaEventElapsedTime(&x, e0, e1);
+            if (r) tot += x;
+        }
+        ms[v] = tot / reps;
+    }
+    cudaEventDestroy(e0); cudaEventDestroy(e1);
+    return cudaGetLastError() == cudaSuccess ? 0 : -3;
 }
