@@ -62,6 +62,12 @@ def lib():
         L.orc_pcg.argtypes = [P, P, P, P, C.c_double, C.c_int32, C.c_int32, C.c_double,
                               C.POINTER(C.c_int32), C.POINTER(C.c_double), P]
         L.orc_ldlt_solve.argtypes = [P, P, P]
+        L.orc_detect_contacts.argtypes = [C.c_int32, P, P, C.c_double, C.c_int32, C.c_int32, C.c_int64,
+                                          P, P, P, P, P, P, P]
+        L.orc_detect_contacts.restype = C.c_int64
+        L.orc_contact_springs.argtypes = [C.c_int32, P, P, P, C.c_int64, P, P, P, P, P, P, C.c_double,
+                                          C.c_double, P, P, P, P, P]
+        L.orc_contact_springs.restype = C.c_int64
         _lib = L
     return _lib
 
@@ -204,3 +210,50 @@ class OracleMatrix:
 
 def assemble(P) -> OracleMatrix:
     return OracleMatrix.from_problem(P)
+
+
+# ---------------------------------------------------------------- NEXT-3: contacts (O-8, O-9)
+
+CONTACT_FIELDS = ("i", "v", "j", "e", "type", "t", "dist2")
+
+
+def detect_contacts(vptr, vxy, d0, v_begin=0, v_end=None) -> dict:
+    """O-8: every (vertex v of block i, edge e of block j != i) with distance < d0, in increasing
+    (v, e); fields i, v, j, e (int32), type (0 VE, 1 VV), t (edge ratio), dist2."""
+    vptr = np.ascontiguousarray(vptr, np.int32)
+    vxy = np.ascontiguousarray(vxy, np.float64).reshape(-1, 2)
+    n = vptr.shape[0] - 1
+    v_end = int(vptr[-1]) if v_end is None else int(v_end)
+    L = lib()
+    out = None
+    cap = 0
+    while True:
+        out = {k: np.empty(max(cap, 1), np.int32) for k in CONTACT_FIELDS[:5]}
+        out["t"] = np.empty(max(cap, 1))
+        out["dist2"] = np.empty(max(cap, 1))
+        cnt = L.orc_detect_contacts(n, _p(vptr), _p(vxy), float(d0), int(v_begin), v_end, cap,
+                                    *[_p(out[k]) for k in CONTACT_FIELDS])
+        if cnt < 0:
+            raise OracleError(ERR_ARG, "detect_contacts")
+        if cnt <= cap:
+            return {k: a[:cnt] for k, a in out.items()}
+        cap = int(cnt)
+
+
+def contact_springs(vptr, vxy, cxy, C_, p_n, shear_ratio) -> dict:
+    """O-9: normal + shear spring of every VE contact, in record order (bi, bj, pen, e, g)."""
+    vptr = np.ascontiguousarray(vptr, np.int32)
+    vxy = np.ascontiguousarray(vxy, np.float64).reshape(-1, 2)
+    cxy = np.ascontiguousarray(cxy, np.float64).reshape(-1, 2)
+    nc = int(C_["i"].shape[0])
+    nve = int((C_["type"] == 0).sum())
+    m = 2 * nve
+    o = {"bi": np.empty(max(m, 1), np.int32), "bj": np.empty(max(m, 1), np.int32), "pen": np.empty(max(m, 1)),
+         "e": np.empty((max(m, 1), 6)), "g": np.empty((max(m, 1), 6))}
+    f = [np.ascontiguousarray(C_[k], np.int32) for k in ("i", "v", "j", "e", "type")]
+    t = np.ascontiguousarray(C_["t"], np.float64)
+    got = lib().orc_contact_springs(vptr.shape[0] - 1, _p(vptr), _p(vxy), _p(cxy), nc, *[_p(a) for a in f], _p(t),
+                                    float(p_n), float(shear_ratio), _p(o["bi"]), _p(o["bj"]), _p(o["pen"]),
+                                    _p(o["e"]), _p(o["g"]))
+    assert got == m
+    return {k: a[:m] for k, a in o.items()}

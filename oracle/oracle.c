@@ -611,3 +611,112 @@ int orc_ldlt_solve(orc_matrix *M, const double *b, double *x) {
     free(A); free(D);
     return ORC_OK;
 }
+
+/*
+ * O-8 (NEXT-3)  Contact detection: the narrow phase's distance judgment and its VE / VV
+ * classification (§III.B; §III.A).  Plain definition, all pairs, no
+ * broad phase.  Blocks are polygons: block b owns vertices vptr[b] .. vptr[b+1]-1 of vxy[V][2],
+ * counter-clockwise; edge e of block b runs from vertex e to the next vertex of b (cyclically).
+ * For every vertex v (of block i) in [v_begin, v_end) and every edge e of every block j != i:
+ *     d = Q2 - Q1,  w = P - Q1,  L2 = d.d,  tn = w.d,  t = clamp(tn / L2, 0, 1),
+ *     C = Q1 + t d,  dist2 = |P - C|^2          (each product and sum rounded as written)
+ * (v, e) is a contact iff dist2 < d0^2; its type is VE (0) if 0 < tn < L2 (the nearest point of
+ * the edge is interior) and VV (1) otherwise (the nearest point is the vertex Q1 or Q2).
+ * Records come out in increasing (v, e), i.e. increasing (i, v, j, e).  At most `cap` are
+ * written; the return value is the total count (or -1 on bad arguments).
+ */
+int64_t orc_detect_contacts(int32_t n, const int32_t *vptr, const double *vxy, double d0, int32_t v_begin,
+                            int32_t v_end, int64_t cap, int32_t *ci, int32_t *cv, int32_t *cj, int32_t *ce,
+                            int32_t *ctype, double *ct, double *cd2) {
+    if (n <= 0 || !vptr || !vxy || !(d0 > 0.0)) return -1;
+    const double r2 = d0 * d0;
+    int64_t cnt = 0;
+    int32_t i = 0;
+    for (int32_t v = v_begin; v < v_end; ++v) {
+        while (!(vptr[i] <= v && v < vptr[i + 1])) ++i;      /* block of vertex v (v ascending) */
+        const double px = vxy[2 * v], py = vxy[2 * v + 1];
+        for (int32_t j = 0; j < n; ++j) {
+            if (j == i) continue;
+            const int32_t a = vptr[j], b = vptr[j + 1];
+            for (int32_t e = a; e < b; ++e) {
+                const int32_t e2 = (e + 1 < b) ? e + 1 : a;
+                const double q1x = vxy[2 * e], q1y = vxy[2 * e + 1];
+                const double dx = vxy[2 * e2] - q1x, dy = vxy[2 * e2 + 1] - q1y;
+                const double wx = px - q1x, wy = py - q1y;
+                const double L2 = dx * dx + dy * dy;
+                const double tn = wx * dx + wy * dy;
+                double t = tn / L2;
+                if (t < 0.0) t = 0.0;
+                if (t > 1.0) t = 1.0;
+                const double cx = q1x + t * dx, cy = q1y + t * dy;
+                const double ex = px - cx, ey = py - cy;
+                const double dist2 = ex * ex + ey * ey;
+                if (dist2 < r2) {
+                    if (cnt < cap) {
+                        ci[cnt] = i; cv[cnt] = v; cj[cnt] = j; ce[cnt] = e;
+                        ctype[cnt] = (tn > 0.0 && tn < L2) ? 0 : 1;
+                        ct[cnt] = t; cd2[cnt] = dist2;
+                    }
+                    ++cnt;
+                }
+            }
+        }
+    }
+    return cnt;
+}
+
+/* T(P)^T u for Shi's first-order displacement function at offset (x, y) from the block centroid
+ * (rows of T: [1, 0, -y, x, 0, y/2] and [0, 1, x, 0, y, x/2]; external, Shi 1988). */
+static void tt_times(double x, double y, double ux, double uy, double *o) {
+    o[0] = ux;
+    o[1] = uy;
+    o[2] = -y * ux + x * uy;
+    o[3] = x * ux;
+    o[4] = y * uy;
+    o[5] = 0.5 * y * ux + 0.5 * x * uy;
+}
+
+/*
+ * O-9 (NEXT-3)  Springs of the VE contacts (the input of O-1): for each record with type
+ * VE, in record order, a normal spring then a shear spring (every contact "lock"; the open-close
+ * state switch is NEXT-4).  With u = d / |d| the edge tangent and nrm = (u.y, -u.x) the outward
+ * normal of the counter-clockwise edge, P the vertex of block i, Q1, Q2 the edge of block j and
+ * t the record's edge ratio:
+ *     e = T_i(P)^T n,   g = -((1 - t) T_j(Q1)^T n + t T_j(Q2)^T n),   n = nrm (normal) or u (shear)
+ * penalties p_n and shear_ratio * p_n.  Writes 2 * (#VE) springs; returns that count.
+ */
+int64_t orc_contact_springs(int32_t n, const int32_t *vptr, const double *vxy, const double *cxy, int64_t nc,
+                            const int32_t *ci, const int32_t *cv, const int32_t *cj, const int32_t *ce,
+                            const int32_t *ctype, const double *ct, double p_n, double shear_ratio,
+                            int32_t *bi, int32_t *bj, double *pen, double *e, double *g) {
+    int64_t s = 0;
+    (void)n;
+    for (int64_t k = 0; k < nc; ++k) {
+        if (ctype[k] != 0) continue;
+        const int32_t i = ci[k], j = cj[k], v = cv[k], q = ce[k];
+        const int32_t q2 = (q + 1 < vptr[j + 1]) ? q + 1 : vptr[j];
+        const double dx = vxy[2 * q2] - vxy[2 * q], dy = vxy[2 * q2 + 1] - vxy[2 * q + 1];
+        const double len = sqrt(dx * dx + dy * dy);
+        const double ux = dx / len, uy = dy / len;
+        const double t = ct[k];
+        const double pix = vxy[2 * v] - cxy[2 * i], piy = vxy[2 * v + 1] - cxy[2 * i + 1];
+        const double q1x = vxy[2 * q] - cxy[2 * j], q1y = vxy[2 * q + 1] - cxy[2 * j + 1];
+        const double q2x = vxy[2 * q2] - cxy[2 * j], q2y = vxy[2 * q2 + 1] - cxy[2 * j + 1];
+        for (int sp = 0; sp < 2; ++sp) {
+            const double nx = sp == 0 ? uy : ux, ny = sp == 0 ? -ux : uy;
+            double a[6], b1[6], b2[6];
+            tt_times(pix, piy, nx, ny, a);
+            tt_times(q1x, q1y, nx, ny, b1);
+            tt_times(q2x, q2y, nx, ny, b2);
+            bi[s] = i;
+            bj[s] = j;
+            pen[s] = sp == 0 ? p_n : shear_ratio * p_n;
+            for (int r = 0; r < 6; ++r) {
+                e[6 * s + r] = a[r];
+                g[6 * s + r] = -((1.0 - t) * b1[r] + t * b2[r]);
+            }
+            ++s;
+        }
+    }
+    return s;
+}

@@ -63,6 +63,12 @@ class SlopeProblem:
     F: np.ndarray               # [6n] float64 load vector
     course: np.ndarray          # [n] int32 course index of each block
     n_contacts: int
+    # geometry (NEXT-3 inputs; block ids after the optional shuffle):
+    verts: np.ndarray = None    # [n, 4, 2] jittered polygon vertices, counter-clockwise
+    centroid: np.ndarray = None  # [n, 2]
+    # the generator's own contacts (vertex cv = 4*i + k of block i against edge ce = 4*j + c of
+    # block j, running to the next vertex of j; tau = edge ratio), before any spring permutation
+    contacts: dict = None
 
     @property
     def m(self) -> int:
@@ -243,6 +249,7 @@ def make_slope(cfg: SlopeConfig) -> SlopeProblem:
     ci = np.concatenate(ci); ck = np.concatenate(ck); cj = np.concatenate(cj)
     c2 = np.concatenate(c2); c3 = np.concatenate(c3)
     nc = ci.size
+    assert ((c2 + 1) % 4 == c3).all()           # every contact edge runs to the next CCW vertex
 
     P1 = V[ci, ck]; P2 = V[cj, c2]; P3 = V[cj, c3]
     d = P3 - P2
@@ -295,16 +302,23 @@ def make_slope(cfg: SlopeConfig) -> SlopeProblem:
     F += 0.1 * area.mean() * rng.standard_normal((n, 6))
     F = F.reshape(-1)
 
+    cent = np.stack([cx, cy], axis=1)
+    cbi, cbj = ci, cj
     if cfg.shuffle:
         perm = rng.permutation(n)               # old id b -> new id perm[b]
         inv = np.empty_like(perm); inv[perm] = np.arange(n)
         kd = kd[inv]; course = course[inv]
         F = F.reshape(n, 6)[inv].reshape(-1)
         bi = perm[bi].astype(np.int32); bj = perm[bj].astype(np.int32)
+        V = V[inv]; cent = cent[inv]
+        cbi, cbj = perm[ci], perm[cj]
+    contacts = {"i": cbi.astype(np.int32), "v": (4 * cbi + ck).astype(np.int32), "j": cbj.astype(np.int32),
+                "e": (4 * cbj + c2).astype(np.int32), "tau": tau}
 
     return SlopeProblem(cfg=cfg, n=n, kdiag=np.ascontiguousarray(kd), bi=bi, bj=bj,
                         pen=pen, e=e, g=g, F=np.ascontiguousarray(F),
-                        course=course.astype(np.int32), n_contacts=int(nc))
+                        course=course.astype(np.int32), n_contacts=int(nc),
+                        verts=np.ascontiguousarray(V), centroid=np.ascontiguousarray(cent), contacts=contacts)
 
 
 def random_vector(n_blocks: int, seed: int) -> np.ndarray:
