@@ -239,6 +239,44 @@ void dda_comm_free(dda_comm_t c);
 dda_status_t dda_rcm_order(int32_t n_blocks, int64_t n_springs, const int32_t *bi, const int32_t *bj,
                            int32_t *perm);
 
+/*
+ * NEXT-3 — contact detection on the GPU (§III.B): the narrow phase's distance
+ * judgment and its VE / VV classification, and the springs of the VE contacts that feed
+ * dda_build_matrix (P:96 contact edge ratio).
+ *
+ * Geometry (device, caller-owned, valid until dda_contacts_free): block b is the polygon of vertices
+ * vptr[b] .. vptr[b+1]-1 of vxy [V][2] (x, y interleaved, 16 B aligned), counter-clockwise, >= 3
+ * vertices; edge e of block b runs from vertex e to the next vertex of b (cyclically).
+ * dda_detect_contacts records every (vertex v of block i, edge e of block j != i) with
+ *     d = Q2 - Q1, w = P - Q1, L2 = d.d, tn = w.d, t = clamp(tn / L2, 0, 1), C = Q1 + t d,
+ *     dist2 = |P - C|^2 < d0^2      (each product and sum rounded as written),
+ * typed VE (0) if 0 < tn < L2 and VV (1) otherwise (reading N3), in increasing (v, e).
+ * The contact arrays are library-owned device memory (dda_contacts_t).  DDA_ERR_ARG: n <= 0, null
+ * or misaligned pointers, d0 not positive and finite, a polygon with < 3 vertices or a non-finite
+ * coordinate.  The call synchronises the stream (counts are read back).
+ */
+typedef struct dda_contacts *dda_contacts_t;
+dda_status_t dda_detect_contacts(int32_t n_blocks, const int32_t *vptr, const double *vxy, double d0,
+                                 void *stream, dda_contacts_t *out);
+/* count = records, n_ve = VE records (each yields 2 springs), n_pairs = broad-phase candidate pairs */
+dda_status_t dda_contacts_info(dda_contacts_t C, int64_t *count, int64_t *n_ve, int64_t *n_pairs);
+/* host buffers of `count` entries (any may be NULL): i, v, j, e, type, t, dist2 */
+dda_status_t dda_contacts_export(dda_contacts_t C, int32_t *i, int32_t *v, int32_t *j, int32_t *e,
+                                 int32_t *type, double *t, double *dist2);
+/*
+ * Springs of the VE records, in record order, each a normal then a shear spring (every contact
+ * "lock"; the open-close state switch is NEXT-4, out of scope): with u = d/|d| the edge tangent and
+ * nrm = (u.y, -u.x) the outward normal of the counter-clockwise edge,
+ *     e = T_i(P)^T n,  g = -((1 - t) T_j(Q1)^T n + t T_j(Q2)^T n),  n = nrm (normal) or u (shear),
+ * T Shi's first-order displacement matrix at the offset from the block centroid cxy [n][2] (device),
+ * penalties p_n and shear_ratio * p_n.  Outputs (device, caller-owned, 2 * n_ve entries; e, g
+ * [2 n_ve][6] 16 B aligned) are exactly dda_build_matrix's spring inputs (bi = vertex block i,
+ * bj = edge block j).  Stream-ordered, no synchronisation.
+ */
+dda_status_t dda_contact_springs(dda_contacts_t C, const double *cxy, double p_n, double shear_ratio,
+                                 int32_t *bi, int32_t *bj, double *pen, double *e, double *g, void *stream);
+void dda_contacts_free(dda_contacts_t C);
+
 /* Number of kernel launches the library has issued in this process (for the
  * benchmark's gpu_launches count). */
 int64_t dda_launch_count(void);

@@ -28,7 +28,8 @@ ABI_SYMBOLS = ("dda_build_matrix", "dda_update_values", "dda_matrix_info", "dda_
                "dda_matrix_free", "dda_status_string", "dda_last_cuda_error", "dda_comm_unique_id",
                "dda_comm_init", "dda_comm_init_loopback", "dda_dist_attach", "dda_spmv_dist",
                "dda_pcg_solve_dist", "dda_comm_free", "dda_spmv_full", "dda_rcm_order",
-               "dda_memory_release", "dda_memory_cached")
+               "dda_memory_release", "dda_memory_cached", "dda_detect_contacts", "dda_contacts_info",
+               "dda_contacts_export", "dda_contact_springs", "dda_contacts_free")
 
 _lib = None
 
@@ -99,6 +100,16 @@ def lib() -> C.CDLL:
         L.dda_memory_release.restype = None
         L.dda_memory_cached.argtypes = []
         L.dda_memory_cached.restype = I64
+        L.dda_detect_contacts.argtypes = [I32, P, P, D, P, C.POINTER(P)]
+        L.dda_detect_contacts.restype = st
+        L.dda_contacts_info.argtypes = [P, C.POINTER(I64), C.POINTER(I64), C.POINTER(I64)]
+        L.dda_contacts_info.restype = st
+        L.dda_contacts_export.argtypes = [P] * 8
+        L.dda_contacts_export.restype = st
+        L.dda_contact_springs.argtypes = [P, P, D, D, P, P, P, P, P, P]
+        L.dda_contact_springs.restype = st
+        L.dda_contacts_free.argtypes = [P]
+        L.dda_contacts_free.restype = None
         L.dda__last_checks.argtypes = [P]
         L.dda__last_checks.restype = C.c_int
         L.dda__pcg_engine.argtypes = [P, C.c_int]
@@ -414,3 +425,65 @@ def renumber(perm, kdiag, bi, bj, F=None):
     if F is not None:
         out = out + (np.ascontiguousarray(np.asarray(F).reshape(-1, 6)[perm].reshape(-1)),)
     return out
+
+
+# ---------------------------------------------------------------- NEXT-3: contact detection
+
+class Contacts:
+    """Library-owned contact records of dda_detect_contacts (include/dda.h)."""
+
+    def __init__(self, handle, vptr, vxy):
+        self._h = handle
+        self._keep = (vptr, vxy)          # the library reads the geometry again in springs()
+        cnt, nve, npr = C.c_int64(), C.c_int64(), C.c_int64()
+        _check(lib().dda_contacts_info(self._h, C.byref(cnt), C.byref(nve), C.byref(npr)), "dda_contacts_info")
+        self.count, self.n_ve, self.n_pairs = int(cnt.value), int(nve.value), int(npr.value)
+
+    def free(self):
+        if self._h is not None:
+            lib().dda_contacts_free(self._h)
+            self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+    def export(self) -> dict:
+        m = self.count
+        o = {k: np.empty(m, np.int32) for k in ("i", "v", "j", "e", "type")}
+        o["t"] = np.empty(m)
+        o["dist2"] = np.empty(m)
+        ptr = lambda a: a.ctypes.data_as(C.c_void_p)
+        _check(lib().dda_contacts_export(self._h, *[ptr(o[k]) for k in ("i", "v", "j", "e", "type", "t", "dist2")]),
+               "dda_contacts_export")
+        return o
+
+    def springs(self, cxy, p_n=40.0, shear_ratio=0.4, stream=None) -> dict:
+        """Springs of the VE contacts as CUDA tensors (bi, bj, pen, e, g) for build_matrix."""
+        torch = _torch()
+        n = self._keep[0].shape[0] - 1
+        m = 2 * self.n_ve
+        dev = self._keep[1].device
+        o = {"bi": torch.empty(m, dtype=torch.int32, device=dev), "bj": torch.empty(m, dtype=torch.int32, device=dev),
+             "pen": torch.empty(m, dtype=torch.float64, device=dev),
+             "e": torch.empty((m, 6), dtype=torch.float64, device=dev),
+             "g": torch.empty((m, 6), dtype=torch.float64, device=dev)}
+        _check(lib().dda_contact_springs(self._h, _dev(cxy, torch.float64, (n, 2), "cxy"), float(p_n),
+                                         float(shear_ratio), *[C.c_void_p(o[k].data_ptr()) for k in
+                                                               ("bi", "bj", "pen", "e", "g")],
+                                         C.c_void_p(_stream(stream))), "dda_contact_springs")
+        return o
+
+
+def detect_contacts(vptr, vxy, d0, stream=None) -> Contacts:
+    """NEXT-3: dda_detect_contacts on CUDA tensors vptr [n+1] int32 and vxy [V, 2] float64."""
+    torch = _torch()
+    n = int(vptr.shape[0]) - 1
+    vp = _dev(vptr, torch.int32, None, "vptr")
+    vx = _dev(vxy, torch.float64, None, "vxy")
+    h = C.c_void_p()
+    _check(lib().dda_detect_contacts(n, vp, vx, float(d0), C.c_void_p(_stream(stream)), C.byref(h)),
+           "dda_detect_contacts")
+    return Contacts(h, vptr, vxy)
