@@ -12,9 +12,15 @@
 //   p = z + beta p
 // Two transports share the driver: NCCL (one partition per process / GPU) and
 // LOOPBACK (all partitions in one process on one GPU; the exchange is a device
-// copy and the "allreduce" a host sum in partition order) — the loopback runs
+// copy and the "allreduce" a device sum in partition order) — the loopback runs
 // the identical partitioned algorithm where only one GPU is available.
-// v1 keeps the CG scalars on the host (two small host reads per iteration).
+// v2: the CG scalars never leave the device.  After each allreduce a one-thread
+// kernel (k_scal_alpha / k_scal_beta) turns the reduced sums into alpha, beta,
+// the stopping test and the loop state (identical on every partition / rank);
+// the vector kernels read them from device memory and return at once when the
+// solve has finished.  The host issues iterations in chunks and reads the
+// state once per chunk (DDA_DIST_CHUNK, default 8) instead of twice per
+// iteration.  The SpMV is the column-pair map (spmv_col.cuh, v5) over own rows.
 #include <nccl.h>
 
 #include <cmath>
@@ -22,6 +28,7 @@
 #include <vector>
 
 #include "precond_dev.cuh"
+#include "spmv_col.cuh"
 
 namespace dda {
 namespace {
@@ -130,11 +137,6 @@ __global__ void __launch_bounds__(DDA_THREADS) k_update_own(int n, const double*
     cta_partial(rz, part, gridDim.x, 1, red);
 }
 
-__global__ void k_pupd_own(int n6, double beta, const double* __restrict__ z, double* p) {
-    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < n6; t += gridDim.x * blockDim.x)
-        p[t] = fma(beta, p[t], z[t]);
-}
-
 __global__ void __launch_bounds__(DDA_THREADS) k_resid_own(int n, const double* __restrict__ F,
                                                            const double* __restrict__ q, double* part) {
     __shared__ double red[WPB];
@@ -167,6 +169,107 @@ __global__ void k_sum_parts(const double* part, int G, int nv, double* out) {
     }
 }
 
+// ---- v2: device-side CG state (one copy per partition; every copy evolves identically)
+struct DState {
+    double rho, alpha, beta, bnorm, tol, rr;
+    int k, maxit, done, status, iters, pad;
+};
+
+struct XLdC {   // x (p and its halo) is written by earlier kernels / NCCL: read-only here
+    const double* __restrict__ x;
+    using Raw = double2;
+    __device__ __forceinline__ Raw raw(int vec, int pair) const {
+        return __ldg(reinterpret_cast<const double2*>(x + 6 * (size_t)vec + 2 * pair));
+    }
+    __device__ __forceinline__ double2 cook(const Raw& r) const { return r; }
+    __device__ __forceinline__ double2 operator()(int vec, int pair) const { return raw(vec, pair); }
+};
+
+// q = K x over own rows, column-pair map; partial of x^T q.  Skipped once the solve is done.
+__global__ void __launch_bounds__(DDA_THREADS, 3) k_spmv_own2(BsrView A, const double* __restrict__ x,
+                                                              double* __restrict__ q, double* part,
+                                                              const DState* st) {
+    __shared__ double red[WPB];
+    if (st && st->done) return;
+    const int lane = threadIdx.x & 31;
+    const XLdC xf{x};
+    double acc = 0.0;
+    for_rows_c<SPMV_FULL, 5>(A, blockIdx.x * WPB + (threadIdx.x >> 5), gridDim.x * WPB, xf, lane,
+                             [&](int i, bool ok, double y0, double y1) {
+                                 if (ok) {
+                                     const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
+                                     *reinterpret_cast<double2*>(q + o) = make_double2(y0, y1);
+                                     const double2 xv = xf(i, ccol_of(lane));
+                                     acc += xv.x * y0 + xv.y * y1;
+                                 }
+                             });
+    cta_partial(acc, part, gridDim.x, 0, red);
+}
+
+// after the sigma allreduce: alpha = rho / sigma (breakdown: done)
+__global__ void k_scal_alpha(DState* st, const double* red) {
+    if (st->done) return;
+    const double sigma = red[0];
+    if (!(sigma > 0.0) || !isfinite(sigma)) { st->status = DDA_ERR_BREAKDOWN; st->done = 1; return; }
+    st->alpha = st->rho / sigma;
+}
+
+__global__ void __launch_bounds__(DDA_THREADS) k_update_own2(int n, const double* __restrict__ dinv, int use_bj,
+                                                             const DState* stt, const double* __restrict__ p,
+                                                             const double* __restrict__ q, double* d, double* r,
+                                                             double* z, double* part) {
+    __shared__ double red[WPB];
+    if (stt->done) return;
+    const double alpha = stt->alpha;
+    const int lane = threadIdx.x & 31, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    double rr = 0, rz = 0;
+    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        double rv = 0.0;
+        if (R.valid) {
+            d[R.idx] = d[R.idx] + alpha * p[R.idx];
+            rv = r[R.idx] - alpha * q[R.idx];
+            r[R.idx] = rv;
+        }
+        rr += rv * rv;
+        const double zz = use_bj ? bj_lane(dinv, R, rv) : rv;
+        if (R.valid) z[R.idx] = zz;
+        rz += rv * zz;
+    }
+    cta_partial(rr, part, gridDim.x, 0, red);
+    cta_partial(rz, part, gridDim.x, 1, red);
+}
+
+// after the (rr, rz) allreduce: stopping test (reading Z1), breakdown, beta, iteration cap
+__global__ void k_scal_beta(DState* st, const double* red) {
+    if (st->done) return;
+    const double rr = red[0], rz = red[1];
+    st->rr = rr;
+    st->iters = st->k + 1;
+    st->k = st->k + 1;
+    if (sqrt(rr) <= st->tol * st->bnorm) { st->status = DDA_OK; st->done = 1; return; }
+    if (!(rz > 0.0) || !isfinite(rz)) { st->status = DDA_ERR_BREAKDOWN; st->done = 1; return; }
+    st->beta = rz / st->rho;
+    st->rho = rz;
+    if (st->k >= st->maxit) { st->status = DDA_ERR_NO_CONVERGENCE; st->done = 1; }
+}
+
+__global__ void k_pupd_own2(int n6, const DState* st, const double* __restrict__ z, double* p) {
+    if (st->done) return;
+    const double beta = st->beta;
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < n6; t += gridDim.x * blockDim.x)
+        p[t] = fma(beta, p[t], z[t]);
+}
+
+// loopback "allreduce": red[0..nv) = sum over partitions, in partition order, of scal[p][0..nv)
+__global__ void k_sum_loopback(const double* const* scal, int P, int nv, double* red) {
+    const int k = threadIdx.x;
+    if (k >= nv) return;
+    double s = 0.0;
+    for (int p = 0; p < P; ++p) s += scal[p][k];
+    red[k] = s;
+}
+
 int grid_of(const void* k, int cap_per_sm) {
     int per = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k, DDA_THREADS, 0);
@@ -192,7 +295,10 @@ struct DistPart {
     double* sendbuf = nullptr;   // device [6 n_send]
     double* x = nullptr;         // device [6 n_local]: p (own) + halo
     double *q = nullptr, *r = nullptr, *z = nullptr, *part = nullptr, *scal = nullptr;
-    int G_spmv = 0, G_vec = 0;
+    double* red = nullptr;       // device: allreduced scalars (v2)
+    void* dst = nullptr;         // device DState (v2)
+    const double** scal_ptrs = nullptr;   // device [P] (loopback: every partition's scal)
+    int G_spmv = 0, G_vec = 0, G_spmv2 = 0;
 };
 
 struct dda_comm {
@@ -249,7 +355,8 @@ extern "C" void dda_comm_free(dda_comm_t c) {
     if (!c) return;
     cudaDeviceSynchronize();
     for (DistPart& p : c->parts) {
-        void* ptrs[] = {p.send_idx, p.sendbuf, p.x, p.q, p.r, p.z, p.part, p.scal};
+        void* ptrs[] = {p.send_idx, p.sendbuf, p.x, p.q, p.r, p.z, p.part, p.scal, p.red, p.dst,
+                        (void*)p.scal_ptrs};
         for (void* v : ptrs)
             if (v) dev_free(v);
     }
@@ -268,7 +375,8 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     DistPart& D = c->parts[slot];
     if (D.K) {                                   // re-attach (e.g. a rebuilt matrix): release the old buffers
         cudaStreamSynchronize(st);
-        void* ptrs[] = {D.send_idx, D.sendbuf, D.x, D.q, D.r, D.z, D.part, D.scal};
+        void* ptrs[] = {D.send_idx, D.sendbuf, D.x, D.q, D.r, D.z, D.part, D.scal, D.red, D.dst,
+                        (void*)D.scal_ptrs};
         for (void* v : ptrs)
             if (v) dev_free(v);
         D = DistPart();
@@ -290,7 +398,13 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     const size_t nl6 = 6 * (size_t)K->n, no6 = 6 * (size_t)n_own;
     D.G_spmv = grid_of((const void*)k_spmv_own, 6);
     D.G_vec = grid_of((const void*)k_update_own, 8);
-    const int Gm = D.G_spmv > D.G_vec ? D.G_spmv : D.G_vec;
+    D.G_spmv2 = grid_of((const void*)k_spmv_own2, 3);
+    {   // no more CTAs than ten-row groups of own rows
+        const int need = (n_own + 10 * WPB - 1) / (10 * WPB);
+        if (D.G_spmv2 > need) D.G_spmv2 = need > 0 ? need : 1;
+    }
+    int Gm = D.G_spmv > D.G_vec ? D.G_spmv : D.G_vec;
+    if (D.G_spmv2 > Gm) Gm = D.G_spmv2;
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.send_idx), (D.n_send + 1) * sizeof(int), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.sendbuf), (6 * (size_t)D.n_send + 1) * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.x), nl6 * sizeof(double), st));
@@ -299,6 +413,9 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.z), no6 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.part), 3 * (size_t)Gm * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.scal), 8 * sizeof(double), st));
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.red), 8 * sizeof(double), st));
+    DDA_CK(dev_alloc(&D.dst, sizeof(DState), st));
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.scal_ptrs), (P + 1) * sizeof(double*), st));
     if (D.n_send)
         DDA_CK(cudaMemcpyAsync(D.send_idx, send_idx, D.n_send * sizeof(int), cudaMemcpyHostToDevice, st));
     DDA_CK(cudaMemsetAsync(D.x, 0, nl6 * sizeof(double), st));
@@ -362,6 +479,21 @@ dda_status_t allreduce_host(dda_comm* c, int nv, double* out, cudaStream_t st) {
     if (c->nranks > 1) DDA_NCCL(ncclAllReduce(D.scal, D.scal, nv, ncclDouble, ncclSum, c->nccl, st));
     DDA_CK(cudaMemcpyAsync(out, D.scal, nv * sizeof(double), cudaMemcpyDeviceToHost, st));
     DDA_CK(cudaStreamSynchronize(st));
+    return DDA_OK;
+}
+
+// v2: D.red[0..nv) = the sum over all partitions / ranks of D.scal[0..nv), on the device
+dda_status_t allreduce_dev(dda_comm* c, int nv, cudaStream_t st) {
+    if (c->loopback) {
+        for (DistPart& D : c->parts) {
+            k_sum_loopback<<<1, 32, 0, st>>>(D.scal_ptrs, (int)c->parts.size(), nv, D.red);
+            DDA_LAUNCHED();
+        }
+        return DDA_OK;
+    }
+    DistPart& D = c->parts[0];
+    if (c->nranks > 1) DDA_NCCL(ncclAllReduce(D.scal, D.red, nv, ncclDouble, ncclSum, c->nccl, st));
+    else DDA_CK(cudaMemcpyAsync(D.red, D.scal, nv * sizeof(double), cudaMemcpyDeviceToDevice, st));
     return DDA_OK;
 }
 
@@ -459,35 +591,58 @@ extern "C" dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double* const* F,
         status = DDA_OK;
     } else if (!(rho > 0.0) || !std::isfinite(rho)) {
         status = DDA_ERR_BREAKDOWN;
-    } else {
-        for (int k = 0; k < maxit; ++k) {
-            DDA_TRY(halo_exchange(c, st));                        // p halo
-            DDA_TRY(spmv_parts(c, true, st));                     // q = K p, p^T q
-            double sigma;
-            DDA_TRY(allreduce_host(c, 1, &sigma, st));
-            if (!(sigma > 0.0) || !std::isfinite(sigma)) { status = DDA_ERR_BREAKDOWN; break; }
-            const double alpha = rho / sigma;
-            for (DistPart& D : c->parts) {
-                k_update_own<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, D.K->dinv, use_bj, alpha, D.x, D.q,
-                                                              d[&D - &c->parts[0]], D.r, D.z, D.part);
-                DDA_LAUNCHED();
-                k_sum_parts<<<1, DDA_THREADS, 0, st>>>(D.part, D.G_vec, 2, D.scal);
-                DDA_LAUNCHED();
-            }
-            double s2[2];
-            DDA_TRY(allreduce_host(c, 2, s2, st));
-            rr = s2[0];
-            const double rz = s2[1];
-            it = k + 1;
-            if (std::sqrt(rr) <= tol * bnorm) { status = DDA_OK; break; }
-            if (!(rz > 0.0) || !std::isfinite(rz)) { status = DDA_ERR_BREAKDOWN; break; }
-            const double beta = rz / rho;
-            rho = rz;
-            for (DistPart& D : c->parts) {
-                k_pupd_own<<<2 * device_sms(), 256, 0, st>>>(6 * D.n_own, beta, D.z, D.x);
-                DDA_LAUNCHED();
-            }
+    } else if (maxit > 0) {
+        // v2: device-side scalars; the host reads the state once per chunk of iterations
+        DState h{};
+        h.rho = rho; h.bnorm = bnorm; h.tol = tol; h.rr = rr; h.maxit = maxit;
+        h.status = DDA_ERR_NO_CONVERGENCE;
+        std::vector<const double*> sp;
+        for (DistPart& D : c->parts) sp.push_back(D.scal);
+        for (DistPart& D : c->parts) {
+            DDA_CK(cudaMemcpyAsync(D.dst, &h, sizeof h, cudaMemcpyHostToDevice, st));
+            if (c->loopback)
+                DDA_CK(cudaMemcpyAsync(D.scal_ptrs, sp.data(), sp.size() * sizeof(double*), cudaMemcpyHostToDevice,
+                                       st));
         }
+        int chunk = 8;
+        if (const char* e = getenv("DDA_DIST_CHUNK")) chunk = atoi(e) > 0 ? atoi(e) : 8;
+        DState out{};
+        for (int k = 0; k < maxit; k += chunk) {
+            for (int ci = 0; ci < chunk && k + ci < maxit; ++ci) {
+                DDA_TRY(halo_exchange(c, st));                    // p halo
+                for (DistPart& D : c->parts) {                    // q = K p, p^T q
+                    k_spmv_own2<<<D.G_spmv2, DDA_THREADS, 0, st>>>(own_view(D), D.x, D.q, D.part,
+                                                                  reinterpret_cast<DState*>(D.dst));
+                    DDA_LAUNCHED();
+                    k_sum_parts<<<1, DDA_THREADS, 0, st>>>(D.part, D.G_spmv2, 1, D.scal);
+                    DDA_LAUNCHED();
+                }
+                DDA_TRY(allreduce_dev(c, 1, st));
+                for (DistPart& D : c->parts) {
+                    k_scal_alpha<<<1, 1, 0, st>>>(reinterpret_cast<DState*>(D.dst), D.red);
+                    DDA_LAUNCHED();
+                    k_update_own2<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, D.K->dinv, use_bj,
+                                                                   reinterpret_cast<DState*>(D.dst), D.x, D.q,
+                                                                   d[&D - &c->parts[0]], D.r, D.z, D.part);
+                    DDA_LAUNCHED();
+                    k_sum_parts<<<1, DDA_THREADS, 0, st>>>(D.part, D.G_vec, 2, D.scal);
+                    DDA_LAUNCHED();
+                }
+                DDA_TRY(allreduce_dev(c, 2, st));
+                for (DistPart& D : c->parts) {
+                    k_scal_beta<<<1, 1, 0, st>>>(reinterpret_cast<DState*>(D.dst), D.red);
+                    DDA_LAUNCHED();
+                    k_pupd_own2<<<2 * device_sms(), 256, 0, st>>>(6 * D.n_own, reinterpret_cast<DState*>(D.dst),
+                                                                  D.z, D.x);
+                    DDA_LAUNCHED();
+                }
+            }
+            DDA_CK(cudaMemcpyAsync(&out, c->parts[0].dst, sizeof out, cudaMemcpyDeviceToHost, st));
+            DDA_CK(cudaStreamSynchronize(st));
+            if (out.done) break;
+        }
+        status = (dda_status_t)out.status;
+        it = out.iters;
     }
     // ---- true residual
     for (size_t p = 0; p < c->parts.size(); ++p) {

@@ -84,6 +84,9 @@ def test_pcg_dist_warm_and_zero(dda, prob):
     assert st2 == dda.OK and it2 <= 1
     zs, itz, rrz, stz = comm.pcg_solve([torch.zeros_like(F) for F in Fs])
     assert stz == dda.OK and itz == 0 and all(not z.any() for z in zs)
+    # iteration cap not a multiple of the host-check chunk (device-side loop state, v2)
+    _, it5, rr5, st5 = comm.pcg_solve(Fs, maxit=13)
+    assert st5 == dda.ERR_NO_CONVERGENCE and it5 == 13 and rr5 > 1e-10
 
 
 def test_pcg_dist_nccl_single_rank(dda, prob):
