@@ -101,3 +101,21 @@ def test_fullsize_pcg(dda, full, engine):
     dm, itm, _, _ = O.pcg(P.F, tol=1e-300, maxit=12, precond="bj")
     assert itm == 12
     assert np.linalg.norm(d12.cpu().numpy() - dm) <= 1e-9 * np.linalg.norm(dm)
+
+
+def test_fullsize_ssor_ai(dda, full):
+    """The scaled SSOR-AI persistent kernel (A7) at the 1M-block bench size: converges to 1e-10 (true
+    residual computed by the oracle) in fewer iterations than BJ, and matches the oracle's SSOR-AI
+    PCG after 8 iterations (reading Z17)."""
+    P, O, t, K = full
+    d, it, rr, st = K.pcg_solve(t["F"], tol=1e-10, precond="ssor_ai")
+    assert st == dda.OK and rr <= 1.01e-10
+    assert K.pcg_engine("ssor_ai") == "scaled"
+    res = P.F - O.spmv_rows(np.arange(6 * P.n, dtype=np.int64), d.cpu().numpy())
+    assert np.linalg.norm(res) / np.linalg.norm(P.F) <= 1.05e-10
+    assert 100 <= it <= 200
+    d8, it8, _, st8 = K.pcg_solve(t["F"], tol=1e-300, maxit=8, precond="ssor_ai")
+    assert st8 == dda.ERR_NO_CONVERGENCE and it8 == 8
+    dm, itm, _, _ = O.pcg(P.F, tol=1e-300, maxit=8, precond="ssor_ai")
+    assert itm == 8
+    assert np.linalg.norm(d8.cpu().numpy() - dm) <= 1e-9 * np.linalg.norm(dm)
