@@ -150,6 +150,7 @@ dda_status_t ensure_workspace(dda_matrix* K, size_t bytes, cudaStream_t st);
 dda_status_t bj_setup(dda_matrix* K, cudaStream_t s, int32_t* bad_block);
 dda_status_t spmv(dda_matrix* K, const double* x, double* y, cudaStream_t s);
 void pcg_graph_free(void* g);
+dda_status_t scaled_setup(dda_matrix* K, cudaStream_t st);   // S_i V_ij S_j^T (needs lfac / sfac of every row)
 dda_status_t ilu_setup(dda_matrix* K, cudaStream_t st, int32_t* bad_block);
 dda_status_t ilu_apply(dda_matrix* K, const double* r, double* z, double* y, double* yh, cudaStream_t st);
 int ilu_grid();

@@ -55,10 +55,6 @@ __device__ __forceinline__ void cta_partial(double v, double* part, int slot_str
     __syncthreads();
 }
 
-__global__ void k_pack(int n_send, const int* __restrict__ idx, const double* __restrict__ x, double* __restrict__ buf) {
-    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < 6 * n_send; t += gridDim.x * blockDim.x)
-        buf[t] = x[6 * (size_t)idx[t / 6] + t % 6];
-}
 
 // q = K x over own rows (A.n = n_own); optional partial of x^T q
 __global__ void __launch_bounds__(DDA_THREADS, 6) k_spmv_own(BsrView A, const double* __restrict__ x,
@@ -270,6 +266,213 @@ __global__ void k_sum_loopback(const double* const* scal, int P, int nv, double*
     red[k] = s;
 }
 
+// ---- v3: the scaled block-Jacobi engine per partition (PCG on S K S^T, reading Z25)
+//
+// Each partition runs the single-GPU scaled iteration on its own rows: phase A forms p = r~ + beta
+// p_old for own and gathered rows (halo rows of r~ and p_old come from the exchange), q = Ks p, and
+// applies the deferred x += alpha p_old; phase B updates r~ and sums rho' and the w-bound of the
+// stopping test; the exact test |L r~| runs only when that bound allows it.  The block scaling needs
+// S_j of the halo rows (their diagonal blocks are complete only on the owner): exchanged once per solve.
+struct SState {
+    double rho, alpha, beta, bnorm, tol, rr, rho_new;
+    int k, maxit, done, status, iters, maybe, pend, checks;
+};
+
+__global__ void k_pack_w(int n_send, int w, const int* __restrict__ idx, const double* __restrict__ x,
+                         double* __restrict__ buf) {
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < w * n_send; t += gridDim.x * blockDim.x)
+        buf[t] = x[(size_t)w * idx[t / w] + t % w];
+}
+
+// row a of the packed lower-triangular M (TR = false: M[a][c], c <= a) or of its transpose (TR: M[c][a],
+// c >= a) applied to the 6-vector spread over the row's lanes; every lane of the warp must call
+__device__ __forceinline__ double tri_apply(const double* __restrict__ M, const Row5& R, double v, bool tr) {
+    const double* blk = M + (size_t)kDinv * (R.valid ? R.i : 0);
+    double z = 0.0;
+#pragma unroll
+    for (int c = 0; c < 6; ++c) {
+        const bool nz = tr ? (c >= R.a) : (c <= R.a);
+        const double m = nz ? __ldg(blk + (tr ? lo_off(c, R.a) : lo_off(R.a, c))) : 0.0;
+        z = fma(m, __shfl_sync(0xffffffffu, v, R.base + c), z);
+    }
+    return z;
+}
+
+// r = F - q (or F); r~ = S r -> rt, p0; x = L^T d0 (or 0) -> d; partials FF, |r|^2, |r~|^2
+__global__ void __launch_bounds__(DDA_THREADS) k_v3_init(int n, const double* __restrict__ F,
+                                                         const double* __restrict__ q, const double* d0, double* d,
+                                                         const double* __restrict__ sfac,
+                                                         const double* __restrict__ lfac, double* rt, double* p0,
+                                                         double* part) {
+    __shared__ double red[WPB];
+    const int lane = threadIdx.x & 31, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    double FF = 0, rr = 0, rz = 0;
+    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        double fv = 0.0, rv = 0.0, dv = 0.0;
+        if (R.valid) {
+            fv = F[R.idx];
+            rv = q ? fv - q[R.idx] : fv;
+            if (d0) dv = d0[R.idx];
+        }
+        FF += fv * fv;
+        rr += rv * rv;
+        const double t0 = tri_apply(sfac, R, rv, false);
+        const double t = R.valid ? t0 : 0.0;
+        const double x0 = tri_apply(lfac, R, dv, true);
+        if (R.valid) {
+            rt[R.idx] = t;
+            p0[R.idx] = t;
+            d[R.idx] = d0 ? x0 : 0.0;
+        }
+        rz += t * t;
+    }
+    cta_partial(FF, part, gridDim.x, 0, red);
+    cta_partial(rr, part, gridDim.x, 1, red);
+    cta_partial(rz, part, gridDim.x, 2, red);
+}
+
+struct XFusedLdg {   // x = r~ + beta p_old (k = 0: p_old = r~, beta = 0)
+    const double* __restrict__ z;
+    const double* __restrict__ p;
+    double beta;
+    using Raw = double2;
+    __device__ __forceinline__ Raw raw(int vec, int pair) const {
+        const size_t o = 6 * (size_t)vec + 2 * pair;
+        const double2 zz = __ldg(reinterpret_cast<const double2*>(z + o));
+        const double2 pp = __ldg(reinterpret_cast<const double2*>(p + o));
+        return make_double2(fma(beta, pp.x, zz.x), fma(beta, pp.y, zz.y));
+    }
+    __device__ __forceinline__ double2 cook(const Raw& r) const { return r; }
+    __device__ __forceinline__ double2 operator()(int vec, int pair) const { return raw(vec, pair); }
+};
+
+// phase A over own rows (A.upper = the scaled blocks)
+// p_k lives in buffer (k & 1) ? PB : PA; p_old of iteration k >= 1 is p_{k-1}
+__global__ void __launch_bounds__(DDA_THREADS, 3) k_v3_a(BsrView A, const double* rt, double* PA, double* PB,
+                                                         double* q, double* x, const SState* st, double* part) {
+    __shared__ double red[WPB];
+    if (st->done) return;
+    const int k = st->k;
+    const double* pold = k == 0 ? rt : ((k & 1) ? PA : PB);
+    double* pnew = (k & 1) ? PB : PA;
+    const double beta = k == 0 ? 0.0 : st->beta;
+    const double ap = st->pend ? st->alpha : 0.0;
+    const int lane = threadIdx.x & 31;
+    const XFusedLdg xf{rt, pold, beta};
+    double acc = 0.0;
+    for_rows_c<SPMV_OFFDIAG, 5>(A, blockIdx.x * WPB + (threadIdx.x >> 5), gridDim.x * WPB, xf, lane,
+                                [&](int i, bool ok, double y0, double y1) {
+                                    if (ok) {
+                                        const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
+                                        const double2 pv = xf(i, ccol_of(lane));
+                                        y0 += pv.x;
+                                        y1 += pv.y;
+                                        if (ap != 0.0) {
+                                            const double2 po = __ldg(reinterpret_cast<const double2*>(pold + o));
+                                            const double2 xo = *reinterpret_cast<const double2*>(x + o);
+                                            *reinterpret_cast<double2*>(x + o) =
+                                                make_double2(xo.x + ap * po.x, xo.y + ap * po.y);
+                                        }
+                                        *reinterpret_cast<double2*>(q + o) = make_double2(y0, y1);
+                                        *reinterpret_cast<double2*>(pnew + o) = pv;
+                                        acc += pv.x * y0 + pv.y * y1;
+                                    }
+                                });
+    cta_partial(acc, part, gridDim.x, 0, red);
+}
+
+__global__ void k_v3_alpha(SState* st, const double* red) {
+    if (st->done) return;
+    st->pend = 0;                                           // phase A applied the deferred x update
+    const double sigma = red[0];
+    if (!(sigma > 0.0) || !isfinite(sigma)) { st->status = DDA_ERR_BREAKDOWN; st->done = 1; return; }
+    st->alpha = st->rho / sigma;
+}
+
+// phase B: r~ -= alpha q; partials |r~|^2 and sum_i w_i |r~_i|^2
+__global__ void __launch_bounds__(DDA_THREADS) k_v3_b(int n, double* rt, const double* __restrict__ q,
+                                                      const double* __restrict__ w, const SState* st, double* part) {
+    __shared__ double red[WPB];
+    if (st->done) return;
+    const double alpha = st->alpha;
+    const int lane = threadIdx.x & 31, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    double rz = 0.0, lb = 0.0;
+    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        if (R.valid) {
+            const double rv = rt[R.idx] - alpha * q[R.idx];
+            rt[R.idx] = rv;
+            rz += rv * rv;
+            lb += __ldg(w + R.i) * (rv * rv);
+        }
+    }
+    cta_partial(rz, part, gridDim.x, 0, red);
+    cta_partial(lb, part, gridDim.x, 1, red);
+}
+
+__global__ void k_v3_rho(SState* st, const double* red) {
+    if (st->done) return;
+    const double rho1 = red[0];
+    const double thr = st->tol * st->bnorm;
+    st->pend = 1;                                           // x += alpha p_k: next phase A or k_v3_final
+    st->iters = st->k + 1;
+    st->rho_new = rho1;
+    st->maybe = 0;
+    if (rho1 == 0.0) { st->rr = 0.0; st->status = DDA_OK; st->k = st->k + 1; st->done = 1; return; }
+    st->maybe = (isfinite(rho1) && !(0.999 * red[1] > thr * thr)) ? 1 : 0;
+}
+
+// the exact stopping test share |L r~|^2 (only when k_v3_rho flagged it)
+__global__ void __launch_bounds__(DDA_THREADS) k_v3_c(int n, const double* __restrict__ rt,
+                                                      const double* __restrict__ lfac, const SState* st,
+                                                      double* part) {
+    __shared__ double red[WPB];
+    const bool on = !st->done && st->maybe;
+    const int lane = threadIdx.x & 31, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    double rl = 0.0;
+    if (on) {
+        for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+            const Row5 R = row5(grp, lane, n);
+            const double rv = R.valid ? rt[R.idx] : 0.0;
+            const double o0 = tri_apply(lfac, R, rv, false);
+            const double o = R.valid ? o0 : 0.0;
+            rl += o * o;
+        }
+    }
+    cta_partial(rl, part, gridDim.x, 0, red);
+}
+
+__global__ void k_v3_check(SState* st, const double* red) {
+    if (st->done) return;
+    if (st->maybe) {
+        st->checks = st->checks + 1;
+        st->rr = red[0];
+        if (sqrt(red[0]) <= st->tol * st->bnorm) { st->status = DDA_OK; st->k = st->k + 1; st->done = 1; return; }
+    }
+    const double rho1 = st->rho_new;
+    st->k = st->k + 1;
+    if (!(rho1 > 0.0) || !isfinite(rho1)) { st->status = DDA_ERR_BREAKDOWN; st->done = 1; return; }
+    st->beta = rho1 / st->rho;
+    st->rho = rho1;
+    if (st->k >= st->maxit) { st->status = DDA_ERR_NO_CONVERGENCE; st->done = 1; }
+}
+
+// the pending x += alpha p of the last iteration, then d = S^T x (own rows)
+__global__ void __launch_bounds__(DDA_THREADS) k_v3_final(int n, double* d, const double* pA, const double* pB,
+                                                          const double* __restrict__ sfac, const SState* st) {
+    const int lane = threadIdx.x & 31, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    const bool pend = st->pend;
+    const double alpha = st->alpha;
+    const double* pk = ((st->k - 1) & 1) ? pB : pA;        // p of the last phase A (iteration k - 1)
+    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        const double xv = R.valid ? (pend ? d[R.idx] + alpha * pk[R.idx] : d[R.idx]) : 0.0;
+        const double dv = tri_apply(sfac, R, xv, true);
+        if (R.valid) d[R.idx] = dv;
+    }
+}
+
 int grid_of(const void* k, int cap_per_sm) {
     int per = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k, DDA_THREADS, 0);
@@ -298,7 +501,8 @@ struct DistPart {
     double* red = nullptr;       // device: allreduced scalars (v2)
     void* dst = nullptr;         // device DState (v2)
     const double** scal_ptrs = nullptr;   // device [P] (loopback: every partition's scal)
-    int G_spmv = 0, G_vec = 0, G_spmv2 = 0;
+    double *rt = nullptr, *pA = nullptr, *pB = nullptr;   // v3: r~, p ping-pong over local rows (own + halo)
+    int G_spmv = 0, G_vec = 0, G_spmv2 = 0, G_a3 = 0;
 };
 
 struct dda_comm {
@@ -356,7 +560,7 @@ extern "C" void dda_comm_free(dda_comm_t c) {
     cudaDeviceSynchronize();
     for (DistPart& p : c->parts) {
         void* ptrs[] = {p.send_idx, p.sendbuf, p.x, p.q, p.r, p.z, p.part, p.scal, p.red, p.dst,
-                        (void*)p.scal_ptrs};
+                        (void*)p.scal_ptrs, p.rt, p.pA, p.pB};
         for (void* v : ptrs)
             if (v) dev_free(v);
     }
@@ -376,7 +580,7 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     if (D.K) {                                   // re-attach (e.g. a rebuilt matrix): release the old buffers
         cudaStreamSynchronize(st);
         void* ptrs[] = {D.send_idx, D.sendbuf, D.x, D.q, D.r, D.z, D.part, D.scal, D.red, D.dst,
-                        (void*)D.scal_ptrs};
+                        (void*)D.scal_ptrs, D.rt, D.pA, D.pB};
         for (void* v : ptrs)
             if (v) dev_free(v);
         D = DistPart();
@@ -403,10 +607,16 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
         const int need = (n_own + 10 * WPB - 1) / (10 * WPB);
         if (D.G_spmv2 > need) D.G_spmv2 = need > 0 ? need : 1;
     }
+    D.G_a3 = grid_of((const void*)k_v3_a, 3);
+    {
+        const int need = (n_own + 10 * WPB - 1) / (10 * WPB);
+        if (D.G_a3 > need) D.G_a3 = need > 0 ? need : 1;
+    }
     int Gm = D.G_spmv > D.G_vec ? D.G_spmv : D.G_vec;
     if (D.G_spmv2 > Gm) Gm = D.G_spmv2;
+    if (D.G_a3 > Gm) Gm = D.G_a3;
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.send_idx), (D.n_send + 1) * sizeof(int), st));
-    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.sendbuf), (6 * (size_t)D.n_send + 1) * sizeof(double), st));
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.sendbuf), (24 * (size_t)D.n_send + 1) * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.x), nl6 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.q), no6 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.r), no6 * sizeof(double), st));
@@ -414,7 +624,13 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.part), 3 * (size_t)Gm * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.scal), 8 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.red), 8 * sizeof(double), st));
-    DDA_CK(dev_alloc(&D.dst, sizeof(DState), st));
+    DDA_CK(dev_alloc(&D.dst, sizeof(DState) > sizeof(SState) ? sizeof(DState) : sizeof(SState), st));
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.rt), nl6 * sizeof(double), st));
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.pA), nl6 * sizeof(double), st));
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.pB), nl6 * sizeof(double), st));
+    DDA_CK(cudaMemsetAsync(D.rt, 0, nl6 * sizeof(double), st));
+    DDA_CK(cudaMemsetAsync(D.pA, 0, nl6 * sizeof(double), st));
+    DDA_CK(cudaMemsetAsync(D.pB, 0, nl6 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.scal_ptrs), (P + 1) * sizeof(double*), st));
     if (D.n_send)
         DDA_CK(cudaMemcpyAsync(D.send_idx, send_idx, D.n_send * sizeof(int), cudaMemcpyHostToDevice, st));
@@ -425,13 +641,24 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
 
 namespace {
 
-// fill x[n_own:] of every local partition from the peers' own rows
-dda_status_t halo_exchange(dda_comm* c, cudaStream_t st) {
+double* part_buf(DistPart& D, int which) {
+    switch (which) {
+        case 1: return D.rt;
+        case 2: return D.pA;
+        case 3: return D.pB;
+        case 4: return D.K->sfac;
+        default: return D.x;
+    }
+}
+
+// fill rows n_own.. of buffer `which` (w doubles per row) of every local partition from the peers' own rows
+dda_status_t halo_exchange_w(dda_comm* c, cudaStream_t st, int which, int w) {
     const int P = c->nranks;
     for (DistPart& D : c->parts) {
         if (D.n_send) {
-            k_pack<<<(6 * D.n_send + 255) / 256 < 1024 ? (6 * D.n_send + 255) / 256 : 1024, 256, 0, st>>>(
-                D.n_send, D.send_idx, D.x, D.sendbuf);
+            const int items = w * D.n_send;
+            k_pack_w<<<(items + 255) / 256 < 1024 ? (items + 255) / 256 : 1024, 256, 0, st>>>(
+                D.n_send, w, D.send_idx, part_buf(D, which), D.sendbuf);
             DDA_LAUNCHED();
         }
     }
@@ -443,25 +670,30 @@ dda_status_t halo_exchange(dda_comm* c, cudaStream_t st) {
                 DistPart& R = c->parts[q];
                 if (S.send_counts[q] != R.recv_counts[p]) return DDA_ERR_ARG;
                 if (!S.send_counts[q]) continue;
-                DDA_CK(cudaMemcpyAsync(R.x + 6 * ((size_t)R.n_own + R.recv_off[p]), S.sendbuf + 6 * (size_t)S.send_off[q],
-                                       6 * sizeof(double) * S.send_counts[q], cudaMemcpyDeviceToDevice, st));
+                DDA_CK(cudaMemcpyAsync(part_buf(R, which) + (size_t)w * ((size_t)R.n_own + R.recv_off[p]),
+                                       S.sendbuf + (size_t)w * S.send_off[q], (size_t)w * sizeof(double) * S.send_counts[q],
+                                       cudaMemcpyDeviceToDevice, st));
             }
         return DDA_OK;
     }
     DistPart& D = c->parts[0];
+    double* dst = part_buf(D, which);
     DDA_NCCL(ncclGroupStart());
     for (int q = 0; q < P; ++q) {
         if (q == c->rank) continue;
         if (D.send_counts[q])
-            DDA_NCCL(ncclSend(D.sendbuf + 6 * (size_t)D.send_off[q], 6 * (size_t)D.send_counts[q], ncclDouble, q,
+            DDA_NCCL(ncclSend(D.sendbuf + (size_t)w * D.send_off[q], (size_t)w * D.send_counts[q], ncclDouble, q,
                               c->nccl, st));
         if (D.recv_counts[q])
-            DDA_NCCL(ncclRecv(D.x + 6 * ((size_t)D.n_own + D.recv_off[q]), 6 * (size_t)D.recv_counts[q], ncclDouble, q,
-                              c->nccl, st));
+            DDA_NCCL(ncclRecv(dst + (size_t)w * ((size_t)D.n_own + D.recv_off[q]), (size_t)w * D.recv_counts[q],
+                              ncclDouble, q, c->nccl, st));
     }
     DDA_NCCL(ncclGroupEnd());
     return DDA_OK;
 }
+
+// fill x[n_own:] of every local partition from the peers' own rows
+dda_status_t halo_exchange(dda_comm* c, cudaStream_t st) { return halo_exchange_w(c, st, 0, 6); }
 
 // sum of the nv scalars D.scal[0..nv) over all partitions / ranks, to the host
 dda_status_t allreduce_host(dda_comm* c, int nv, double* out, cudaStream_t st) {
@@ -541,6 +773,131 @@ extern "C" dda_status_t dda_spmv_dist(dda_comm_t c, const double* const* x_own, 
     return DDA_OK;
 }
 
+namespace {
+
+BsrView own_view_sc(const DistPart& D) {
+    BsrView A = view_of(D.K);
+    A.n = D.n_own;
+    A.upper = D.K->sc_upper;
+    return A;
+}
+
+// v3 solve (BJ, scaled engine per partition): fills d, *status, *it; *zero = F was 0 (d = 0 set)
+dda_status_t dist_scaled_solve(dda_comm* c, const double* const* F, const double* const* d0, double* const* d,
+                               double tol, int32_t maxit, dda_status_t* status, int* it, bool* zero,
+                               double* bnorm_out, cudaStream_t st) {
+    *zero = false;
+    *it = 0;
+    // S_j of the halo rows from their owners, then the scaled blocks S_i V_ij S_j^T of every local block
+    DDA_TRY(halo_exchange_w(c, st, 4, kDinv));
+    for (DistPart& D : c->parts) {
+        D.K->scaled_valid = false;
+        DDA_TRY(scaled_setup(D.K, st));
+    }
+    const bool have_d0 = d0 != nullptr;
+    if (have_d0) {                                          // q = K d0 over own rows (unscaled)
+        for (size_t p = 0; p < c->parts.size(); ++p) {
+            DistPart& D = c->parts[p];
+            if (d0[p]) DDA_CK(cudaMemcpyAsync(D.x, d0[p], 6 * sizeof(double) * D.n_own, cudaMemcpyDeviceToDevice, st));
+            else DDA_CK(cudaMemsetAsync(D.x, 0, 6 * sizeof(double) * D.n_own, st));
+        }
+        DDA_TRY(halo_exchange(c, st));
+        DDA_TRY(spmv_parts(c, false, st));
+    }
+    for (size_t p = 0; p < c->parts.size(); ++p) {
+        DistPart& D = c->parts[p];
+        k_v3_init<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, F[p], have_d0 ? D.q : nullptr, have_d0 ? d0[p] : nullptr,
+                                                   d[p], D.K->sfac, D.K->lfac, D.rt, D.pA, D.part);
+        DDA_LAUNCHED();
+        k_sum_parts<<<1, DDA_THREADS, 0, st>>>(D.part, D.G_vec, 3, D.scal);
+        DDA_LAUNCHED();
+    }
+    double s3[3];
+    DDA_TRY(allreduce_host(c, 3, s3, st));
+    const double FF = s3[0], bnorm = std::sqrt(FF), rr = s3[1], rho = s3[2];
+    *bnorm_out = bnorm;
+    if (FF == 0.0) {                                        // reading Z2
+        for (size_t p = 0; p < c->parts.size(); ++p)
+            DDA_CK(cudaMemsetAsync(d[p], 0, 6 * sizeof(double) * c->parts[p].n_own, st));
+        DDA_CK(cudaStreamSynchronize(st));
+        *zero = true;
+        *status = DDA_OK;
+        return DDA_OK;
+    }
+    SState h{};
+    h.rho = rho; h.bnorm = bnorm; h.tol = tol; h.rr = rr; h.maxit = maxit;
+    h.status = DDA_ERR_NO_CONVERGENCE;
+    if (std::sqrt(rr) <= tol * bnorm) { h.status = DDA_OK; h.done = 1; }
+    else if (!(rho > 0.0) || !std::isfinite(rho)) { h.status = DDA_ERR_BREAKDOWN; h.done = 1; }
+    else if (maxit <= 0) { h.done = 1; }
+    std::vector<const double*> sp;
+    for (DistPart& D : c->parts) sp.push_back(D.scal);
+    for (DistPart& D : c->parts) {
+        DDA_CK(cudaMemcpyAsync(D.dst, &h, sizeof h, cudaMemcpyHostToDevice, st));
+        if (c->loopback)
+            DDA_CK(cudaMemcpyAsync(D.scal_ptrs, sp.data(), sp.size() * sizeof(double*), cudaMemcpyHostToDevice, st));
+    }
+    int chunk = 8;
+    if (const char* e = getenv("DDA_DIST_CHUNK")) chunk = atoi(e) > 0 ? atoi(e) : 8;
+    SState out = h;
+    for (int k = 0; !h.done && k < maxit; k += chunk) {
+        for (int ci = 0; ci < chunk && k + ci < maxit; ++ci) {
+            const int j = k + ci;
+            DDA_TRY(halo_exchange_w(c, st, 1, 6));                               // r~
+            if (j >= 1) DDA_TRY(halo_exchange_w(c, st, ((j - 1) & 1) ? 3 : 2, 6));   // p_{j-1}
+            for (size_t p = 0; p < c->parts.size(); ++p) {
+                DistPart& D = c->parts[p];
+                SState* ds = reinterpret_cast<SState*>(D.dst);
+                k_v3_a<<<D.G_a3, DDA_THREADS, 0, st>>>(own_view_sc(D), D.rt, D.pA, D.pB, D.q, d[p], ds, D.part);
+                DDA_LAUNCHED();
+                k_sum_parts<<<1, DDA_THREADS, 0, st>>>(D.part, D.G_a3, 1, D.scal);
+                DDA_LAUNCHED();
+            }
+            DDA_TRY(allreduce_dev(c, 1, st));
+            for (DistPart& D : c->parts) {
+                SState* ds = reinterpret_cast<SState*>(D.dst);
+                k_v3_alpha<<<1, 1, 0, st>>>(ds, D.red);
+                DDA_LAUNCHED();
+                k_v3_b<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, D.rt, D.q, D.K->bj_w, ds, D.part);
+                DDA_LAUNCHED();
+                k_sum_parts<<<1, DDA_THREADS, 0, st>>>(D.part, D.G_vec, 2, D.scal);
+                DDA_LAUNCHED();
+            }
+            DDA_TRY(allreduce_dev(c, 2, st));
+            for (DistPart& D : c->parts) {
+                SState* ds = reinterpret_cast<SState*>(D.dst);
+                k_v3_rho<<<1, 1, 0, st>>>(ds, D.red);
+                DDA_LAUNCHED();
+                k_v3_c<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, D.rt, D.K->lfac, ds, D.part);
+                DDA_LAUNCHED();
+                k_sum_parts<<<1, DDA_THREADS, 0, st>>>(D.part, D.G_vec, 1, D.scal);
+                DDA_LAUNCHED();
+            }
+            DDA_TRY(allreduce_dev(c, 1, st));
+            for (DistPart& D : c->parts) {
+                k_v3_check<<<1, 1, 0, st>>>(reinterpret_cast<SState*>(D.dst), D.red);
+                DDA_LAUNCHED();
+            }
+        }
+        DDA_CK(cudaMemcpyAsync(&out, c->parts[0].dst, sizeof out, cudaMemcpyDeviceToHost, st));
+        DDA_CK(cudaStreamSynchronize(st));
+        if (out.done) break;
+    }
+    for (size_t p = 0; p < c->parts.size(); ++p) {          // d = S^T x (after the pending x update)
+        DistPart& D = c->parts[p];
+        k_v3_final<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, d[p], D.pA, D.pB, D.K->sfac,
+                                                    reinterpret_cast<SState*>(D.dst));
+        DDA_LAUNCHED();
+    }
+    DDA_CK(cudaMemcpyAsync(&out, c->parts[0].dst, sizeof out, cudaMemcpyDeviceToHost, st));
+    DDA_CK(cudaStreamSynchronize(st));
+    *status = (dda_status_t)out.status;
+    *it = out.iters;
+    return DDA_OK;
+}
+
+}  // namespace
+
 extern "C" dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double* const* F, const double* const* d0,
                                            double* const* d, double tol, int32_t maxit, dda_precond_t pc,
                                            int32_t* iters, double* rel_res, void* stream) {
@@ -554,6 +911,35 @@ extern "C" dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double* const* F,
         if (!D.K) return DDA_ERR_ARG;
     if (use_bj)
         for (DistPart& D : c->parts) DDA_TRY(bj_setup_rows(D.K, D.n_own, st, nullptr));
+    // v3 (default for block-Jacobi): the scaled engine per partition; DDA_DIST_SCALED=0 selects v2
+    const char* dse = getenv("DDA_DIST_SCALED");
+    if (use_bj && !(dse && dse[0] == '0')) {
+        dda_status_t status = DDA_ERR_NO_CONVERGENCE;
+        int it = 0;
+        bool zero = false;
+        double bnorm = 0.0;
+        DDA_TRY(dist_scaled_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, st));
+        if (zero) return DDA_OK;
+        // true residual ||F - K d|| / ||F|| (unscaled, over the partitions)
+        for (size_t p = 0; p < c->parts.size(); ++p) {
+            DistPart& D = c->parts[p];
+            DDA_CK(cudaMemcpyAsync(D.x, d[p], 6 * sizeof(double) * D.n_own, cudaMemcpyDeviceToDevice, st));
+        }
+        DDA_TRY(halo_exchange(c, st));
+        DDA_TRY(spmv_parts(c, false, st));
+        for (size_t p = 0; p < c->parts.size(); ++p) {
+            DistPart& D = c->parts[p];
+            k_resid_own<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, F[p], D.q, D.part);
+            DDA_LAUNCHED();
+            k_sum_parts<<<1, DDA_THREADS, 0, st>>>(D.part, D.G_vec, 1, D.scal);
+            DDA_LAUNCHED();
+        }
+        double res;
+        DDA_TRY(allreduce_host(c, 1, &res, st));
+        if (iters) *iters = it;
+        if (rel_res) *rel_res = std::sqrt(res) / bnorm;
+        return status;
+    }
     const bool have_d0 = d0 != nullptr;
     // ---- setup: r = F - K d0
     if (have_d0) {

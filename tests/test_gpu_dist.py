@@ -60,8 +60,19 @@ def test_spmv_dist_loopback(dda, prob, nparts):
     assert (np.abs(y - yo) <= 1e-12 * bound).all()
 
 
+@pytest.fixture(params=["v3", "v2"])
+def dist_version(request, monkeypatch):
+    """v3 = the scaled block-Jacobi engine per partition (default); v2 = the unscaled loop
+    (DDA_DIST_SCALED=0, read by the library on every solve)."""
+    if request.param == "v2":
+        monkeypatch.setenv("DDA_DIST_SCALED", "0")
+    else:
+        monkeypatch.delenv("DDA_DIST_SCALED", raising=False)
+    return request.param
+
+
 @pytest.mark.parametrize("nparts", [1, 2, 4])
-def test_pcg_dist_loopback(dda, prob, nparts):
+def test_pcg_dist_loopback(dda, prob, nparts, dist_version):
     P, O = prob
     comm, lps, Ks = _setup(dda, P, nparts)
     Fs = [torch.from_numpy(lp.F).cuda() for lp in lps]
@@ -74,7 +85,7 @@ def test_pcg_dist_loopback(dda, prob, nparts):
     assert np.linalg.norm(d - dm) / np.linalg.norm(dm) <= 1e-9
 
 
-def test_pcg_dist_warm_and_zero(dda, prob):
+def test_pcg_dist_warm_and_zero(dda, prob, dist_version):
     P, O = prob
     comm, lps, Ks = _setup(dda, P, 3)
     Fs = [torch.from_numpy(lp.F).cuda() for lp in lps]
@@ -89,7 +100,7 @@ def test_pcg_dist_warm_and_zero(dda, prob):
     assert st5 == dda.ERR_NO_CONVERGENCE and it5 == 13 and rr5 > 1e-10
 
 
-def test_pcg_dist_nccl_single_rank(dda, prob):
+def test_pcg_dist_nccl_single_rank(dda, prob, dist_version):
     P, O = prob
     uid = dda.Comm.unique_id()
     comm = dda.Comm.nccl(1, 0, uid)
