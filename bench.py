@@ -459,8 +459,10 @@ def run_dist(args, P, world, rank, local):
     pcg = statistics.mean(e[1].elapsed_time(e[2]) for e in evs)
     K, iters, rel_res, status = res[-1]
     assert status == dda.OK and rel_res <= 1.01e-10, (status, rel_res)
-    u = K.nnzb / max(lp.n_local, 1)
-    local_bytes = lp.n_own * (bytes_per_row_spmv(u) + 672.0) * iters
+    # v3 (block-Jacobi): the scaled engine per rank, 300u + 448 algorithmic bytes per own row and
+    # iteration as on one GPU; u over the rank's own rows
+    u = K.nnzb / max(lp.n_own, 1)
+    local_bytes = lp.n_own * (300.0 * u + 448.0) * iters
     ach = local_bytes / (pcg * 1e-3) / 1e9
     tt = torch.tensor([ms, pcg, asm], device="cuda")
     dist.all_reduce(tt, op=dist.ReduceOp.MAX)
@@ -500,7 +502,9 @@ def run_dist(args, P, world, rank, local):
                        "l2": "inputs larger than L2 per rank at 1M/N; no flush"},
             "phases_ms": {"assemble_max": asm_max, "pcg_max": pcg_max, "pcg_iters": iters,
                           "pcg_us_per_iter": 1000.0 * pcg_max / max(iters, 1), "true_rel_res": rel_res},
-            "roofline": {"kernel": "rank 0: k_spmv_own + k_update_own (+ NCCL halo/allreduce)", "bound": "hbm",
+            "roofline": {"kernel": "rank 0: dist v3 scaled engine (k_v3_a fused p-update + Ks SpMV, k_v3_b, "
+                                   "one-thread scalar kernels; NCCL halo of r~ and p, device-buffer allreduces)",
+                         "bound": "hbm",
                          "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
                          "traffic": None, "peak_source": peak_src, "per": "GPU (rank 0)"},
             "e2e": e2e, "cpu_baseline": None, "gpu_launches": int(launches), "clocks": clk.summary(),
