@@ -141,3 +141,16 @@ def test_contacts_bad_input(dda):
     vptr, vxy, _ = _random_polygons(4, 1)
     with pytest.raises(dda.DDAError):
         _gpu(dda, vptr, vxy, 0.0)
+
+
+def test_contacts_mixed_sizes(dda):
+    """One large polygon among small ones: the broad-phase cell is sized by the largest block, so the
+    small blocks crowd into few cells — records must still equal the oracle's."""
+    vptr, vxy, cxy = _random_polygons(150, 9)
+    big = np.array([[3.0, 3.0], [9.0, 3.2], [9.5, 8.0], [3.2, 9.0]])
+    vptr2 = np.concatenate([vptr, [vptr[-1] + 4]]).astype(np.int32)
+    vxy2 = np.concatenate([vxy, big])
+    O = oracle.detect_contacts(vptr2, vxy2, 0.3)
+    Cg, G = _gpu(dda, vptr2, vxy2, 0.3)
+    assert (O["i"] == 150).any() or (O["j"] == 150).any()
+    _same(G, O)
