@@ -166,8 +166,12 @@ dda_status_t dda_precond_apply(dda_matrix_t K, dda_precond_t pc, double omega, c
  *  pc      preconditioner;  omega: SSOR-AI relaxation (1.0 default, ignored otherwise)
  *  iters   host out: iterations performed
  *  rel_res host out: TRUE relative residual ||F - K d||_2 / ||F||_2 (one extra SpMV)
- * The whole iteration runs on the device (one persistent cooperative kernel);
- * the host reads the result once at the end.  Returns DDA_OK,
+ * The whole iteration runs on the device; the host reads the result once at the end.
+ * Block-Jacobi and SSOR-AI run PCG on the block-scaled S K S^T (S = blockdiag(L_i^{-1}),
+ * same iterates, reading Z25) in ONE persistent cooperative kernel, whose CTAs must all be
+ * co-resident: on a GPU shared with other work the launch can fail with DDA_ERR_CUDA
+ * (DDA_SCALED_LOOP=graph selects the CUDA-graph while loop for block-Jacobi instead).
+ * ILU(0) and the unpreconditioned solve run a CUDA-graph device-side while loop.  Returns DDA_OK,
  * DDA_ERR_NO_CONVERGENCE (d, iters, rel_res still filled), DDA_ERR_BREAKDOWN
  * (d = last iterate), DDA_ERR_NOT_SPD (preconditioner setup).  F = 0 gives
  * d = 0, iters = 0, rel_res = 0, DDA_OK (reading Z2).  Synchronising.
