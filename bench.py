@@ -168,10 +168,12 @@ def dist_env():
 
 # ----------------------------------------------------------------------------- CPU oracle legs
 
-def oracle_step_sample(n_sample: int, seed: int = 1005):
+def oracle_step_sample(n_sample: int, seed: int = 1005, spmv_stats: dict = None):
     """Oracle (one thread, as it stands) on a bounded sample of the workload: the full
     step (assembly O-1 + expansion O-2, block inverses, PCG to 1e-10) on a slope of
-    ~n_sample blocks from the same recipe.  Returns (seconds, n, iters)."""
+    ~n_sample blocks from the same recipe.  Returns (seconds, n, iters).  If spmv_stats is
+    given, it also times (outside the step) one oracle SpMV on 1 thread and the OpenMP
+    all-cores variant (SURVEY §8(d)'s labelled second number) and fills the dict."""
     import oracle
     from synth import make_slope, preset
     P = make_slope(preset(n_sample, seed=seed))
@@ -180,6 +182,14 @@ def oracle_step_sample(n_sample: int, seed: int = 1005):
     M.full_csr()
     d, it, rr, st = M.pcg(P.F, tol=1e-10, maxit=10000, precond="bj")
     t1 = time.perf_counter()
+    if spmv_stats is not None:
+        x = np.random.default_rng(7).uniform(-1.0, 1.0, 6 * P.n)
+        one, par, th = [], [], 1
+        for _ in range(3):
+            a = time.perf_counter(); M.spmv(x); one.append(time.perf_counter() - a)
+            a = time.perf_counter(); _, th = M.spmv_par(x); par.append(time.perf_counter() - a)
+        spmv_stats.update({"spmv_1_thread_ms": 1000.0 * statistics.median(one),
+                           "spmv_all_cores_ms": 1000.0 * statistics.median(par), "all_cores_threads": th})
     return t1 - t0, P.n, it
 
 
@@ -374,12 +384,19 @@ def main():
     # ---- CPU oracle baseline (rank 0, N=1 only)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
-        s, n_s, it_s = oracle_step_sample(args.cpu_sample_blocks)
+        sst = {}
+        s, n_s, it_s = oracle_step_sample(args.cpu_sample_blocks, spmv_stats=sst)
         scale = n / n_s
         cpu = {"value": 1000.0 * s * scale, "unit": UNIT, "cores": 1, "kind": "oracle",
                "sample": (f"oracle full step (assembly+expansion, BJ inverses, PCG to 1e-10: {it_s} iters) on a "
                           f"{n_s}-block slope of the same recipe, 1 thread, {s:.1f} s, scaled x{scale:.2f} by "
-                          f"block count"), "host_cores": os.cpu_count()}
+                          f"block count"), "host_cores": os.cpu_count(),
+               "spmv_oracle": {"one_thread_ms_scaled": sst.get("spmv_1_thread_ms", 0.0) * scale,
+                               "all_cores_ms_scaled": sst.get("spmv_all_cores_ms", 0.0) * scale,
+                               "all_cores_threads": sst.get("all_cores_threads", 1),
+                               "note": (f"one oracle SpMV (full scalar CSR, O-3) on the {n_s}-block sample, "
+                                        "1 thread and OpenMP all cores (labelled second number, SURVEY §8(d)), "
+                                        "scaled by block count; the GPU SpMV is the line's spmv.ms")}}
 
     line = {
         "metric": METRIC, "value": ms_step, "unit": UNIT, "n_gpus": world, "steps": args.steps,

@@ -31,7 +31,7 @@ PC = {"none": 0, "bj": 1, "ssor_ai": 2, "ilu0": 3}
 def build(force: bool = False) -> str:
     """Compile liboracle.so with gcc (no FMA contraction: values round as written)."""
     if force or not os.path.exists(_LIB) or os.path.getmtime(_LIB) < os.path.getmtime(_SRC):
-        subprocess.check_call(["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math",
+        subprocess.check_call(["gcc", "-O2", "-std=c11", "-ffp-contract=off", "-fno-fast-math", "-fopenmp",
                                "-fPIC", "-shared", "-Wall", "-Wno-unused-label", "-o", _LIB, _SRC, "-lm"])
     return _LIB
 
@@ -55,6 +55,7 @@ def lib():
         L.orc_full_export.argtypes = [P, P, P, P]
         L.orc_spmv.argtypes = [P, P, P]
         L.orc_spmv_rows.argtypes = [P, P, C.c_int64, P, P]
+        L.orc_spmv_par.argtypes = [P, P, P, C.POINTER(C.c_int32)]
         L.orc_bj_inv.argtypes = [P, P, C.POINTER(C.c_int32)]
         L.orc_ssor_ai_apply.argtypes = [P, P, C.c_double, P, P]
         L.orc_ilu0_factor.argtypes = [P]
@@ -149,6 +150,16 @@ class OracleMatrix:
             raise OracleError(st, "spmv")
         return y
 
+
+    def spmv_par(self, x):
+        """O-3 split over OpenMP threads (timing variant, bitwise equal to spmv).  Returns (y, threads)."""
+        x = np.ascontiguousarray(x, np.float64)
+        y = np.empty(6 * self.n)
+        th = C.c_int32()
+        st = lib().orc_spmv_par(self.h, _p(x), _p(y), C.byref(th))
+        if st != OK:
+            raise OracleError(st, "spmv_par")
+        return y, int(th.value)
     def spmv_rows(self, rows, x):
         rows = np.ascontiguousarray(rows, np.int64)
         x = np.ascontiguousarray(x, np.float64)

@@ -165,3 +165,12 @@ def test_shuffled_ordering_same_operator():
     ip, ix, dv = Mb.full_csr()
     pa = np.sort(np.linalg.eigvalsh(sp.csr_matrix((dv, ix, ip), shape=(6 * b.n,) * 2).toarray()))
     assert np.allclose(ea, pa, rtol=1e-11, atol=1e-11 * ea.max())
+
+
+def test_spmv_par_equals_spmv():
+    """The OpenMP timing variant of O-3 sums every row in the same order: bitwise equal."""
+    P = make_slope(preset(2000, seed=1041))
+    M = oracle.assemble(P)
+    x = np.random.default_rng(3).uniform(-1, 1, 6 * P.n)
+    y, th = M.spmv_par(x)
+    assert th >= 1 and np.array_equal(y, M.spmv(x))
