@@ -214,10 +214,14 @@ dda_status_t dda_solve_host(int32_t n_blocks, const double *kdiag, int64_t n_spr
  * dda_pcg_solve_dist: F[p], d0[p] (entry or whole array may be NULL), d[p]:
  * device [6 n_own] per local partition (one entry for NCCL).  Same stop rule,
  * statuses and reported TRUE residual as dda_pcg_solve; DDA_PC_BJ or
- * DDA_PC_NONE (SSOR-AI and ILU(0) are single-GPU only).  Per iteration: one
- * halo exchange of p, the symmetric SpMV over own rows, two allreduces
- * (p^T q; r^T r and r^T z).  Synchronising.  dda_spmv_dist: y = K x over own
- * rows (x, y device [6 n_own] per partition).
+ * DDA_PC_NONE (SSOR-AI and ILU(0) are single-GPU only).  Block-Jacobi runs the
+ * scaled engine per partition (PCG on S K S^T, reading Z25; S of the halo rows is
+ * exchanged once per solve); per iteration: halo exchanges of r~ and p, the fused
+ * p-update + SpMV over own rows, allreduces of p^T q and of (|r~|^2, the stopping
+ * bound), and of |L r~|^2 when the exact stopping test is due.  The CG scalars
+ * stay on the device; the host reads the loop state once per DDA_DIST_CHUNK (8)
+ * iterations.  DDA_DIST_SCALED=0 selects the unscaled loop.  Synchronising.
+ * dda_spmv_dist: y = K x over own rows (x, y device [6 n_own] per partition).
  */
 typedef struct dda_comm *dda_comm_t;
 dda_status_t dda_comm_unique_id(void *id128);
