@@ -291,13 +291,22 @@ extern "C" void dda_matrix_free(dda_matrix_t K) {
 extern "C" dda_status_t dda_build_matrix(int32_t n, const double* kdiag, int64_t m, const int32_t* bi,
                                          const int32_t* bj, const double* pen, const double* e, const double* g,
                                          void* stream, dda_matrix_t* out) {
+    return dda::build_matrix_impl(n, kdiag, m, bi, bj, pen, e, g, reinterpret_cast<cudaStream_t>(stream), nullptr,
+                                  out);
+}
+
+// values_ready (may be null): the stream waits for it before the first use of kdiag / e / g, so the
+// host->device copies of those arrays can overlap the key sorts (dda_solve_host)
+dda_status_t dda::build_matrix_impl(int32_t n, const double* kdiag, int64_t m, const int32_t* bi, const int32_t* bj,
+                                    const double* pen, const double* e, const double* g, cudaStream_t stream,
+                                    cudaEvent_t values_ready, dda_matrix_t* out) {
     if (!out) return DDA_ERR_ARG;
     *out = nullptr;
     if (n <= 0 || m < 0 || !kdiag) return DDA_ERR_ARG;
     if (m > 0 && (!bi || !bj || !pen || !e || !g)) return DDA_ERR_ARG;
     if (m > (int64_t)INT_MAX / 2 || (int64_t)n > (int64_t)INT_MAX / 36) return DDA_ERR_ARG;
     if (m > 0 && ((reinterpret_cast<uintptr_t>(e) | reinterpret_cast<uintptr_t>(g)) & 15)) return DDA_ERR_ARG;
-    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    cudaStream_t st = stream;
 
     dda_matrix* K = new dda_matrix();
     DDA_CK(cudaGetDevice(&K->device));
@@ -402,6 +411,7 @@ extern "C" dda_status_t dda_build_matrix(int32_t n, const double* kdiag, int64_t
 
     trace("build: structure issued");
     // ---- values (the final step that moves data)
+    if (values_ready) DDA_CK(cudaStreamWaitEvent(st, values_ready, 0));
     {
         dda_status_t sv = run_values(K, kdiag, pen, e, g, st);
         if (sv != DDA_OK) return sv;

@@ -568,19 +568,41 @@ extern "C" dda_status_t dda_solve_host(int32_t n, const double* kdiag, int64_t m
     double* dg = reinterpret_cast<double*>(buf + off[6]);
     int32_t* dbi = reinterpret_cast<int32_t*>(buf + off[7]);
     int32_t* dbj = reinterpret_cast<int32_t*>(buf + off[8]);
-    DDA_CK(cudaMemcpyAsync(dk, kdiag, sizeof(double) * 36 * (size_t)n, cudaMemcpyHostToDevice, st));
-    DDA_CK(cudaMemcpyAsync(dF, F, sizeof(double) * N, cudaMemcpyHostToDevice, st));
-    if (d0) DDA_CK(cudaMemcpyAsync(dd0, d0, sizeof(double) * N, cudaMemcpyHostToDevice, st));
+    // The key arrays (bi, bj, pen) go first on the caller's stream; e, g, kdiag (needed only by the
+    // value step of the assembly) and F, d0 (needed by the solve) follow on a second stream, so their
+    // transfer overlaps the key sorts.  The caller's stream waits on two events before using them.
+    struct Aux {
+        cudaStream_t cs = nullptr;
+        cudaEvent_t vals = nullptr, rhs = nullptr, start = nullptr;
+        ~Aux() {
+            if (cs) { cudaStreamSynchronize(cs); cudaStreamDestroy(cs); }
+            if (vals) cudaEventDestroy(vals);
+            if (rhs) cudaEventDestroy(rhs);
+            if (start) cudaEventDestroy(start);
+        }
+    } aux;
+    DDA_CK(cudaStreamCreateWithFlags(&aux.cs, cudaStreamNonBlocking));
+    DDA_CK(cudaEventCreateWithFlags(&aux.vals, cudaEventDisableTiming));
+    DDA_CK(cudaEventCreateWithFlags(&aux.rhs, cudaEventDisableTiming));
+    DDA_CK(cudaEventCreateWithFlags(&aux.start, cudaEventDisableTiming));
+    DDA_CK(cudaEventRecord(aux.start, st));                 // the buffer is allocated stream-ordered on st
+    DDA_CK(cudaStreamWaitEvent(aux.cs, aux.start, 0));
     if (m > 0) {
-        DDA_CK(cudaMemcpyAsync(dpen, pen, sizeof(double) * m, cudaMemcpyHostToDevice, st));
-        DDA_CK(cudaMemcpyAsync(de, e, sizeof(double) * 6 * m, cudaMemcpyHostToDevice, st));
-        DDA_CK(cudaMemcpyAsync(dg, g, sizeof(double) * 6 * m, cudaMemcpyHostToDevice, st));
         DDA_CK(cudaMemcpyAsync(dbi, bi, sizeof(int32_t) * m, cudaMemcpyHostToDevice, st));
         DDA_CK(cudaMemcpyAsync(dbj, bj, sizeof(int32_t) * m, cudaMemcpyHostToDevice, st));
+        DDA_CK(cudaMemcpyAsync(dpen, pen, sizeof(double) * m, cudaMemcpyHostToDevice, st));
+        DDA_CK(cudaMemcpyAsync(de, e, sizeof(double) * 6 * m, cudaMemcpyHostToDevice, aux.cs));
+        DDA_CK(cudaMemcpyAsync(dg, g, sizeof(double) * 6 * m, cudaMemcpyHostToDevice, aux.cs));
     }
+    DDA_CK(cudaMemcpyAsync(dk, kdiag, sizeof(double) * 36 * (size_t)n, cudaMemcpyHostToDevice, aux.cs));
+    DDA_CK(cudaEventRecord(aux.vals, aux.cs));
+    DDA_CK(cudaMemcpyAsync(dF, F, sizeof(double) * N, cudaMemcpyHostToDevice, aux.cs));
+    if (d0) DDA_CK(cudaMemcpyAsync(dd0, d0, sizeof(double) * N, cudaMemcpyHostToDevice, aux.cs));
+    DDA_CK(cudaEventRecord(aux.rhs, aux.cs));
     dda_matrix_t K = nullptr;
-    dda_status_t s = dda_build_matrix(n, dk, m, dbi, dbj, dpen, de, dg, stream, &K);
+    dda_status_t s = build_matrix_impl(n, dk, m, dbi, dbj, dpen, de, dg, st, aux.vals, &K);
     if (s != DDA_OK) return s;
+    DDA_CK(cudaStreamWaitEvent(st, aux.rhs, 0));
     s = dda_pcg_solve(K, dF, d0 ? dd0 : nullptr, dd, tol, maxit, pc, omega, iters, rel_res, stream);
     if (s == DDA_OK || s == DDA_ERR_NO_CONVERGENCE || s == DDA_ERR_BREAKDOWN) {
         cudaError_t ce = cudaMemcpyAsync(d, dd, sizeof(double) * N, cudaMemcpyDeviceToHost, st);
