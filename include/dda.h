@@ -169,8 +169,10 @@ dda_status_t dda_precond_apply(dda_matrix_t K, dda_precond_t pc, double omega, c
  * The whole iteration runs on the device; the host reads the result once at the end.
  * Block-Jacobi and SSOR-AI run PCG on the block-scaled S K S^T (S = blockdiag(L_i^{-1}),
  * same iterates, reading Z25) in ONE persistent cooperative kernel, whose CTAs must all be
- * co-resident: on a GPU shared with other work the launch can fail with DDA_ERR_CUDA
- * (DDA_SCALED_LOOP=graph selects the CUDA-graph while loop for block-Jacobi instead).
+ * co-resident.  When the occupancy query finds no room for it, the solve falls back before
+ * writing any state (block-Jacobi: the CUDA-graph while loop with the same phases as kernels;
+ * SSOR-AI: the unscaled graph engine); a cooperative launch that still fails returns
+ * DDA_ERR_CUDA (DDA_SCALED_LOOP=graph selects the graph loop for block-Jacobi explicitly).
  * ILU(0) and the unpreconditioned solve run a CUDA-graph device-side while loop.  Returns DDA_OK,
  * DDA_ERR_NO_CONVERGENCE (d, iters, rel_res still filled), DDA_ERR_BREAKDOWN
  * (d = last iterate), DDA_ERR_NOT_SPD (preconditioner setup).  F = 0 gives

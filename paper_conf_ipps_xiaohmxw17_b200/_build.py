@@ -45,12 +45,29 @@ def needs_build() -> bool:
 
 
 def build(force: bool = False, verbose: bool = False, extra=()) -> str:
+    """nvcc -c every csrc/*.cu in parallel (one process per file), then link libdda.so."""
     if not force and not needs_build():
         return LIB
+    from concurrent.futures import ThreadPoolExecutor
+
     nvcc = os.environ.get("NVCC", "nvcc")
     ninc, nlib = nccl_dirs()
-    cmd = [nvcc, *NVCC_FLAGS, *extra, "-I", INCLUDE, "-I", CSRC, "-I", ninc, *sources(), "-o", LIB + ".tmp",
-           "-L", nlib, "-l:libnccl.so.2", "-Xlinker", "-rpath=" + nlib]
+    objdir = os.path.join(PKG, "build")
+    os.makedirs(objdir, exist_ok=True)
+    flags = [f for f in NVCC_FLAGS if f != "-shared"]
+
+    def compile_one(src):
+        obj = os.path.join(objdir, os.path.basename(src)[:-3] + ".o")
+        cmd = [nvcc, *flags, *extra, "-I", INCLUDE, "-I", CSRC, "-I", ninc, "-c", src, "-o", obj]
+        if verbose:
+            print(" ".join(cmd))
+        subprocess.check_call(cmd)
+        return obj
+
+    with ThreadPoolExecutor(max_workers=min(16, os.cpu_count() or 4)) as ex:
+        objs = list(ex.map(compile_one, sources()))
+    cmd = [nvcc, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-Xcompiler", "-fPIC", *objs,
+           "-o", LIB + ".tmp", "-L", nlib, "-l:libnccl.so.2", "-Xlinker", "-rpath=" + nlib]
     if verbose:
         print(" ".join(cmd))
     subprocess.check_call(cmd)

@@ -585,6 +585,16 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
             if (v) dev_free(v);
         D = DistPart();
     }
+    for (int q = 0; q < P; ++q)
+        if (send_counts[q] < 0 || recv_counts[q] < 0 || (q == c->rank && !c->loopback && (send_counts[q] || recv_counts[q])))
+            return DDA_ERR_ARG;
+    {   // every send index is an own row (k_pack_w gathers them without bounds checks)
+        int64_t ns = 0;
+        for (int q = 0; q < P; ++q) ns += send_counts[q];
+        if (ns && !send_idx) return DDA_ERR_ARG;
+        for (int64_t t = 0; t < ns; ++t)
+            if (send_idx[t] < 0 || send_idx[t] >= n_own) return DDA_ERR_ARG;
+    }
     D.K = K;
     D.n_own = n_own;
     D.n_local = K->n;
@@ -635,6 +645,20 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     if (D.n_send)
         DDA_CK(cudaMemcpyAsync(D.send_idx, send_idx, D.n_send * sizeof(int), cudaMemcpyHostToDevice, st));
     DDA_CK(cudaMemsetAsync(D.x, 0, nl6 * sizeof(double), st));
+    if (!c->loopback && P > 1) {   // the peers' send counts must equal this rank's receive counts
+        int* cnt = nullptr;
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&cnt), (size_t)P * (P + 1) * sizeof(int), st));
+        DDA_CK(cudaMemcpyAsync(cnt, send_counts, P * sizeof(int), cudaMemcpyHostToDevice, st));
+        const ncclResult_t r = ncclAllGather(cnt, cnt + P, P, ncclInt32, c->nccl, st);
+        std::vector<int> all((size_t)P * P);
+        if (r == ncclSuccess)
+            DDA_CK(cudaMemcpyAsync(all.data(), cnt + P, (size_t)P * P * sizeof(int), cudaMemcpyDeviceToHost, st));
+        DDA_CK(cudaStreamSynchronize(st));
+        dev_free_on(cnt, st);
+        if (r != ncclSuccess) return DDA_ERR_NCCL;
+        for (int q = 0; q < P; ++q)
+            if (all[(size_t)q * P + c->rank] != recv_counts[q]) return DDA_ERR_ARG;
+    }
     DDA_CK(cudaStreamSynchronize(st));
     return DDA_OK;
 }

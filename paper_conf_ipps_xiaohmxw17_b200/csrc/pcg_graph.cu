@@ -752,9 +752,13 @@ struct XFusedW {
 };
 
 // Fixed-order grid sums of NV values per thread: CTA partials -> part[(slot+k)*Gmax + cta], grid
-// barrier, then every CTA sums the G partials in the order grid_reduce_last uses.  Slots: 0 (phase
-// A), 1-2 (phase B), 0 (phase C); a slot is rewritten only after at least one further barrier, so
-// no CTA can still be reading it.
+// barrier, then every CTA sums the G partials in the order grid_reduce_last uses.  k_sp_loop slots:
+// 0 (phase A), 1-2 (phase B), 3 (phase C).  A CTA writes slot s only after passing at least one
+// barrier that follows every read of s: phase A's slot 0 is read before barrier B, phase B's slots
+// before barrier C or the next iteration's barrier A, phase C's slot 3 before the next barrier A.
+// (Phase C on slot 0 would race: a fast CTA's next phase A rewrites slot 0 while a slow CTA is
+// still summing the exact-test partials, and the CTAs could then disagree on the stop decision.)
+// k_sp_ssor: 0 (A), 1-2 (L), 0 (C, followed by the U barrier before the next A), 3 (U).
 template <int NV>
 __device__ __forceinline__ void grid_allsum(const GArgs& a, cg::grid_group& grid, int slot, double (&v)[NV],
                                             double (&tot)[NV]) {
@@ -882,7 +886,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_loop(const GArgs a) {
                 rl += o * o;
             }
             double cv[1] = {rl}, ctot[1];
-            grid_allsum<1>(a, grid, 0, cv, ctot);
+            grid_allsum<1>(a, grid, 3, cv, ctot);   // slot 3: slot 0 is rewritten by the next phase A
             const double rr = ctot[0];
             checks += 1;
             rr_last = rr;
@@ -1220,9 +1224,23 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         g_scaled_loop = (e && (e[0] == 'g' || e[0] == '0')) ? 0 : 1;
     }
     // scaled SSOR-AI exists as a persistent kernel only (k_sp_ssor)
-    const bool persist = scaled && (g_scaled_loop == 1 || pc == DDA_PC_SSOR_AI);
+    bool persist = scaled && (g_scaled_loop == 1 || pc == DDA_PC_SSOR_AI);
     const void* persist_kernel = pc == DDA_PC_SSOR_AI ? reinterpret_cast<const void*>(k_sp_ssor)
                                                       : reinterpret_cast<const void*>(k_sp_loop<3>);
+    if (persist) {
+        // The persistent kernels need every CTA co-resident (cooperative launch).  If not even one CTA
+        // per SM fits (e.g. a smaller shared-memory carve-out forced by the caller's context), fall
+        // back before any state is written: scaled BJ to the CUDA-graph while loop (same phases as
+        // kernels), SSOR-AI to the unscaled graph engine.
+        int per_sm = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, persist_kernel, DDA_THREADS, 0);
+        if (per_sm < 1) {
+            trace("solve: cooperative grid does not fit, graph loop fallback");
+            if (pc == DDA_PC_SSOR_AI)
+                return pcg_graph_solve(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, st, false);
+            persist = false;
+        }
+    }
     const int key = scaled ? (persist ? 200 : 100) + (int)pc : (int)pc;
     PcgGraph*& G = reinterpret_cast<PcgGraph*&>(K->graph_engine);
     if (G && G->pc != key) {
@@ -1244,7 +1262,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
             int per_sm = 0;
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, persist_kernel, DDA_THREADS, 0);
             if (per_sm > 3) per_sm = 3;
-            if (per_sm < 1) return DDA_ERR_CUDA;
+            if (per_sm < 1) per_sm = 1;   // (checked above)
             g_persist = device_sms() * per_sm;
             // small (L2-resident) systems are barrier-latency bound: no more CTAs than ten-row groups
             // need (DDA_PERSIST_CTAS overrides, tuning aid)

@@ -149,14 +149,26 @@ extern "C" dda_status_t dda_spmv_full(dda_matrix_t K, const double* x, double* y
     if (!K || !x || !y || x == y) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (!K->full_ptr) {
+        // allocate into locals and publish only when all three exist (a partial expansion must not
+        // be taken for a built one on the next call)
         const size_t nb = (size_t)K->n + 2 * (size_t)K->nnzb;
-        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->full_ptr), ((size_t)K->n + 1) * sizeof(int32_t), st));
-        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->full_col), nb * sizeof(int32_t), st));
-        DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->full_val), nb * kBlk * sizeof(double), st));
-        k_full_ptr<<<(K->n + 256) / 256, 256, 0, st>>>(K->n, K->row_ptr, K->low_ptr, K->full_ptr);
+        int32_t *fp = nullptr, *fc = nullptr;
+        double* fv = nullptr;
+        cudaError_t e = dev_alloc(reinterpret_cast<void**>(&fp), ((size_t)K->n + 1) * sizeof(int32_t), st);
+        if (e == cudaSuccess) e = dev_alloc(reinterpret_cast<void**>(&fc), nb * sizeof(int32_t), st);
+        if (e == cudaSuccess) e = dev_alloc(reinterpret_cast<void**>(&fv), nb * kBlk * sizeof(double), st);
+        if (e != cudaSuccess) {
+            if (fp) dev_free_on(fp, st);
+            if (fc) dev_free_on(fc, st);
+            return cuda_fail(e);
+        }
+        k_full_ptr<<<(K->n + 256) / 256, 256, 0, st>>>(K->n, K->row_ptr, K->low_ptr, fp);
         DDA_LAUNCHED();
-        k_full_fill<<<device_sms() * 8, 256, 0, st>>>(K->n, view_of(K), K->full_ptr, K->full_col, K->full_val);
+        k_full_fill<<<device_sms() * 8, 256, 0, st>>>(K->n, view_of(K), fp, fc, fv);
         DDA_LAUNCHED();
+        K->full_ptr = fp;
+        K->full_col = fc;
+        K->full_val = fv;
     }
     BsrView F = view_of(K);
     F.row_ptr = K->full_ptr;
