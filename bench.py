@@ -168,29 +168,91 @@ def dist_env():
 
 # ----------------------------------------------------------------------------- CPU oracle legs
 
-def oracle_step_sample(n_sample: int, seed: int = 1005, spmv_stats: dict = None):
-    """Oracle (one thread, as it stands) on a bounded sample of the workload: the full
-    step (assembly O-1 + expansion O-2, block inverses, PCG to 1e-10) on a slope of
-    ~n_sample blocks from the same recipe.  Returns (seconds, n, iters).  If spmv_stats is
-    given, it also times (outside the step) one oracle SpMV on 1 thread and the OpenMP
-    all-cores variant (SURVEY §8(d)'s labelled second number) and fills the dict."""
+ORACLE_1M = os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "r02_oracle_1m.json")
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def oracle_iters_for(P):
+    """The oracle's own BJ-PCG iteration count to 1e-10 on this exact system, from the committed
+    record of tools/oracle_1m.py (synth + oracle only; checked by problem fingerprint), or None."""
+    try:
+        rec = json.load(open(ORACLE_1M))
+    except (OSError, ValueError):
+        return None, None
+    import hashlib
+    h = hashlib.sha256()
+    for a in (P.bi, P.bj, P.pen, P.F):
+        h.update(np.ascontiguousarray(a).tobytes())
+    if rec.get("n_blocks") != P.n or rec.get("fingerprint") != h.hexdigest()[:16]:
+        return None, None
+    return int(rec["oracle_iters"]), rec
+
+
+def oracle_step_at_size(P, k_sample: int = 8, spmv_stats: dict = None):
+    """The oracle (as it stands, one pinned host core) on THE WORKLOAD ITSELF, bounded by PCG
+    iterations: assembly O-1 + expansion O-2 are timed whole; the PCG (block inverses, r0, the
+    iterations, the true residual) is timed at maxit = 1 and at maxit = 1 + k_sample, which gives
+    the per-iteration time; the step is assembly + PCG(1) + (I - 1) x per-iteration, with I the
+    oracle's own iteration count on this system (tools/oracle_1m.py's committed full solve; if it
+    is missing or stale the full solve runs here once).  Returns (ms, info dict)."""
     import oracle
-    from synth import make_slope, preset
-    P = make_slope(preset(n_sample, seed=seed))
-    t0 = time.perf_counter()
-    M = oracle.assemble(P)
-    M.full_csr()
-    d, it, rr, st = M.pcg(P.F, tol=1e-10, maxit=10000, precond="bj")
-    t1 = time.perf_counter()
+    oracle.build()
+    aff = os.sched_getaffinity(0)
+    core = sorted(aff)[0]
+    os.sched_setaffinity(0, {core})
+    try:
+        t0 = time.perf_counter()
+        M = oracle.assemble(P)
+        M.full_csr()
+        t1 = time.perf_counter()
+        M.pcg(P.F, tol=1e-300, maxit=1, precond="bj")
+        t2 = time.perf_counter()
+        M.pcg(P.F, tol=1e-300, maxit=1 + k_sample, precond="bj")
+        t3 = time.perf_counter()
+        iters, rec = oracle_iters_for(P)
+        src = "profiles/r02_oracle_1m.json (tools/oracle_1m.py: the oracle's full solve of this system)"
+        if iters is None:
+            _, iters, _, _ = M.pcg(P.F, tol=1e-10, maxit=10000, precond="bj")
+            src = "the oracle's full solve, run here"
+        if spmv_stats is not None:
+            x = np.random.default_rng(7).uniform(-1.0, 1.0, 6 * P.n)
+            one = []
+            for _ in range(3):
+                a = time.perf_counter(); M.spmv(x); one.append(time.perf_counter() - a)
+            spmv_stats["spmv_1_thread_ms"] = 1000.0 * statistics.median(one)
+    finally:
+        os.sched_setaffinity(0, aff)
     if spmv_stats is not None:
+        os.sched_setaffinity(0, aff)
         x = np.random.default_rng(7).uniform(-1.0, 1.0, 6 * P.n)
-        one, par, th = [], [], 1
+        par, th = [], 1
         for _ in range(3):
-            a = time.perf_counter(); M.spmv(x); one.append(time.perf_counter() - a)
             a = time.perf_counter(); _, th = M.spmv_par(x); par.append(time.perf_counter() - a)
-        spmv_stats.update({"spmv_1_thread_ms": 1000.0 * statistics.median(one),
-                           "spmv_all_cores_ms": 1000.0 * statistics.median(par), "all_cores_threads": th})
-    return t1 - t0, P.n, it
+        spmv_stats.update({"spmv_all_cores_ms": 1000.0 * statistics.median(par), "all_cores_threads": th})
+    per_it = (t3 - t2) / k_sample
+    ms = 1000.0 * ((t1 - t0) + (t2 - t1) + (iters - 1) * per_it)
+    info = {"assemble_expand_ms": 1000.0 * (t1 - t0), "pcg_1_iter_ms": 1000.0 * (t2 - t1),
+            "per_iter_ms": 1000.0 * per_it, "iters": iters, "iters_source": src, "k_sample": k_sample,
+            "measured_s": t3 - t0, "pinned_core": core, "cpu_model": cpu_model()}
+    return ms, info
+
+
+def oracle_sample_text(P, info):
+    return (f"the oracle on the workload itself ({P.n} blocks), one pinned core ({info['cpu_model']}): "
+            f"assembly+expansion {info['assemble_expand_ms']:.0f} ms and BJ-PCG (block inverses, r0, 1 "
+            f"iteration, true residual) {info['pcg_1_iter_ms']:.0f} ms measured whole; PCG iterations "
+            f"measured over {info['k_sample']} ({info['per_iter_ms']:.1f} ms each) and counted at the "
+            f"oracle's own {info['iters']} iterations to 1e-10 ({info['iters_source']}); no block-count "
+            f"scaling; {info['measured_s']:.1f} s of CPU time measured")
 
 
 def run_reference(args):
@@ -198,27 +260,23 @@ def run_reference(args):
     world, rank, _ = dist_env()
     if rank != 0:
         return
-    n_full = args.blocks
-    n_s = args.ref_sample_blocks
-    import oracle
-    oracle.build()
+    from synth import make_slope, preset
+    P = make_slope(preset(args.blocks, seed=1005))
     for _ in range(args.warmup):
-        oracle_step_sample(n_s)
-    times, its, ns = [], [], []
+        oracle_step_at_size(P, k_sample=2)
+    times, info = [], None
     for _ in range(args.steps):
-        s, n_act, it = oracle_step_sample(n_s)
-        times.append(s); its.append(it); ns.append(n_act)
-    n_act = ns[0]
-    scale = n_full / n_act
-    ms = 1000.0 * statistics.median(times) * scale
-    sample = (f"oracle full step (assembly+expansion, BJ inverses, PCG to 1e-10) on a {n_act}-block slope "
-              f"from the same recipe ({its[0]} iters), 1 thread, scaled x{scale:.2f} by block count to "
-              f"the {n_full}-block workload")
+        ms, info = oracle_step_at_size(P, k_sample=args.ref_iter_sample)
+        times.append(ms)
+    ms = statistics.median(times)
+    sample = oracle_sample_text(P, info)
     line = {"impl": "reference", "metric": METRIC, "value": ms, "unit": UNIT, "higher_is_better": False,
             "n_gpus": world, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-            "config": {"workload": workload_name(n_full)},
-            "cpu_baseline": {"value": ms, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+            "config": {"workload": workload_name(args.blocks), "n_blocks": P.n,
+                       "sample": f"PCG iterations sampled: {info['k_sample']} of {info['iters']} per step"},
+            "cpu_baseline": {"value": ms, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
+                             "cpu_model": info["cpu_model"]},
             "e2e": {"value": ms, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
@@ -241,8 +299,8 @@ def main():
     ap.add_argument("--spmv-reps", type=int, default=20)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--cpu-sample-blocks", type=int, default=65_536)
-    ap.add_argument("--ref-sample-blocks", type=int, default=16_384)
+    ap.add_argument("--cpu-iter-sample", type=int, default=8, help="oracle PCG iterations timed (cpu_baseline)")
+    ap.add_argument("--ref-iter-sample", type=int, default=4, help="oracle PCG iterations timed per reference step")
     ap.add_argument("--clock-period", type=float, default=0.05, help="NVML clock sampling period (s)")
     args = ap.parse_args()
     if args.warmup < 3:
@@ -385,18 +443,15 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         sst = {}
-        s, n_s, it_s = oracle_step_sample(args.cpu_sample_blocks, spmv_stats=sst)
-        scale = n / n_s
-        cpu = {"value": 1000.0 * s * scale, "unit": UNIT, "cores": 1, "kind": "oracle",
-               "sample": (f"oracle full step (assembly+expansion, BJ inverses, PCG to 1e-10: {it_s} iters) on a "
-                          f"{n_s}-block slope of the same recipe, 1 thread, {s:.1f} s, scaled x{scale:.2f} by "
-                          f"block count"), "host_cores": os.cpu_count(),
-               "spmv_oracle": {"one_thread_ms_scaled": sst.get("spmv_1_thread_ms", 0.0) * scale,
-                               "all_cores_ms_scaled": sst.get("spmv_all_cores_ms", 0.0) * scale,
+        ms_cpu, info = oracle_step_at_size(P, k_sample=args.cpu_iter_sample, spmv_stats=sst)
+        cpu = {"value": ms_cpu, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": oracle_sample_text(P, info),
+               "cpu_model": info["cpu_model"], "host_cores": os.cpu_count(),
+               "spmv_oracle": {"one_thread_ms": sst.get("spmv_1_thread_ms", 0.0),
+                               "all_cores_ms": sst.get("spmv_all_cores_ms", 0.0),
                                "all_cores_threads": sst.get("all_cores_threads", 1),
-                               "note": (f"one oracle SpMV (full scalar CSR, O-3) on the {n_s}-block sample, "
-                                        "1 thread and OpenMP all cores (labelled second number, SURVEY §8(d)), "
-                                        "scaled by block count; the GPU SpMV is the line's spmv.ms")}}
+                               "note": ("one oracle SpMV (full scalar CSR, O-3) on the workload, 1 pinned thread "
+                                        "and the OpenMP all-cores twin (labelled second number, SURVEY §8(d)); "
+                                        "the GPU SpMV is the line's spmv.ms")}}
 
     line = {
         "metric": METRIC, "value": ms_step, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -433,12 +488,14 @@ def run_dist(args, P, world, rank, local):
     import torch
     import torch.distributed as dist
     import paper_conf_ipps_xiaohmxw17_b200 as dda
-    from paper_conf_ipps_xiaohmxw17_b200.partition import row_bounds, local_from_slope
-
-    bounds = row_bounds(P.n, world)
-    lp = local_from_slope(P, bounds, rank)
+    bounds = dda.row_bounds(P.n, world)
+    r0, r1 = int(bounds[rank]), int(bounds[rank + 1])
+    n_own = r1 - r0
+    # every rank gets the global spring list; dda_build_matrix_dist selects the springs of its rows
     dev = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
-    t = {k: dev(getattr(lp, k)) for k in ("kdiag", "bi", "bj", "pen", "e", "g", "F")}
+    t = {k: dev(getattr(P, k)) for k in ("bi", "bj", "pen", "e", "g")}
+    t["kdiag"] = dev(P.kdiag[r0:r1])
+    t["F"] = dev(P.F[6 * r0:6 * r1])
     obj = [dda.Comm.unique_id() if rank == 0 else None]
     dist.broadcast_object_list(obj, src=0)
     comm = dda.Comm.nccl(world, rank, obj[0])
@@ -447,8 +504,7 @@ def run_dist(args, P, world, rank, local):
 
     def step(ev=None):
         if ev: ev[0].record(stream)
-        K = dda.build_matrix(t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
-        comm.attach(0, K, lp)
+        K = comm.build_matrix_dist(0, P.n, bounds, t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
         if ev: ev[1].record(stream)
         ds, it, rr, st = comm.pcg_solve([t["F"]], tol=1e-10, maxit=10000, precond=args.precond)
         if ev: ev[2].record(stream)
@@ -478,8 +534,9 @@ def run_dist(args, P, world, rank, local):
     assert status == dda.OK and rel_res <= 1.01e-10, (status, rel_res)
     # v3 (block-Jacobi): the scaled engine per rank, 300u + 448 algorithmic bytes per own row and
     # iteration as on one GPU; u over the rank's own rows
-    u = K.nnzb / max(lp.n_own, 1)
-    local_bytes = lp.n_own * (300.0 * u + 448.0) * iters
+    info = comm.info(0, nparts=world)
+    u = K.nnzb / max(n_own, 1)
+    local_bytes = n_own * (300.0 * u + 448.0) * iters
     ach = local_bytes / (pcg * 1e-3) / 1e9
     tt = torch.tensor([ms, pcg, asm], device="cuda")
     dist.all_reduce(tt, op=dist.ReduceOp.MAX)
@@ -488,14 +545,15 @@ def run_dist(args, P, world, rank, local):
     e2e = None
     if not args.no_e2e:
         pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
-        h = {k: pin(getattr(lp, k)) for k in ("kdiag", "bi", "bj", "pen", "e", "g", "F")}
-        hd = torch.empty(6 * lp.n_own, dtype=torch.float64).pin_memory()
+        h = {k: pin(getattr(P, k)) for k in ("bi", "bj", "pen", "e", "g")}
+        h["kdiag"] = pin(P.kdiag[r0:r1])
+        h["F"] = pin(P.F[6 * r0:6 * r1])
+        hd = torch.empty(6 * n_own, dtype=torch.float64).pin_memory()
         a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         dist.barrier()
         a0.record(stream)
         dd = {k: v.cuda(non_blocking=True) for k, v in h.items()}
-        K2 = dda.build_matrix(dd["kdiag"], dd["bi"], dd["bj"], dd["pen"], dd["e"], dd["g"])
-        comm.attach(0, K2, lp)
+        K2 = comm.build_matrix_dist(0, P.n, bounds, dd["kdiag"], dd["bi"], dd["bj"], dd["pen"], dd["e"], dd["g"])
         ds, _, _, _ = comm.pcg_solve([dd["F"]], tol=1e-10, precond=args.precond)
         hd.copy_(ds[0], non_blocking=True)
         a1.record(stream)
@@ -505,7 +563,8 @@ def run_dist(args, P, world, rank, local):
         h2d = sum(v.numel() * v.element_size() for v in h.values())
         e2e = {"value": float(e2.item()), "unit": UNIT, "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": int(hd.numel() * 8),
-               "api": "dda_build_matrix + dda_dist_attach + dda_pcg_solve_dist (per-rank pinned host inputs)"}
+               "api": "dda_build_matrix_dist + dda_pcg_solve_dist (per-rank pinned host inputs: the global springs, "
+                      "own diagonal terms and F)"}
     if rank == 0:
         line = {
             "metric": METRIC, "value": ms, "unit": UNIT, "n_gpus": world, "steps": args.steps,
@@ -514,8 +573,9 @@ def run_dist(args, P, world, rank, local):
             "config": {"workload": workload_name(args.blocks), "n_blocks": P.n, "dof": 6 * P.n, "springs": P.m,
                        "precond": args.precond, "tol": 1e-10, "start": "cold (d0 = 0)",
                        "parallelism": f"block-row partition over {world} ranks (NCCL halo + allreduce)",
-                       "rank0_rows": lp.n_own, "rank0_halo": lp.n_halo,
-                       "step": "local dda_build_matrix + dda_dist_attach + dda_pcg_solve_dist",
+                       "rank0_rows": n_own, "rank0_halo": info["n_halo"],
+                       "step": "dda_build_matrix_dist (select + renumber + assemble + plan, device) + "
+                               "dda_pcg_solve_dist",
                        "l2": "inputs larger than L2 per rank at 1M/N; no flush"},
             "phases_ms": {"assemble_max": asm_max, "pcg_max": pcg_max, "pcg_iters": iters,
                           "pcg_us_per_iter": 1000.0 * pcg_max / max(iters, 1), "true_rel_res": rel_res},

@@ -118,8 +118,9 @@ def test_invalid_input(dda, bad):
     assert ei.value.status == dda.ERR_ARG
 
 
-def test_update_values_matches_fresh_build(dda):
-    P, _ = case("tiny")
+@pytest.mark.parametrize("name", ["tiny", "paper"])
+def test_update_values_matches_fresh_build(dda, name):
+    P, _ = case(name)
     t = dda.problem_to_device(P)
     K = dda.build_matrix(t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
     rng = np.random.default_rng(5)
@@ -182,8 +183,9 @@ def test_spmv_deterministic(dda):
 
 # ------------------------------------------------------------------ A3 / A7 preconditioners
 
-def test_bj_inverse(dda):
-    P, O = case("tiny")
+@pytest.mark.parametrize("name", ["tiny", "paper"])
+def test_bj_inverse(dda, name):
+    P, O = case(name)
     K = dda.build_from_problem(P)
     dinv = K.bj_setup(full=True).cpu().numpy()
     ref = O.bj_inv()
