@@ -200,7 +200,8 @@ dda_status_t dda_solve_host(int32_t n_blocks, const double *kdiag, int64_t n_spr
  * global rows, same order) followed by halo rows grouped by owning peer
  * (ascending peer, global order within a peer); it is assembled from every
  * spring that touches an own row, so its own rows are exact global rows.
- * (paper_conf_ipps_xiaohmxw17_b200/partition.py builds these inputs.)
+ * dda_build_matrix_dist (below) builds a partition and attaches it in one call; dda_dist_attach
+ * takes a partition built elsewhere.
  *
  * Transports: NCCL (dda_comm_init: one partition per process / GPU; rank 0
  * creates the 128-byte id with dda_comm_unique_id and the caller broadcasts it)
@@ -232,6 +233,40 @@ dda_status_t dda_comm_init_loopback(int32_t nparts, dda_comm_t *out);
 dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t K, int32_t n_own, const int32_t *send_counts,
                              const int32_t *send_idx, const int32_t *recv_counts, void *stream);
 dda_status_t dda_spmv_dist(dda_comm_t c, const double *const *x_own, double *const *y_own, void *stream);
+
+/*
+ * dda_build_matrix_dist — the partition-local assembly on the device (§8(b); A1 per partition,
+ * P:100-110, with P:104's "a contact contributes to rows i and j" deciding which springs a
+ * partition needs).  Partition `part` (0 for NCCL, 0..nparts-1 for loopback) owns the global
+ * block rows [row_bounds[me], row_bounds[me+1]) with me = its partition index (the NCCL rank, or
+ * `part`).  The call:
+ *   1. selects, in spring order, the springs with an endpoint in the own range;
+ *   2. forms the halo = their remote endpoints, sorted and unique (ascending global id, hence
+ *      grouped by owning partition);
+ *   3. numbers own row g as g - row_bounds[me] and halo row h as n_own + (rank of h in the halo);
+ *   4. assembles the local matrix with dda_build_matrix (halo rows get zero diagonal terms; the
+ *      own rows are then bit-identical to the global rows);
+ *   5. derives the exchange plan (the own rows each peer needs, ascending; the halo rows each
+ *      peer sends) and attaches matrix and plan to the communicator (dda_dist_attach).
+ *  n_global     global block count; row_bounds: host [nparts+1], 0 = b_0 < b_1 < ... = n_global,
+ *               identical on every partition
+ *  kdiag_own    device [n_own][6][6] diagonal terms of the own rows (global rows b_me..b_me+1-1)
+ *  n_springs, bi, bj, pen, e, g   device, GLOBAL block ids: the whole spring list, or any list
+ *               that contains every spring touching an own row (others are skipped)
+ *  out          receives the local matrix (caller-owned: dda_matrix_free after the last
+ *               distributed call that uses it; re-building a partition re-attaches)
+ * F / d of the partition are the global vectors' own-row slices [6 b_me, 6 b_me+1).  Errors:
+ * DDA_ERR_ARG for a bad partition index or bounds, ids out of [0, n_global) or bi == bj (checked
+ * on the device), or anything dda_build_matrix rejects.  Synchronising (sizes are read back).
+ * dda_dist_info reports a partition's n_own, n_halo and exchange plan (host arrays [nparts],
+ * send_idx [sum send_counts]; any may be NULL).
+ */
+dda_status_t dda_build_matrix_dist(dda_comm_t c, int32_t part, int32_t n_global, const int32_t *row_bounds,
+                                   const double *kdiag_own, int64_t n_springs, const int32_t *bi, const int32_t *bj,
+                                   const double *pen, const double *e, const double *g, void *stream,
+                                   dda_matrix_t *out);
+dda_status_t dda_dist_info(dda_comm_t c, int32_t part, int32_t *n_own, int32_t *n_halo, int32_t *send_counts,
+                           int32_t *recv_counts, int32_t *send_idx);
 dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double *const *F, const double *const *d0, double *const *d,
                                 double tol, int32_t maxit, dda_precond_t pc, int32_t *iters, double *rel_res,
                                 void *stream);
@@ -285,7 +320,72 @@ dda_status_t dda_contacts_export(dda_contacts_t C, int32_t *i, int32_t *v, int32
  */
 dda_status_t dda_contact_springs(dda_contacts_t C, const double *cxy, double p_n, double shear_ratio,
                                  int32_t *bi, int32_t *bj, double *pen, double *e, double *g, void *stream);
+/*
+ * Second classification (§III.A; §III.B): the angle judgment and the VV1 / VV2 split
+ * (reading N3-2; the oracle's O-10).  For record (vertex P = v of block i, edge
+ * Q1 -> Q2 of block j) with a = P_prev - P, b = P_next - P (P's two edges), d = Q2 - Q1,
+ * N = (d.y, -d.x) and s2 = sin_tol^2:
+ *     keep iff  a.x b.y - a.y b.x < 0  (P convex)  and, for x in {a, b},
+ *               N.x >= 0 or (N.x)^2 <= (s2 |N|^2) |x|^2   (no edge of P enters e's inner side by
+ *                                                          more than asin(sin_tol))
+ *     a kept VE record stays VE (class 0); a kept VV record is VV1 (class 1) if d is parallel to
+ *     a or b within the tolerance ((d x a)^2 <= (s2 |d|^2) |a|^2, or with b), else VV2 (class 2).
+ * Every product and sum is rounded as written.  The kept records are then stored class by class
+ * (VE, VV1, VV2; increasing (v, e) within a class) by a stable radix sort on the class: the set is
+ * replaced in place, `type` of dda_contacts_export becomes the class, dda_contacts_info's count and
+ * n_ve the kept records, and dda_contact_springs then emits a normal and a shear spring for EVERY
+ * record (VV1 / VV2 at the record's edge with t = 0 or 1), 2 * count springs.  sin_tol in [0, 1);
+ * a set can be classified once (DDA_ERR_ARG otherwise).  Synchronising (class counts are read
+ * back).  dda_contacts_classes reports the class counts and whether the set is classified.
+ */
+dda_status_t dda_classify_contacts(dda_contacts_t C, double sin_tol, void *stream);
+dda_status_t dda_contacts_classes(dda_contacts_t C, int64_t *n_ve, int64_t *n_vv1, int64_t *n_vv2,
+                                  int32_t *classified);
 void dda_contacts_free(dda_contacts_t C);
+
+/*
+ * NEXT-4 — interpenetration check and open-close state switch (§III.A, third classification:
+ * the switch integers p1, p2 and the categories C1-C5; §III.D, branch-restructured
+ * kernels; P:27 loop 3).  Reading N4 (the oracle's O-11 / O-12).  The contacts are
+ * the records of a CLASSIFIED set (dda_classify_contacts); contact k owns springs 2k (normal,
+ * e_n, g_n) and 2k+1 (shear) of dda_contact_springs, passed back as e, g (device [2 count][6]).
+ * States (device int32 [count]): 0 open, 1 slide, 2 lock.
+ *
+ * dda_contact_init: the signed gaps dn0 = n.(P - Q1) of every record (n the outward unit normal
+ *   of its edge) and the contact endpoints sorted by block (cached in C); if state != NULL, the
+ *   initial states: lock if dn0 <= 0 (touching / penetrating), else open.  Stream-ordered.
+ * dda_contact_loads: out (device [6n]) = F (device [6n], or NULL for 0) + the gap load of the
+ *   closed normal springs, F_i += f e_n, F_j += f g_n with f = -(pen[2k] dn0_k), summed per block in
+ *   contact order (deterministic; pen device [2 count]).  Stream-ordered.
+ * dda_contact_check: for the solution d (device [6n]):
+ *     un = e_n.d_i + g_n.d_j, us = e_s.d_i + g_s.d_j, dn = dn0 + un,
+ *     closed' = dn <= (closed ? open_tol : 0), lock' = closed' and not (p_s |us| > tan_phi (-p_n dn))
+ *     p1 = closed' - closed, p2 = lock' - lock;
+ *     VE / VV1: C1 p1 != 0; C2 p1 == 0 & p2 != 0; C3 p1 == p2 == 0 & closed'.
+ *     VV2: C4 p1 != 0; C5 p1 == 0 & p2 != 0.  Otherwise category 0.
+ *   state is updated in place; pen (device [2 count]) receives the next assembly's penalties
+ *   (normal p_n if closed', shear shear_ratio p_n if lock', else 0); cat (device [count], may be
+ *   NULL) the categories; cat_order (device [count], may be NULL) the contact ids grouped by
+ *   category (stable); counts (host [6]) the number per category 0..5.  Products and sums are
+ *   rounded as written, so states are bit-identical to the oracle's for the same d.  Synchronising.
+ * dda_open_close: loop 3 — with the penalties of `state`: dda_update_values(K, kdiag, pen, e, g);
+ *   F_eff = F + gap load; dda_pcg_solve(K, F_eff, d0 = d, d) with block-Jacobi (warm start);
+ *   dda_contact_check; until no contact switches (no C1, C2, C4, C5) or max_oc iterations.  K must
+ *   have been built from this set's springs (K's n = the contacts' n, 2 count springs); d (device
+ *   [6n]) is the warm start in and the solution out; state in/out; pen out.  oc_iters, pcg_iters
+ *   (total), converged (1 / 0) and rel_res (last solve) are host outputs.  DDA_ERR_ARG for a set
+ *   that is not classified and initialised (dda_contact_init).  Synchronising.
+ */
+dda_status_t dda_contact_init(dda_contacts_t C, int32_t *state, void *stream);
+dda_status_t dda_contact_loads(dda_contacts_t C, const double *e, const double *g, const double *pen, const double *F,
+                               double *out, void *stream);
+dda_status_t dda_contact_check(dda_contacts_t C, const double *d, const double *e, const double *g, double p_n,
+                               double shear_ratio, double tan_phi, double open_tol, int32_t *state, double *pen,
+                               int32_t *cat, int32_t *cat_order, int64_t *counts, void *stream);
+dda_status_t dda_open_close(dda_matrix_t K, dda_contacts_t C, const double *kdiag, const double *F, const double *e,
+                            const double *g, double p_n, double shear_ratio, double tan_phi, double open_tol,
+                            double tol, int32_t maxit, int32_t max_oc, int32_t *state, double *pen, double *d,
+                            int32_t *oc_iters, int32_t *pcg_iters, int32_t *converged, double *rel_res, void *stream);
 
 /* Number of kernel launches the library has issued in this process (for the
  * benchmark's gpu_launches count). */

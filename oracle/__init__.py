@@ -69,6 +69,10 @@ def lib():
         L.orc_contact_springs.argtypes = [C.c_int32, P, P, P, C.c_int64, P, P, P, P, P, P, C.c_double,
                                           C.c_double, P, P, P, P, P]
         L.orc_contact_springs.restype = C.c_int64
+        L.orc_classify_contacts.argtypes = [C.c_int32, P, P, C.c_int64, P, P, P, P, P, C.c_double, P]
+        L.orc_contact_loads.argtypes = [C.c_int32, P, P, C.c_int64, P, P, P, P, P, P, P, P, P]
+        L.orc_contact_check.argtypes = [C.c_int32, P, P, C.c_int64, P, P, P, P, P, P, P, P, C.c_double,
+                                        C.c_double, C.c_double, C.c_double, P, P, P]
         _lib = L
     return _lib
 
@@ -268,3 +272,123 @@ def contact_springs(vptr, vxy, cxy, C_, p_n, shear_ratio) -> dict:
                                     _p(o["e"]), _p(o["g"]))
     assert got == m
     return {k: a[:m] for k, a in o.items()}
+
+
+CLASS_NAMES = {-1: "abandoned", 0: "VE", 1: "VV1", 2: "VV2"}
+
+
+def classify_contacts(vptr, vxy, C_, sin_tol) -> np.ndarray:
+    """O-10: the angle judgment and the VV1 / VV2 split of every record of O-8: class -1
+    (abandoned), 0 (VE), 1 (VV1), 2 (VV2), per record."""
+    vptr = np.ascontiguousarray(vptr, np.int32)
+    vxy = np.ascontiguousarray(vxy, np.float64).reshape(-1, 2)
+    nc = int(C_["i"].shape[0])
+    cls = np.empty(max(nc, 1), np.int32)
+    f = [np.ascontiguousarray(C_[k], np.int32) for k in ("i", "v", "j", "e", "type")]
+    st = lib().orc_classify_contacts(vptr.shape[0] - 1, _p(vptr), _p(vxy), nc, *[_p(a) for a in f],
+                                     float(sin_tol), _p(cls))
+    if st != OK:
+        raise OracleError(st, "classify_contacts")
+    return cls[:nc]
+
+
+def classified_contacts(vptr, vxy, C_, sin_tol) -> dict:
+    """The classified contact set ("valid data will be stored in a successive array"): the
+    records that pass the angle judgment, grouped by class (VE, VV1, VV2; stable, so increasing
+    (v, e) within a class), with `type` = the class."""
+    cls = classify_contacts(vptr, vxy, C_, sin_tol)
+    keep = np.nonzero(cls >= 0)[0]
+    order = keep[np.argsort(cls[keep], kind="stable")]
+    out = {k: np.ascontiguousarray(C_[k][order]) for k in CONTACT_FIELDS}
+    out["type"] = cls[order].astype(np.int32)
+    return out
+
+
+def classified_springs(vptr, vxy, cxy, Cc, p_n, shear_ratio) -> dict:
+    """O-9 applied to EVERY record of a classified set (VE, VV1 and VV2 alike: normal + shear
+    spring at the record's edge and edge ratio, t = 0 or 1 for the VV classes), in record order."""
+    allve = dict(Cc)
+    allve["type"] = np.zeros_like(Cc["type"])
+    return contact_springs(vptr, vxy, cxy, allve, p_n, shear_ratio)
+
+
+STATE_NAMES = {0: "open", 1: "slide", 2: "lock"}
+
+
+def contact_check(vptr, vxy, Cc, d, e, g, p_n, shear_ratio, tan_phi, open_tol, state):
+    """O-11: one interpenetration check / open-close switch over a classified set Cc whose springs
+    (e, g: [2 count, 6], O-9 order) were formed for it.  Returns (new state, category 0..5 per
+    contact, penalties [2 count] for the next assembly); `state` is not modified."""
+    vptr = np.ascontiguousarray(vptr, np.int32)
+    vxy = np.ascontiguousarray(vxy, np.float64).reshape(-1, 2)
+    nc = int(Cc["i"].shape[0])
+    st = np.array(state, np.int32, copy=True).reshape(-1)
+    assert st.shape[0] == nc
+    pen = np.empty(max(2 * nc, 1))
+    cat = np.empty(max(nc, 1), np.int32)
+    f = [np.ascontiguousarray(Cc[k], np.int32) for k in ("i", "v", "j", "e", "type")]
+    dd = np.ascontiguousarray(d, np.float64)
+    ee = np.ascontiguousarray(e, np.float64).reshape(-1, 6)
+    gg = np.ascontiguousarray(g, np.float64).reshape(-1, 6)
+    assert ee.shape[0] == 2 * nc and gg.shape[0] == 2 * nc
+    r = lib().orc_contact_check(vptr.shape[0] - 1, _p(vptr), _p(vxy), nc, *[_p(a) for a in f], _p(dd), _p(ee),
+                                _p(gg), float(p_n), float(shear_ratio), float(tan_phi), float(open_tol), _p(st), _p(pen),
+                                _p(cat))
+    if r != OK:
+        raise OracleError(r, "contact_check")
+    return st[:nc], cat[:nc], pen[:2 * nc]
+
+
+def contact_loads(n, vptr, vxy, Cc, e, g, pen):
+    """O-12: the gap load Fc [6n] of the closed normal springs (pen [2 count]) and the initial states
+    (lock if the vertex touches or penetrates its edge, else open)."""
+    vptr = np.ascontiguousarray(vptr, np.int32)
+    vxy = np.ascontiguousarray(vxy, np.float64).reshape(-1, 2)
+    nc = int(Cc["i"].shape[0])
+    Fc = np.empty(6 * n)
+    st0 = np.empty(max(nc, 1), np.int32)
+    f = [np.ascontiguousarray(Cc[k], np.int32) for k in ("i", "v", "j", "e")]
+    ee = np.ascontiguousarray(e, np.float64).reshape(-1, 6)
+    gg = np.ascontiguousarray(g, np.float64).reshape(-1, 6)
+    pp = np.ascontiguousarray(pen, np.float64) if pen is not None else None
+    r = lib().orc_contact_loads(int(n), _p(vptr), _p(vxy), nc, *[_p(a) for a in f], _p(ee), _p(gg),
+                                _p(pp) if pp is not None else None, _p(Fc), _p(st0))
+    if r != OK:
+        raise OracleError(r, "contact_loads")
+    return Fc, st0[:nc]
+
+
+def state_penalties(state, p_n, shear_ratio):
+    """Spring penalties of contact states (reading N4): normal p_n if closed (slide / lock), shear
+    shear_ratio * p_n if lock, else 0 (the spring stays in the list with p = 0, reading Z10)."""
+    state = np.asarray(state)
+    pen = np.zeros(2 * state.size)
+    pen[0::2] = np.where(state >= 1, p_n, 0.0)
+    pen[1::2] = np.where(state == 2, shear_ratio * p_n, 0.0)
+    return pen
+
+
+def open_close_loop(n, kdiag, F, vptr, vxy, cxy, Cc, p_n, shear_ratio, tan_phi, open_tol, tol=1e-10, max_oc=30,
+                    precond="bj"):
+    """Loop 3 on the oracle, reading N4: initial states from the gaps (O-12); then repeat
+    { assemble K (O-1) with the penalties of the states; F_eff = F + gap load (O-12); solve (O-5)
+    warm-started from the previous solution; check (O-11) } until no contact changes state
+    (no C1, C2, C4, C5).  Returns (d, states, history [(pcg iters, category counts)], converged)."""
+    sp = classified_springs(vptr, vxy, cxy, Cc, p_n, shear_ratio)
+    _, state = contact_loads(n, vptr, vxy, Cc, sp["e"], sp["g"], None)
+    pen = state_penalties(state, p_n, shear_ratio)
+    d = np.zeros(6 * n)
+    hist = []
+    for _ in range(max_oc):
+        Fc, _ = contact_loads(n, vptr, vxy, Cc, sp["e"], sp["g"], pen)
+        M = OracleMatrix(n, kdiag, sp["bi"], sp["bj"], pen, sp["e"], sp["g"])
+        d, it, rr, st = M.pcg(F + Fc, d0=d, tol=tol, precond=precond)
+        if st != OK:
+            raise OracleError(st, "open_close_loop pcg")
+        state, cat, pen = contact_check(vptr, vxy, Cc, d, sp["e"], sp["g"], p_n, shear_ratio, tan_phi, open_tol,
+                                        state)
+        counts = np.bincount(cat, minlength=6)
+        hist.append((it, counts))
+        if counts[1] + counts[2] + counts[4] + counts[5] == 0:
+            return d, state, hist, True
+    return d, state, hist, False

@@ -743,3 +743,159 @@ int64_t orc_contact_springs(int32_t n, const int32_t *vptr, const double *vxy, c
     }
     return s;
 }
+
+/*
+ * O-10 (NEXT-3)  The angle judgment and the VV1 / VV2 split (§III.A, second
+ * classification: "some data of VE and VV are abandoned if they cannot fulfill the contact angle
+ * condition; the other data of VV will be divided into VV1 and VV2; the contacts with parallel
+ * edges are classified as VV1 or as VV2 otherwise"; §III.B).  The paper gives no formula; the
+ * reading (N3-2) after Shi's contact rules (external) is, for record k = (vertex P =
+ * v of block i, edge e = Q1 -> Q2 of block j), with P_prev / P_next the neighbours of v in block i:
+ *     a = P_prev - P,  b = P_next - P         (the two edges of block i at P, pointing away)
+ *     d = Q2 - Q1,     N = (d.y, -d.x)        (outward normal of the counter-clockwise edge)
+ *     s2 = sin_tol * sin_tol,  NN = N.N
+ *     convex:  a.x b.y - a.y b.x < 0          (P is a convex corner of block i)
+ *     out(x):  N.x >= 0  or  (N.x)^2 <= (s2 NN) |x|^2      (edge x of P does not point into the
+ *                                                          inner side of e by more than the
+ *                                                          tolerance angle asin(sin_tol))
+ * the record passes the angle judgment iff convex and out(a) and out(b); a passing VE record stays
+ * VE (class 0); a passing VV record is VV1 (class 1) if one of P's edges is parallel to e within
+ * the tolerance, (d x a)^2 <= (s2 NN) |a|^2 or (d x b)^2 <= (s2 NN) |b|^2, else VV2 (class 2);
+ * a failing record is abandoned (class -1).  Every product and sum is rounded as written.
+ */
+int orc_classify_contacts(int32_t n, const int32_t *vptr, const double *vxy, int64_t nc, const int32_t *ci,
+                          const int32_t *cv, const int32_t *cj, const int32_t *ce, const int32_t *ctype,
+                          double sin_tol, int32_t *cls) {
+    if (n <= 0 || !vptr || !vxy || !(sin_tol >= 0.0) || !(sin_tol < 1.0)) return ORC_ERR_ARG;
+    const double s2 = sin_tol * sin_tol;
+    for (int64_t k = 0; k < nc; ++k) {
+        const int32_t i = ci[k], v = cv[k], j = cj[k], q = ce[k];
+        const int32_t vp = (v > vptr[i]) ? v - 1 : vptr[i + 1] - 1;
+        const int32_t vn = (v + 1 < vptr[i + 1]) ? v + 1 : vptr[i];
+        const int32_t q2 = (q + 1 < vptr[j + 1]) ? q + 1 : vptr[j];
+        const double px = vxy[2 * v], py = vxy[2 * v + 1];
+        const double ax = vxy[2 * vp] - px, ay = vxy[2 * vp + 1] - py;
+        const double bx = vxy[2 * vn] - px, by = vxy[2 * vn + 1] - py;
+        const double dx = vxy[2 * q2] - vxy[2 * q], dy = vxy[2 * q2 + 1] - vxy[2 * q + 1];
+        const double Nx = dy, Ny = -dx;
+        const double NN = Nx * Nx + Ny * Ny;
+        const double aa = ax * ax + ay * ay, bb = bx * bx + by * by;
+        const double lim = s2 * NN;
+        const int convex = (ax * by - ay * bx) < 0.0;
+        const double fa = Nx * ax + Ny * ay, fb = Nx * bx + Ny * by;
+        const int out_a = fa >= 0.0 || fa * fa <= lim * aa;
+        const int out_b = fb >= 0.0 || fb * fb <= lim * bb;
+        if (!(convex && out_a && out_b)) {
+            cls[k] = -1;
+        } else if (ctype[k] == 0) {
+            cls[k] = 0;
+        } else {
+            const double xa = dx * ay - dy * ax, xb = dx * by - dy * bx;
+            const int par = xa * xa <= lim * aa || xb * xb <= lim * bb;
+            cls[k] = par ? 1 : 2;
+        }
+    }
+    return ORC_OK;
+}
+
+/* signed distance of record k's vertex from its edge line, n.(P - Q1), n = (u.y, -u.x), as O-11 */
+static double contact_gap(const int32_t *vptr, const double *vxy, int32_t v, int32_t j, int32_t q) {
+    const int32_t q2 = (q + 1 < vptr[j + 1]) ? q + 1 : vptr[j];
+    const double dx = vxy[2 * q2] - vxy[2 * q], dy = vxy[2 * q2 + 1] - vxy[2 * q + 1];
+    const double len = sqrt(dx * dx + dy * dy);
+    const double ux = dx / len, uy = dy / len;
+    const double nx = uy, ny = -ux;
+    return nx * (vxy[2 * v] - vxy[2 * q]) + ny * (vxy[2 * v + 1] - vxy[2 * q + 1]);
+}
+
+/*
+ * O-11 (NEXT-4)  Interpenetration check and open-close state switch of one open-close iteration
+ * (§III.A, third classification; §III.D; loop 3 of §I).  The paper
+ * names the switch integers p1, p2 in {-1, 0, 1} and the categories C1-C5 but gives no formulas;
+ * the reading (N4) after Shi's open-close rules (external):
+ * contact k is record k of a classified set (class 0 VE, 1 VV1, 2 VV2) whose springs are 2k (normal,
+ * vectors e_n, g_n) and 2k+1 (shear, e_s, g_s) of O-9; d is the solution of K d = F.  With u the
+ * unit tangent of the record's edge (u = d/|d|, as O-9) and n = (u.y, -u.x) its outward normal:
+ *     dn0 = n.x (P.x - Q1.x) + n.y (P.y - Q1.y)        signed distance of the vertex (> 0 outside)
+ *     un  = sum_r e_n[r] d_i[r] + sum_r g_n[r] d_j[r]   relative normal displacement (r = 0..5 in
+ *     us  = sum_r e_s[r] d_i[r] + sum_r g_s[r] d_j[r]   order, e before g, from +0.0)
+ *     dn  = dn0 + un
+ *     closed = dn <= (was closed ? open_tol : 0)  (an open contact closes when it touches; a closed
+ *              one opens only when its vertex separates by more than the tension tolerance)
+ *     fn = -p_n dn;   fs = (shear_ratio p_n) |us|
+ *     lock   = closed and not (fs > tan_phi fn)         (Mohr-Coulomb, no cohesion)
+ *     state' = 0 open / 1 slide / 2 lock;   p1 = closed' - closed;   p2 = lock' - lock
+ * Categories: VE and VV1: C1 |p1| > 0; C2 p1 = 0 and |p2| > 0; C3 p1 = p2 = 0 and closed'
+ * ("some other condition" read as: the contact stays in contact); VV2: C4 |p1| > 0; C5 p1 = 0 and
+ * |p2| > 0; otherwise 0 (abandoned: nothing to re-check).  Penalties of the next assembly: normal
+ * p_n if closed' else 0, shear shear_ratio p_n if lock' else 0 (an open contact keeps its springs
+ * with p = 0, reading Z10, so the spring list and the matrix structure do not change).
+ * state[k] is read (previous) and overwritten (new); cat[k] receives 0..5; pen [2 nc].
+ */
+int orc_contact_check(int32_t n, const int32_t *vptr, const double *vxy, int64_t nc, const int32_t *ci,
+                      const int32_t *cv, const int32_t *cj, const int32_t *ce, const int32_t *cls, const double *d,
+                      const double *e, const double *g, double p_n, double shear_ratio, double tan_phi,
+                      double open_tol, int32_t *state, double *pen, int32_t *cat) {
+    if (n <= 0 || !(p_n >= 0.0) || !(shear_ratio >= 0.0) || !(tan_phi >= 0.0) || !(open_tol >= 0.0))
+        return ORC_ERR_ARG;
+    const double ps = shear_ratio * p_n;
+    for (int64_t k = 0; k < nc; ++k) {
+        const int32_t i = ci[k], v = cv[k], j = cj[k], q = ce[k];
+        const double dn0 = contact_gap(vptr, vxy, v, j, q);
+        const double *en = e + 12 * k, *es = e + 12 * k + 6, *gn = g + 12 * k, *gs = g + 12 * k + 6;
+        double un = 0.0, us = 0.0;
+        for (int r = 0; r < 6; ++r) un = un + en[r] * d[6 * (int64_t)i + r];
+        for (int r = 0; r < 6; ++r) un = un + gn[r] * d[6 * (int64_t)j + r];
+        for (int r = 0; r < 6; ++r) us = us + es[r] * d[6 * (int64_t)i + r];
+        for (int r = 0; r < 6; ++r) us = us + gs[r] * d[6 * (int64_t)j + r];
+        const double dn = dn0 + un;
+        const int old = state[k];
+        const int closed = dn <= (old >= 1 ? open_tol : 0.0);
+        const double fn = -p_n * dn;
+        const double fs = ps * fabs(us);
+        const int lock = closed && !(fs > tan_phi * fn);
+        const int p1 = closed - (old >= 1);
+        const int p2 = lock - (old == 2);
+        int c = 0;
+        if (cls[k] == 2) {
+            if (p1 != 0) c = 4;
+            else if (p2 != 0) c = 5;
+        } else {
+            if (p1 != 0) c = 1;
+            else if (p2 != 0) c = 2;
+            else if (closed) c = 3;
+        }
+        cat[k] = c;
+        state[k] = closed ? (lock ? 2 : 1) : 0;
+        pen[2 * k] = closed ? p_n : 0.0;
+        pen[2 * k + 1] = lock ? ps : 0.0;
+    }
+    return ORC_OK;
+}
+
+/*
+ * O-12 (NEXT-4)  Contact initialisation and the gap load of the open-close loop (reading N4).
+ * The normal spring of a closed contact stores the energy p_n (dn0 + un)^2 / 2 (un = e_n.d_i +
+ * g_n.d_j, dn0 = the signed gap of O-11): its stiffness p_n [e_n; g_n][e_n; g_n]^T is assembled by
+ * O-1 from the spring list, and its load is
+ *     F_i += f e_n,   F_j += f g_n,    f = -(pen[2k] * dn0_k)
+ * summed into Fc (zeroed here) for k = 0, 1, ... in that order, each product f * e[r] rounded and
+ * then added (Fc[b] is the plain sequential sum over the contacts touching b, in contact order).
+ * Initial states (when state0 != NULL): lock (2) if dn0 <= 0 (touching or penetrating), else open.
+ */
+int orc_contact_loads(int32_t n, const int32_t *vptr, const double *vxy, int64_t nc, const int32_t *ci,
+                      const int32_t *cv, const int32_t *cj, const int32_t *ce, const double *e, const double *g,
+                      const double *pen, double *Fc, int32_t *state0) {
+    if (n <= 0) return ORC_ERR_ARG;
+    for (int64_t t = 0; t < 6 * (int64_t)n; ++t) Fc[t] = 0.0;
+    for (int64_t k = 0; k < nc; ++k) {
+        const double dn0 = contact_gap(vptr, vxy, cv[k], cj[k], ce[k]);
+        if (state0) state0[k] = dn0 <= 0.0 ? 2 : 0;
+        if (!pen) continue;
+        const double f = -(pen[2 * k] * dn0);
+        const int64_t i = ci[k], j = cj[k];
+        for (int r = 0; r < 6; ++r) Fc[6 * i + r] = Fc[6 * i + r] + f * e[12 * k + r];
+        for (int r = 0; r < 6; ++r) Fc[6 * j + r] = Fc[6 * j + r] + f * g[12 * k + r];
+    }
+    return ORC_OK;
+}

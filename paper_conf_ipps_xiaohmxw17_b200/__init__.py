@@ -29,7 +29,9 @@ ABI_SYMBOLS = ("dda_build_matrix", "dda_update_values", "dda_matrix_info", "dda_
                "dda_comm_init", "dda_comm_init_loopback", "dda_dist_attach", "dda_spmv_dist",
                "dda_pcg_solve_dist", "dda_comm_free", "dda_spmv_full", "dda_rcm_order",
                "dda_memory_release", "dda_memory_cached", "dda_detect_contacts", "dda_contacts_info",
-               "dda_contacts_export", "dda_contact_springs", "dda_contacts_free")
+               "dda_contacts_export", "dda_contact_springs", "dda_contacts_free", "dda_build_matrix_dist",
+               "dda_dist_info", "dda_classify_contacts", "dda_contacts_classes",
+               "dda_contact_init", "dda_contact_loads", "dda_contact_check", "dda_open_close")
 
 _lib = None
 
@@ -110,6 +112,22 @@ def lib() -> C.CDLL:
         L.dda_contact_springs.restype = st
         L.dda_contacts_free.argtypes = [P]
         L.dda_contacts_free.restype = None
+        L.dda_build_matrix_dist.argtypes = [P, I32, I32, P, P, I64, P, P, P, P, P, P, C.POINTER(P)]
+        L.dda_build_matrix_dist.restype = st
+        L.dda_dist_info.argtypes = [P, I32, P, P, P, P, P]
+        L.dda_dist_info.restype = st
+        L.dda_classify_contacts.argtypes = [P, D, P]
+        L.dda_classify_contacts.restype = st
+        L.dda_contacts_classes.argtypes = [P, P, P, P, P]
+        L.dda_contacts_classes.restype = st
+        L.dda_contact_init.argtypes = [P, P, P]
+        L.dda_contact_init.restype = st
+        L.dda_contact_loads.argtypes = [P, P, P, P, P, P, P]
+        L.dda_contact_loads.restype = st
+        L.dda_contact_check.argtypes = [P, P, P, P, D, D, D, D, P, P, P, P, P, P]
+        L.dda_contact_check.restype = st
+        L.dda_open_close.argtypes = [P, P, P, P, P, P, D, D, D, D, D, I32, I32, P, P, P, P, P, P, P, P]
+        L.dda_open_close.restype = st
         L.dda__last_checks.argtypes = [P]
         L.dda__last_checks.restype = C.c_int
         L.dda__pcg_engine.argtypes = [P, C.c_int]
@@ -360,6 +378,41 @@ class Comm:
                                      C.c_void_p(_stream(stream))), "dda_dist_attach")
         self.parts[part if self.nparts_local > 1 else 0] = (K, lp)
 
+    def build_matrix_dist(self, part: int, n_global: int, bounds, kdiag_own, bi, bj, pen, e, g,
+                          stream=None) -> "Matrix":
+        """dda_build_matrix_dist: select this partition's springs (global ids, CUDA tensors), renumber,
+        assemble and attach with the exchange plan, all in the library.  bounds: [nparts+1] row
+        bounds (host); kdiag_own: [n_own, 6, 6] CUDA float64."""
+        torch = _torch()
+        m = int(bi.shape[0])
+        b = np.ascontiguousarray(bounds, np.int32)
+        me = part if (self.nparts_local > 1 and 0 <= part < b.shape[0] - 1) else None
+        n_own = None if me is None else int(b[me + 1] - b[me])
+        h = C.c_void_p()
+        _check(lib().dda_build_matrix_dist(
+            self._h, int(part), int(n_global), b.ctypes.data_as(C.c_void_p),
+            _dev(kdiag_own, torch.float64, (n_own, 6, 6) if n_own is not None else None, "kdiag_own"), m,
+            _dev(bi, torch.int32, (m,), "bi"), _dev(bj, torch.int32, (m,), "bj"),
+            _dev(pen, torch.float64, (m,), "pen"), _dev(e, torch.float64, (m, 6), "e"),
+            _dev(g, torch.float64, (m, 6), "g"), C.c_void_p(_stream(stream)), C.byref(h)), "dda_build_matrix_dist")
+        K = Matrix(h)
+        self.parts[part if self.nparts_local > 1 else 0] = (K, None)
+        return K
+
+    def info(self, part: int = 0, nparts: int = None) -> dict:
+        """dda_dist_info: n_own, n_halo and the exchange plan of an attached partition."""
+        P = nparts if nparts is not None else self.nparts_local
+        n_own, n_halo = C.c_int32(), C.c_int32()
+        sc, rc = np.zeros(P, np.int32), np.zeros(P, np.int32)
+        _check(lib().dda_dist_info(self._h, int(part), C.cast(C.byref(n_own), C.c_void_p),
+                                   C.cast(C.byref(n_halo), C.c_void_p), sc.ctypes.data_as(C.c_void_p),
+                                   rc.ctypes.data_as(C.c_void_p), None), "dda_dist_info")
+        si = np.zeros(max(int(sc.sum()), 1), np.int32)
+        _check(lib().dda_dist_info(self._h, int(part), None, None, None, None, si.ctypes.data_as(C.c_void_p)),
+               "dda_dist_info")
+        return {"n_own": int(n_own.value), "n_halo": int(n_halo.value), "send_counts": sc, "recv_counts": rc,
+                "send_idx": si[:int(sc.sum())]}
+
     @staticmethod
     def _ptrs(ts):
         arr = (C.c_void_p * len(ts))(*[C.c_void_p(t.data_ptr()) if t is not None else None for t in ts])
@@ -393,6 +446,13 @@ class Comm:
             self.free()
         except Exception:
             pass
+
+
+def row_bounds(n: int, nparts: int) -> np.ndarray:
+    """Contiguous block-row ranges [b[p], b[p+1]) of equal size (int32, for dda_build_matrix_dist)."""
+    if nparts < 1 or n < nparts:
+        raise ValueError("need 1 <= nparts <= n")
+    return np.array([(p * n) // nparts for p in range(nparts + 1)], dtype=np.int32)
 
 
 def build_local(lp, device="cuda") -> Matrix:
@@ -438,6 +498,74 @@ class Contacts:
         cnt, nve, npr = C.c_int64(), C.c_int64(), C.c_int64()
         _check(lib().dda_contacts_info(self._h, C.byref(cnt), C.byref(nve), C.byref(npr)), "dda_contacts_info")
         self.count, self.n_ve, self.n_pairs = int(cnt.value), int(nve.value), int(npr.value)
+        self.classified, self.n_vv1, self.n_vv2 = False, 0, 0
+
+    def classify(self, sin_tol=0.35, stream=None):
+        """dda_classify_contacts: angle judgment + VV1 / VV2 split; the set becomes the kept records
+        grouped by class (type = 0 VE, 1 VV1, 2 VV2)."""
+        _check(lib().dda_classify_contacts(self._h, C.c_double(sin_tol), C.c_void_p(_stream(stream))),
+               "dda_classify_contacts")
+        cnt, nve, npr = C.c_int64(), C.c_int64(), C.c_int64()
+        _check(lib().dda_contacts_info(self._h, C.byref(cnt), C.byref(nve), C.byref(npr)), "dda_contacts_info")
+        v1, v2, cl = C.c_int64(), C.c_int64(), C.c_int32()
+        ref = lambda x: C.cast(C.byref(x), C.c_void_p)
+        _check(lib().dda_contacts_classes(self._h, None, ref(v1), ref(v2), ref(cl)), "dda_contacts_classes")
+        self.count, self.n_ve = int(cnt.value), int(nve.value)
+        self.classified, self.n_vv1, self.n_vv2 = bool(cl.value), int(v1.value), int(v2.value)
+        return self
+
+    # ---- NEXT-4: interpenetration check / open-close switch (dda_contact_*)
+    def init_states(self, stream=None):
+        """dda_contact_init: gaps + endpoint sort; returns the initial states (CUDA int32 [count])."""
+        torch = _torch()
+        state = torch.empty(max(self.count, 1), dtype=torch.int32, device="cuda")
+        _check(lib().dda_contact_init(self._h, C.c_void_p(state.data_ptr()), C.c_void_p(_stream(stream))),
+               "dda_contact_init")
+        return state[:self.count]
+
+    def loads(self, sp, pen, F=None, stream=None):
+        """dda_contact_loads: F (or 0) + the gap load of the closed normal springs (CUDA [6n])."""
+        torch = _torch()
+        n = self._keep[0].shape[0] - 1
+        out = torch.empty(6 * n, dtype=torch.float64, device="cuda")
+        _check(lib().dda_contact_loads(self._h, C.c_void_p(sp["e"].data_ptr()), C.c_void_p(sp["g"].data_ptr()),
+                                       C.c_void_p(pen.data_ptr()), C.c_void_p(F.data_ptr()) if F is not None else None,
+                                       C.c_void_p(out.data_ptr()), C.c_void_p(_stream(stream))), "dda_contact_loads")
+        return out
+
+    def check(self, d, sp, state, p_n=40.0, shear_ratio=0.4, tan_phi=0.577, open_tol=0.01, stream=None):
+        """dda_contact_check: updates `state` in place; returns (pen, cat, cat_order, counts[6])."""
+        torch = _torch()
+        m = max(self.count, 1)
+        pen = torch.empty(2 * m, dtype=torch.float64, device="cuda")
+        cat = torch.empty(m, dtype=torch.int32, device="cuda")
+        order = torch.empty(m, dtype=torch.int32, device="cuda")
+        counts = np.zeros(6, np.int64)
+        _check(lib().dda_contact_check(self._h, C.c_void_p(d.data_ptr()), C.c_void_p(sp["e"].data_ptr()),
+                                       C.c_void_p(sp["g"].data_ptr()), float(p_n), float(shear_ratio), float(tan_phi),
+                                       float(open_tol), C.c_void_p(state.data_ptr()), C.c_void_p(pen.data_ptr()),
+                                       C.c_void_p(cat.data_ptr()), C.c_void_p(order.data_ptr()),
+                                       counts.ctypes.data_as(C.c_void_p), C.c_void_p(_stream(stream))),
+               "dda_contact_check")
+        k = self.count
+        return pen[:2 * k], cat[:k], order[:k], counts
+
+    def open_close(self, K, kdiag, F, sp, state, d=None, p_n=40.0, shear_ratio=0.4, tan_phi=0.577, open_tol=0.01,
+                   tol=1e-10, maxit=10000, max_oc=30, stream=None):
+        """dda_open_close (loop 3): returns (d, state, pen, oc_iters, pcg_iters, converged, rel_res)."""
+        torch = _torch()
+        n = self._keep[0].shape[0] - 1
+        d = torch.zeros(6 * n, dtype=torch.float64, device="cuda") if d is None else d
+        pen = torch.empty(max(2 * self.count, 1), dtype=torch.float64, device="cuda")
+        oc, pit, conv, rr = C.c_int32(), C.c_int32(), C.c_int32(), C.c_double()
+        ref = lambda x: C.cast(C.byref(x), C.c_void_p)
+        _check(lib().dda_open_close(K.handle, self._h, C.c_void_p(kdiag.data_ptr()), C.c_void_p(F.data_ptr()),
+                                    C.c_void_p(sp["e"].data_ptr()), C.c_void_p(sp["g"].data_ptr()), float(p_n),
+                                    float(shear_ratio), float(tan_phi), float(open_tol), float(tol), int(maxit),
+                                    int(max_oc), C.c_void_p(state.data_ptr()), C.c_void_p(pen.data_ptr()),
+                                    C.c_void_p(d.data_ptr()), ref(oc), ref(pit), ref(conv), ref(rr),
+                                    C.c_void_p(_stream(stream))), "dda_open_close")
+        return d, state, pen[:2 * self.count], int(oc.value), int(pit.value), bool(conv.value), float(rr.value)
 
     def free(self):
         if self._h is not None:
@@ -464,7 +592,7 @@ class Contacts:
         """Springs of the VE contacts as CUDA tensors (bi, bj, pen, e, g) for build_matrix."""
         torch = _torch()
         n = self._keep[0].shape[0] - 1
-        m = 2 * self.n_ve
+        m = 2 * (self.count if self.classified else self.n_ve)
         dev = self._keep[1].device
         o = {"bi": torch.empty(m, dtype=torch.int32, device=dev), "bj": torch.empty(m, dtype=torch.int32, device=dev),
              "pen": torch.empty(m, dtype=torch.float64, device=dev),

@@ -31,16 +31,6 @@
 
 #include "dda_internal.cuh"
 
-struct dda_contacts {
-    int device = 0;
-    int32_t n = 0;
-    int64_t count = 0, n_ve = 0, n_pairs = 0;
-    const int32_t* vptr = nullptr;   // caller's geometry (must outlive dda_contact_springs)
-    const double* vxy = nullptr;
-    int32_t *ci = nullptr, *cv = nullptr, *cj = nullptr, *ce = nullptr, *ctype = nullptr;
-    double *ct = nullptr, *cd2 = nullptr;
-};
-
 namespace dda {
 namespace {
 
@@ -236,6 +226,68 @@ __global__ void k_isve(int64_t m, const int32_t* __restrict__ ctype, int32_t* __
         f[t] = ctype[t] == 0 ? 1 : 0;
 }
 
+// Angle judgment and VV1 / VV2 split (reading N3-2, the oracle's O-10): key = class + 1 (0 abandoned,
+// 1 VE, 2 VV1, 3 VV2), every product and sum rounded as written (__dmul_rn / __dadd_rn / __dsub_rn)
+__global__ void k_classify(int64_t m, const int32_t* __restrict__ vptr, const double* __restrict__ vxy,
+                           const int32_t* __restrict__ ci, const int32_t* __restrict__ cv,
+                           const int32_t* __restrict__ cj, const int32_t* __restrict__ ce,
+                           const int32_t* __restrict__ ctype, double s2, uint32_t* __restrict__ key,
+                           int32_t* __restrict__ idx) {
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < m; k += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t i = ci[k], v = cv[k], j = cj[k], q = ce[k];
+        const int32_t vp = (v > vptr[i]) ? v - 1 : vptr[i + 1] - 1;
+        const int32_t vn = (v + 1 < vptr[i + 1]) ? v + 1 : vptr[i];
+        const int32_t q2 = (q + 1 < vptr[j + 1]) ? q + 1 : vptr[j];
+        const double2 P = *reinterpret_cast<const double2*>(vxy + 2 * (size_t)v);
+        const double2 Pa = *reinterpret_cast<const double2*>(vxy + 2 * (size_t)vp);
+        const double2 Pb = *reinterpret_cast<const double2*>(vxy + 2 * (size_t)vn);
+        const double2 Q1 = *reinterpret_cast<const double2*>(vxy + 2 * (size_t)q);
+        const double2 Q2 = *reinterpret_cast<const double2*>(vxy + 2 * (size_t)q2);
+        const double ax = __dsub_rn(Pa.x, P.x), ay = __dsub_rn(Pa.y, P.y);
+        const double bx = __dsub_rn(Pb.x, P.x), by = __dsub_rn(Pb.y, P.y);
+        const double dx = __dsub_rn(Q2.x, Q1.x), dy = __dsub_rn(Q2.y, Q1.y);
+        const double Nx = dy, Ny = -dx;
+        const double NN = __dadd_rn(__dmul_rn(Nx, Nx), __dmul_rn(Ny, Ny));
+        const double aa = __dadd_rn(__dmul_rn(ax, ax), __dmul_rn(ay, ay));
+        const double bb = __dadd_rn(__dmul_rn(bx, bx), __dmul_rn(by, by));
+        const double lim = __dmul_rn(s2, NN);
+        const bool convex = __dsub_rn(__dmul_rn(ax, by), __dmul_rn(ay, bx)) < 0.0;
+        const double fa = __dadd_rn(__dmul_rn(Nx, ax), __dmul_rn(Ny, ay));
+        const double fb = __dadd_rn(__dmul_rn(Nx, bx), __dmul_rn(Ny, by));
+        const bool out_a = fa >= 0.0 || __dmul_rn(fa, fa) <= __dmul_rn(lim, aa);
+        const bool out_b = fb >= 0.0 || __dmul_rn(fb, fb) <= __dmul_rn(lim, bb);
+        uint32_t c;
+        if (!(convex && out_a && out_b)) {
+            c = 0;
+        } else if (ctype[k] == 0) {
+            c = 1;
+        } else {
+            const double xa = __dsub_rn(__dmul_rn(dx, ay), __dmul_rn(dy, ax));
+            const double xb = __dsub_rn(__dmul_rn(dx, by), __dmul_rn(dy, bx));
+            const bool par = __dmul_rn(xa, xa) <= __dmul_rn(lim, aa) || __dmul_rn(xb, xb) <= __dmul_rn(lim, bb);
+            c = par ? 2 : 3;
+        }
+        key[k] = c;
+        idx[k] = (int32_t)k;
+    }
+}
+
+// start[c] = first position of key c in the sorted keys (c = 0..3; start[4] = m), set by the heads
+__global__ void k_class_bounds(int64_t m, const uint32_t* __restrict__ skey, int64_t* __restrict__ start) {
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < m; t += (int64_t)gridDim.x * blockDim.x) {
+        const uint32_t c = skey[t];
+        const uint32_t p = t > 0 ? skey[t - 1] : 0u;
+        if (t == 0) for (uint32_t z = 0; z <= c; ++z) start[z] = 0;
+        else for (uint32_t z = p + 1; z <= c; ++z) start[z] = t;
+        if (t == m - 1) for (uint32_t z = c + 1; z <= 4; ++z) start[z] = m;
+    }
+}
+
+__global__ void k_class_type(int64_t m, const uint32_t* __restrict__ skey, int32_t* __restrict__ type) {
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < m; t += (int64_t)gridDim.x * blockDim.x)
+        type[t] = (int32_t)skey[t] - 1;
+}
+
 // T(P)^T u for Shi's first-order T at offset (x, y) from the centroid, rounded as the oracle writes it
 __device__ __forceinline__ void tt_times(double x, double y, double ux, double uy, double* o) {
     o[0] = ux;
@@ -252,9 +304,9 @@ __global__ void k_springs(int64_t m, const int32_t* __restrict__ slot, const int
                           const int32_t* __restrict__ cj, const int32_t* __restrict__ ce,
                           const int32_t* __restrict__ ctype, const double* __restrict__ ct, double p_n, double ps,
                           int32_t* __restrict__ bi, int32_t* __restrict__ bj, double* __restrict__ pen,
-                          double* __restrict__ e, double* __restrict__ g) {
+                          double* __restrict__ e, double* __restrict__ g, int all) {
     for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < m; k += (int64_t)gridDim.x * blockDim.x) {
-        if (ctype[k] != 0) continue;
+        if (!all && ctype[k] != 0) continue;
         const int32_t i = ci[k], j = cj[k], v = cv[k], q = ce[k];
         const int32_t q2 = (q + 1 < vptr[j + 1]) ? q + 1 : vptr[j];
         const double dx = __dsub_rn(vxy[2 * (size_t)q2], vxy[2 * (size_t)q]);
@@ -269,7 +321,7 @@ __global__ void k_springs(int64_t m, const int32_t* __restrict__ slot, const int
         const double q2x = __dsub_rn(vxy[2 * (size_t)q2], cxy[2 * (size_t)j]);
         const double q2y = __dsub_rn(vxy[2 * (size_t)q2 + 1], cxy[2 * (size_t)j + 1]);
         const double omt = __dsub_rn(1.0, t);
-        const int64_t s0 = 2 * (int64_t)slot[k];
+        const int64_t s0 = 2 * (all ? k : (int64_t)slot[k]);
 #pragma unroll
         for (int sp = 0; sp < 2; ++sp) {
             const double nx = sp == 0 ? uy : ux, ny = sp == 0 ? -ux : uy;
@@ -335,7 +387,7 @@ extern "C" void dda_contacts_free(dda_contacts_t C) {
     cudaGetDevice(&prev);
     cudaSetDevice(C->device);
     cudaDeviceSynchronize();
-    void* ptrs[] = {C->ci, C->cv, C->cj, C->ce, C->ctype, C->ct, C->cd2};
+    void* ptrs[] = {C->ci, C->cv, C->cj, C->ce, C->ctype, C->ct, C->cd2, C->gap, C->eperm, C->estart};
     for (void* p : ptrs)
         if (p) dev_free(p);
     cudaSetDevice(prev);
@@ -527,10 +579,17 @@ extern "C" dda_status_t dda_contact_springs(dda_contacts_t C, const double* cxy,
                                             void* stream) {
     if (!C || !cxy || !(p_n >= 0.0) || !(shear_ratio >= 0.0) || !isfinite(p_n) || !isfinite(shear_ratio))
         return DDA_ERR_ARG;
-    if (C->n_ve == 0) return DDA_OK;
+    const int64_t m = C->count;
+    if ((C->classified ? m : C->n_ve) == 0) return DDA_OK;
     if (!bi || !bj || !pen || !e || !g) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-    const int64_t m = C->count;
+    const double ps = shear_ratio * p_n;                     // the oracle's shear_ratio * p_n
+    if (C->classified) {                                     // every record (VE, VV1, VV2), slot = record
+        k_springs<<<cgrid(m), CT, 0, st>>>(m, nullptr, C->vptr, C->vxy, cxy, C->ci, C->cv, C->cj, C->ce, C->ctype,
+                                           C->ct, p_n, ps, bi, bj, pen, e, g, 1);
+        DDA_LAUNCHED();
+        return DDA_OK;
+    }
     CTmp tmp(st);
     int32_t *f = nullptr, *slot = nullptr;
     DDA_CK(tmp.get(&f, (size_t)m + 1));
@@ -545,9 +604,77 @@ extern "C" dda_status_t dda_contact_springs(dda_contacts_t C, const double* cxy,
         DDA_CK(tmp.get(&ts, tb));
         DDA_CK(cub::DeviceScan::ExclusiveSum(ts, tb, f, slot, (int)m, st));
     }
-    const double ps = shear_ratio * p_n;                     // the oracle's shear_ratio * p_n
     k_springs<<<cgrid(m), CT, 0, st>>>(m, slot, C->vptr, C->vxy, cxy, C->ci, C->cv, C->cj, C->ce, C->ctype, C->ct,
-                                       p_n, ps, bi, bj, pen, e, g);
+                                       p_n, ps, bi, bj, pen, e, g, 0);
     DDA_LAUNCHED();
+    return DDA_OK;
+}
+
+// Second classification: the angle judgment abandons records, the rest is stored
+// class by class in successive arrays (VE, VV1, VV2; increasing (v, e) within a class) — a stable
+// 2-bit radix sort of the class keys ("scan and radix sort methods are used to classify or abandon
+// data") and one gather per field.
+extern "C" dda_status_t dda_classify_contacts(dda_contacts_t C, double sin_tol, void* stream) {
+    if (!C || !(sin_tol >= 0.0) || !(sin_tol < 1.0) || C->classified) return DDA_ERR_ARG;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    const int64_t m = C->count;
+    C->classified = true;
+    if (m == 0) return DDA_OK;
+    CTmp tmp(st);
+    uint32_t *key = nullptr, *skey = nullptr;
+    int32_t *idx = nullptr, *sidx = nullptr;
+    int64_t* start = nullptr;
+    DDA_CK(tmp.get(&key, m)); DDA_CK(tmp.get(&skey, m));
+    DDA_CK(tmp.get(&idx, m)); DDA_CK(tmp.get(&sidx, m));
+    DDA_CK(tmp.get(&start, 5));
+    const double s2 = sin_tol * sin_tol;                     // the oracle's sin_tol * sin_tol
+    k_classify<<<cgrid(m), CT, 0, st>>>(m, C->vptr, C->vxy, C->ci, C->cv, C->cj, C->ce, C->ctype, s2, key, idx);
+    DDA_LAUNCHED();
+    size_t tb = 0;
+    DDA_CK(cub::DeviceRadixSort::SortPairs(nullptr, tb, key, skey, idx, sidx, (int)m, 0, 2, st));
+    char* ts = nullptr;
+    DDA_CK(tmp.get(&ts, tb));
+    DDA_CK(cub::DeviceRadixSort::SortPairs(ts, tb, key, skey, idx, sidx, (int)m, 0, 2, st));
+    note_launch(2);
+    k_class_bounds<<<cgrid(m), CT, 0, st>>>(m, skey, start);
+    DDA_LAUNCHED();
+    int64_t hs[5];
+    DDA_CK(cudaMemcpyAsync(hs, start, sizeof hs, cudaMemcpyDeviceToHost, st));
+    DDA_CK(cudaStreamSynchronize(st));
+    const int64_t kept = m - hs[1];
+    const int32_t* keep_idx = sidx + hs[1];
+    int32_t *ni = nullptr, *nv = nullptr, *nj = nullptr, *ne = nullptr, *nt = nullptr;
+    double *ntt = nullptr, *nd2 = nullptr;
+    auto owned = [&](auto** p) { return dev_alloc(reinterpret_cast<void**>(p), kept ? kept * sizeof(**p) : 16, st); };
+    DDA_CK(owned(&ni)); DDA_CK(owned(&nv)); DDA_CK(owned(&nj)); DDA_CK(owned(&ne)); DDA_CK(owned(&nt));
+    DDA_CK(owned(&ntt)); DDA_CK(owned(&nd2));
+    if (kept > 0) {
+        k_gather<int32_t><<<cgrid(kept), CT, 0, st>>>(kept, keep_idx, C->ci, ni);
+        k_gather<int32_t><<<cgrid(kept), CT, 0, st>>>(kept, keep_idx, C->cv, nv);
+        k_gather<int32_t><<<cgrid(kept), CT, 0, st>>>(kept, keep_idx, C->cj, nj);
+        k_gather<int32_t><<<cgrid(kept), CT, 0, st>>>(kept, keep_idx, C->ce, ne);
+        k_gather<double><<<cgrid(kept), CT, 0, st>>>(kept, keep_idx, C->ct, ntt);
+        k_gather<double><<<cgrid(kept), CT, 0, st>>>(kept, keep_idx, C->cd2, nd2);
+        k_class_type<<<cgrid(kept), CT, 0, st>>>(kept, skey + hs[1], nt);
+        note_launch(6);
+        DDA_LAUNCHED();
+    }
+    void* old[] = {C->ci, C->cv, C->cj, C->ce, C->ctype, C->ct, C->cd2};
+    for (void* p : old) dev_free_on(p, st);
+    C->ci = ni; C->cv = nv; C->cj = nj; C->ce = ne; C->ctype = nt; C->ct = ntt; C->cd2 = nd2;
+    C->count = kept;
+    C->n_ve = hs[2] - hs[1];
+    C->n_vv1 = hs[3] - hs[2];
+    C->n_vv2 = hs[4] - hs[3];
+    return DDA_OK;
+}
+
+extern "C" dda_status_t dda_contacts_classes(dda_contacts_t C, int64_t* n_ve, int64_t* n_vv1, int64_t* n_vv2,
+                                             int32_t* classified) {
+    if (!C) return DDA_ERR_ARG;
+    if (n_ve) *n_ve = C->n_ve;
+    if (n_vv1) *n_vv1 = C->n_vv1;
+    if (n_vv2) *n_vv2 = C->n_vv2;
+    if (classified) *classified = C->classified ? 1 : 0;
     return DDA_OK;
 }

@@ -90,6 +90,14 @@ __device__ __forceinline__ double2 ld_cg2(const double* p) { return *reinterpret
 __device__ __forceinline__ double ld_cg(const double* p) { return *p; }
 #endif
 
+// CTA barrier after lane-divergent code (if (lane == 0) ..., tree steps): __syncthreads() is the
+// .aligned bar.sync, which every thread of a warp must reach converged; __syncwarp() reconverges
+// first (compute-sanitizer synccheck flagged the bare barrier as divergent)
+__device__ __forceinline__ void cta_barrier() {
+    __syncwarp();
+    __syncthreads();
+}
+
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
@@ -145,6 +153,23 @@ struct dda_matrix {
     int last_checks = 0;            // scaled engine: exact stopping tests in the last solve
 };
 
+// contact records of dda_detect_contacts (contact.cu) and the open-close state (openclose.cu)
+struct dda_contacts {
+    int device = 0;
+    int32_t n = 0;
+    int64_t count = 0, n_ve = 0, n_pairs = 0;
+    bool classified = false;         // dda_classify_contacts ran: ctype = class (0 VE, 1 VV1, 2 VV2)
+    int64_t n_vv1 = 0, n_vv2 = 0;
+    const int32_t* vptr = nullptr;   // caller's geometry (must outlive dda_contact_springs)
+    const double* vxy = nullptr;
+    int32_t *ci = nullptr, *cv = nullptr, *cj = nullptr, *ce = nullptr, *ctype = nullptr;
+    double *ct = nullptr, *cd2 = nullptr;
+    // NEXT-4 (dda_contact_init): signed gaps and the contact endpoints sorted by block
+    double* gap = nullptr;           // [count] n.(P - Q1)
+    int32_t* eperm = nullptr;        // [2 count] endpoint records 2k + side, stably sorted by block
+    int32_t* estart = nullptr;       // [n + 1] segment starts into eperm
+};
+
 namespace dda {
 dda_status_t ensure_workspace(dda_matrix* K, size_t bytes, cudaStream_t st);
 dda_status_t bj_setup(dda_matrix* K, cudaStream_t s, int32_t* bad_block);
@@ -157,6 +182,8 @@ dda_status_t build_matrix_impl(int32_t n, const double* kdiag, int64_t m, const 
 dda_status_t ilu_setup(dda_matrix* K, cudaStream_t st, int32_t* bad_block);
 dda_status_t ilu_apply(dda_matrix* K, const double* r, double* z, double* y, double* yh, cudaStream_t st);
 int ilu_grid();
+int comm_nparts(const dda_comm* c);                 // partitions of the communicator (NCCL: ranks)
+int comm_part_index(const dda_comm* c, int part);   // global partition index of local slot `part`, -1 if invalid
 dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, double* d, double tol,
                              int32_t maxit, dda_precond_t pc, double omega, int32_t* iters, double* rel_res,
                              cudaStream_t st, bool scaled);

@@ -46,13 +46,13 @@ __device__ __forceinline__ void cta_partial(double v, double* part, int slot_str
     const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
     v = warp_sum(v);
     if (lane == 0) red[wib] = v;
-    __syncthreads();
+    cta_barrier();
     if (threadIdx.x == 0) {
         double s = 0.0;
         for (int w = 0; w < WPB; ++w) s += red[w];
         part[k * slot_stride + blockIdx.x] = s;
     }
-    __syncthreads();
+    cta_barrier();
 }
 
 
@@ -155,13 +155,13 @@ __global__ void k_sum_parts(const double* part, int G, int nv, double* out) {
         double s = 0.0;
         for (int j = threadIdx.x; j < G; j += blockDim.x) s += part[k * G + j];
         red[threadIdx.x] = s;
-        __syncthreads();
+        cta_barrier();
         for (int h = blockDim.x / 2; h > 0; h >>= 1) {
             if (threadIdx.x < h) red[threadIdx.x] += red[threadIdx.x + h];
-            __syncthreads();
+            cta_barrier();
         }
         if (threadIdx.x == 0) out[k] = red[0];
-        __syncthreads();
+        cta_barrier();
     }
 }
 
@@ -512,6 +512,12 @@ struct dda_comm {
     std::vector<DistPart> parts;
 };
 
+int dda::comm_nparts(const dda_comm* c) { return c->nranks; }
+int dda::comm_part_index(const dda_comm* c, int part) {
+    if (c->loopback) return (part >= 0 && part < c->nranks) ? part : -1;
+    return part == 0 ? c->rank : -1;
+}
+
 static dda_status_t nccl_fail(ncclResult_t r) {
     (void)r;
     return DDA_ERR_NCCL;
@@ -566,6 +572,26 @@ extern "C" void dda_comm_free(dda_comm_t c) {
     }
     if (c->nccl) ncclCommDestroy(c->nccl);
     delete c;
+}
+
+extern "C" dda_status_t dda_dist_info(dda_comm_t c, int32_t part, int32_t* n_own, int32_t* n_halo,
+                                      int32_t* send_counts, int32_t* recv_counts, int32_t* send_idx) {
+    if (!c) return DDA_ERR_ARG;
+    const int slot = c->loopback ? part : 0;
+    if (slot < 0 || slot >= (int)c->parts.size() || (!c->loopback && part != 0)) return DDA_ERR_ARG;
+    const DistPart& D = c->parts[slot];
+    if (!D.K) return DDA_ERR_ARG;
+    if (n_own) *n_own = D.n_own;
+    if (n_halo) *n_halo = D.n_local - D.n_own;
+    for (int q = 0; q < c->nranks; ++q) {
+        if (send_counts) send_counts[q] = D.send_counts[q];
+        if (recv_counts) recv_counts[q] = D.recv_counts[q];
+    }
+    if (send_idx && D.n_send) {
+        if (cudaMemcpy(send_idx, D.send_idx, D.n_send * sizeof(int), cudaMemcpyDeviceToHost) != cudaSuccess)
+            return DDA_ERR_CUDA;
+    }
+    return DDA_OK;
 }
 
 extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t K, int32_t n_own,

@@ -68,13 +68,13 @@ __device__ __forceinline__ void cta_partials(double (&v)[NV], double* part, int 
 #pragma unroll
         for (int k = 0; k < NV; ++k) red[wib][k] = v[k];
     }
-    __syncthreads();
+    cta_barrier();
     if (threadIdx.x < NV) {
         double s = 0.0;
         for (int w = 0; w < WPB; ++w) s += red[w][threadIdx.x];
         part[threadIdx.x * G + blockIdx.x] = s;
     }
-    __syncthreads();
+    cta_barrier();
 }
 
 // fixed-order sum of part[k*G .. k*G+G) for k < NV, identical in every CTA
@@ -90,10 +90,10 @@ __device__ __forceinline__ void grid_sums(const double* part, int G, double (&ou
             if (lane == 0) bc[k] = s;
         }
     }
-    __syncthreads();
+    cta_barrier();
 #pragma unroll
     for (int k = 0; k < NV; ++k) out[k] = bc[k];
-    __syncthreads();
+    cta_barrier();
 }
 
 // ---------------------------------------------------------------- phases

@@ -1,4 +1,9 @@
-"""Block-row partition of K·d = F for the multi-GPU solve.
+"""TEST HELPER — host (numpy) reference of the block-row partition.
+
+The product builds partitions on the device behind the C ABI (dda_build_matrix_dist,
+csrc/dist_build.cu); this module is the independent host-side statement of the same
+selection / numbering / exchange plan that the tests compare it with, and the
+distributed-PCG emulation of tests/test_partition.py runs on it.
 
 The paper is single-GPU; multi-GPU is its future work.  The path
 shards by block rows: rank p owns the contiguous rows [r_p, r_{p+1}).  Each
@@ -16,7 +21,7 @@ exchange per SpMV fills x[n_own:] — the segment received from peer q is
 contiguous (halo grouped by owner), so it is received in place; the segment
 sent to q lists the own rows that q holds as halo, in q's order.
 
-This module is host logic (numpy); the solve runs in libdda (dist.cu).
+(Host logic, numpy; the product equivalent is dda_build_matrix_dist.)
 """
 from __future__ import annotations
 

@@ -154,3 +154,74 @@ def test_contacts_mixed_sizes(dda):
     Cg, G = _gpu(dda, vptr2, vxy2, 0.3)
     assert (O["i"] == 150).any() or (O["j"] == 150).any()
     _same(G, O)
+
+
+# ------------------------------------------------------------------ second classification (O-10)
+
+ANGLE = os.path.join(os.path.dirname(__file__), "golden", "contact_angle_classes.json")
+
+
+@pytest.mark.parametrize("case", ["aligned", "corner", "dart"])
+def test_classify_golden(dda, case):
+    G = json.load(open(ANGLE))
+    c = G["cases"][case]
+    vptr, vxy = np.array(c["vptr"], np.int32), np.array(c["vxy"], float)
+    for tol, want in c["classes"].items():
+        Cg, _ = _gpu(dda, vptr, vxy, G["d0"])
+        Cg.classify(float(tol))
+        got = Cg.export()
+        w = np.array(want)
+        keep = np.nonzero(w >= 0)[0]
+        order = keep[np.argsort(w[keep], kind="stable")]
+        assert np.array_equal(got["v"], np.array(c["v"])[order]) and np.array_equal(got["e"], np.array(c["e"])[order])
+        assert np.array_equal(got["type"], w[order]), tol
+        assert (Cg.n_ve, Cg.n_vv1, Cg.n_vv2) == tuple(int((w == k).sum()) for k in (0, 1, 2))
+        if "first_springs" in c and tol == "0.35":
+            sp = Cg.springs(torch.tensor(c["centroid"], dtype=torch.float64).cuda(), 3.0, 0.5)
+            assert np.array_equal(sp["e"][:2].cpu().numpy(), np.array(c["first_springs"]["e"], float))
+            assert np.array_equal(sp["g"][:2].cpu().numpy(), np.array(c["first_springs"]["g"], float))
+
+
+@pytest.mark.parametrize("name,d0,tol", [("tiny", 0.35, 0.35), ("ragged_1k", 0.2, 0.35), ("polygons", 0.15, 0.35),
+                                         ("polygons", 0.15, 0.0), ("polygons", 0.15, 0.8)])
+def test_classify_vs_oracle(dda, name, d0, tol):
+    """The classified set (records kept by the angle judgment, grouped VE / VV1 / VV2) and the
+    springs of every class, bit-exact against O-10 + O-9."""
+    if name == "polygons":
+        vptr, vxy, cxy = _random_polygons(600, 3)
+    else:
+        P = make_slope(preset("tiny") if name == "tiny" else preset(1000, seed=1041))
+        vptr, vxy, cxy = _slope_geom(P)
+    O = oracle.detect_contacts(vptr, vxy, d0)
+    Oc = oracle.classified_contacts(vptr, vxy, O, tol)
+    Cg, _ = _gpu(dda, vptr, vxy, d0)
+    Cg.classify(tol)
+    _same(Cg.export(), Oc)
+    if name == "polygons" and tol == 0.35:
+        assert Cg.n_vv2 > 0 and Cg.n_vv1 > 0 and Cg.count < O["v"].size
+    so = oracle.classified_springs(vptr, vxy, cxy, Oc, 40.0, 0.4)
+    sg = Cg.springs(torch.from_numpy(cxy).cuda(), 40.0, 0.4)
+    for k in ("bi", "bj", "pen", "e", "g"):
+        assert np.array_equal(sg[k].cpu().numpy(), so[k]), k
+
+
+def test_classify_full_size_sampled(dda):
+    """1M blocks: the classified records of a vertex sample equal the oracle's classification of that
+    vertex's records (the class grouping keeps increasing (v, e) inside each class)."""
+    P = make_slope(preset(1_000_000, seed=1005))
+    vptr, vxy, cxy = _slope_geom(P)
+    Cg, _ = _gpu(dda, vptr, vxy, 0.2)
+    n0 = Cg.count
+    Cg.classify(0.35)
+    G = Cg.export()
+    assert Cg.count == Cg.n_ve + Cg.n_vv1 + Cg.n_vv2 and Cg.count < n0
+    assert np.all(np.diff(G["type"]) >= 0)
+    rng = np.random.default_rng(5)
+    V = vxy.shape[0]
+    for v in np.unique(np.concatenate([[0, V - 1], rng.integers(0, V, 24)])):
+        O = oracle.detect_contacts(vptr, vxy, 0.2, int(v), int(v) + 1)
+        Oc = oracle.classified_contacts(vptr, vxy, O, 0.35)
+        sel = G["v"] == v
+        _same({k: G[k][sel] for k in FIELDS}, Oc)
+    sg = Cg.springs(torch.from_numpy(cxy).cuda(), 40.0, 0.4)
+    assert sg["bi"].shape[0] == 2 * Cg.count

@@ -11,7 +11,7 @@ import pytest
 torch = pytest.importorskip("torch")
 
 import oracle
-from paper_conf_ipps_xiaohmxw17_b200.partition import row_bounds, local_from_slope
+from partition_ref import row_bounds, local_from_slope
 from synth import make_slope, preset, random_vector
 
 pytestmark = pytest.mark.gpu
@@ -98,6 +98,94 @@ def test_pcg_dist_warm_and_zero(dda, prob, dist_version):
     # iteration cap not a multiple of the host-check chunk (device-side loop state, v2)
     _, it5, rr5, st5 = comm.pcg_solve(Fs, maxit=13)
     assert st5 == dda.ERR_NO_CONVERGENCE and it5 == 13 and rr5 > 1e-10
+
+
+def _setup_device(dda, P, nparts, shuffle_springs=False):
+    """Partitions built behind the C ABI (dda_build_matrix_dist) from the GLOBAL spring list."""
+    b = dda.row_bounds(P.n, nparts)
+    comm = dda.Comm.loopback(nparts)
+    t = dda.problem_to_device(P)
+    Ks, Fs = [], []
+    for r in range(nparts):
+        r0, r1 = int(b[r]), int(b[r + 1])
+        Ks.append(comm.build_matrix_dist(r, P.n, b, t["kdiag"][r0:r1].contiguous(), t["bi"], t["bj"], t["pen"],
+                                         t["e"], t["g"]))
+        Fs.append(t["F"][6 * r0:6 * r1].contiguous())
+    return comm, b, Ks, Fs
+
+
+@pytest.mark.parametrize("nparts", [1, 2, 3, 4])
+def test_build_matrix_dist_matches_host_reference(dda, prob, nparts):
+    """The device partition (selection, halo, numbering, assembly, plan) equals the host reference
+    tests/partition_ref.py: local structure and values bit-exact against the ORACLE's assembly of the
+    reference local problem, and the same n_halo / send / receive plan."""
+    P, O = prob
+    comm, b, Ks, Fs = _setup_device(dda, P, nparts)
+    bref = row_bounds(P.n, nparts)
+    assert np.array_equal(b, bref)
+    for r in range(nparts):
+        lp = local_from_slope(P, bref, r)
+        Ol = oracle.OracleMatrix(lp.n_local, lp.kdiag, lp.bi, lp.bj, lp.pen, lp.e, lp.g)
+        S, ex = Ol.export(), Ks[r].export()
+        for k in ("row_ptr", "col_idx", "low_ptr", "low_row", "low_to_up"):
+            assert np.array_equal(ex[k], getattr(S, k)), (r, k)
+        assert np.array_equal(ex["diag"], S.diag) and np.array_equal(ex["upper"], S.upper), r
+        inf = comm.info(r)
+        assert inf["n_own"] == lp.n_own and inf["n_halo"] == lp.n_halo
+        assert np.array_equal(inf["send_counts"], lp.send_counts)
+        assert np.array_equal(inf["recv_counts"], lp.recv_counts)
+        assert np.array_equal(inf["send_idx"], lp.send_idx)
+
+
+@pytest.mark.parametrize("nparts", [2, 4])
+def test_pcg_dist_device_built(dda, prob, nparts, dist_version):
+    """Partitions from dda_build_matrix_dist solved by dda_pcg_solve_dist, vs the oracle (Z17)."""
+    P, O = prob
+    comm, b, Ks, Fs = _setup_device(dda, P, nparts)
+    ds, it, rr, st = comm.pcg_solve(Fs, tol=1e-10, precond="bj")
+    assert st == dda.OK and rr <= 1.01e-10
+    do, ito, rro, sto = O.pcg(P.F, tol=1e-10, precond="bj")
+    assert abs(it - ito) <= max(2, int(0.01 * ito))
+    dm, _, _, _ = O.pcg(P.F, tol=1e-300, maxit=it, precond="bj")
+    d = np.concatenate([t.cpu().numpy() for t in ds])
+    assert np.linalg.norm(d - dm) / np.linalg.norm(dm) <= 1e-9
+    y = np.concatenate([t.cpu().numpy() for t in comm.spmv([torch.from_numpy(d[6 * b[r]:6 * b[r + 1]].copy()).cuda()
+                                                               for r in range(nparts)])])
+    assert np.linalg.norm(y - O.spmv(d)) <= 1e-12 * np.linalg.norm(y)
+
+
+def test_build_matrix_dist_errors(dda, prob):
+    P, O = prob
+    comm = dda.Comm.loopback(2)
+    t = dda.problem_to_device(P)
+    b = dda.row_bounds(P.n, 2)
+    kd = t["kdiag"][: int(b[1])].contiguous()
+    for bad_b in (np.array([0, 5, 5], np.int32), np.array([1, 5, P.n], np.int32)):
+        kdb = t["kdiag"][: int(bad_b[1] - bad_b[0])].contiguous()
+        with pytest.raises(dda.DDAError):
+            comm.build_matrix_dist(0, P.n, bad_b, kdb, t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+    with pytest.raises(dda.DDAError):                 # partition index out of range
+        comm.build_matrix_dist(2, P.n, b, kd, t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+    bi = t["bi"].clone()
+    bi[3] = P.n                                       # id out of range
+    with pytest.raises(dda.DDAError):
+        comm.build_matrix_dist(0, P.n, b, kd, bi, t["bj"], t["pen"], t["e"], t["g"])
+
+
+def test_pcg_dist_nccl_single_rank_oracle(dda, prob):
+    """NCCL transport (one rank), partition built on the device, against the oracle (Z17)."""
+    P, O = prob
+    comm = dda.Comm.nccl(1, 0, dda.Comm.unique_id())
+    t = dda.problem_to_device(P)
+    b = dda.row_bounds(P.n, 1)
+    comm.build_matrix_dist(0, P.n, b, t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+    ds, it, rr, st = comm.pcg_solve([t["F"]])
+    assert st == dda.OK and rr <= 1.01e-10
+    do, ito, _, _ = O.pcg(P.F, tol=1e-10, precond="bj")
+    assert abs(it - ito) <= max(2, int(0.01 * ito))
+    dm, _, _, _ = O.pcg(P.F, tol=1e-300, maxit=it, precond="bj")
+    assert np.linalg.norm(ds[0].cpu().numpy() - dm) / np.linalg.norm(dm) <= 1e-9
+    comm.free()
 
 
 def test_pcg_dist_nccl_single_rank(dda, prob, dist_version):

@@ -114,3 +114,98 @@ def test_invariances():
     C5 = oracle.detect_contacts(vptr, vxy, 0.2, a, b)
     sel = (C["v"] >= a) & (C["v"] < b)
     assert np.array_equal(C5["e"], C["e"][sel]) and np.array_equal(C5["dist2"], C["dist2"][sel])
+
+
+# ------------------------------------------------------------------ O-10: angle judgment, VV1 / VV2
+
+ANGLE = os.path.join(os.path.dirname(__file__), "golden", "contact_angle_classes.json")
+
+
+@pytest.mark.parametrize("case", ["aligned", "corner", "dart"])
+def test_golden_angle_classes(case):
+    G = json.load(open(ANGLE))
+    c = G["cases"][case]
+    vptr, vxy = np.array(c["vptr"], np.int32), np.array(c["vxy"], float)
+    C = oracle.detect_contacts(vptr, vxy, G["d0"])
+    assert np.array_equal(C["v"], c["v"]) and np.array_equal(C["e"], c["e"])
+    for tol, want in c["classes"].items():
+        assert np.array_equal(oracle.classify_contacts(vptr, vxy, C, float(tol)), want), tol
+    if "first_springs" in c:
+        Cc = oracle.classified_contacts(vptr, vxy, C, 0.35)
+        sp = oracle.classified_springs(vptr, vxy, np.array(c["centroid"], float), Cc, 3.0, 0.5)
+        assert np.array_equal(sp["e"][:2], np.array(c["first_springs"]["e"], float))
+        assert np.array_equal(sp["g"][:2], np.array(c["first_springs"]["g"], float))
+        assert np.array_equal(sp["pen"][:2], [3.0, 1.5])
+
+
+def _rot90(vxy):
+    """(x, y) -> (-y, x): exact in binary, preserves orientation, lengths and angles."""
+    return np.stack([-vxy[:, 1], vxy[:, 0]], axis=1)
+
+
+@pytest.mark.parametrize("name", ["tiny", "ragged"])
+def test_angle_classes_invariant_and_generator_contacts(name):
+    """Exact invariances of O-10 (rotation by 90 degrees, scaling by 2); every contact of the slope
+    generator's own layout list (shared brick edges) passes the angle judgment, as VE or, at an
+    edge end, VV1; the classified set is the passing records grouped VE, VV1, VV2."""
+    P = make_slope(preset("tiny") if name == "tiny" else preset(400, seed=1047))
+    vptr, vxy, cxy = _geom(P)
+    C = oracle.detect_contacts(vptr, vxy, 0.35)
+    cls = oracle.classify_contacts(vptr, vxy, C, 0.35)
+    assert set(np.unique(cls)) <= {-1, 0, 1, 2}
+    assert ((cls == 0) <= (C["type"] == 0)).all() and ((cls >= 1) <= (C["type"] == 1)).all()
+    Cr = oracle.detect_contacts(vptr, _rot90(vxy), 0.35)
+    assert np.array_equal(Cr["v"], C["v"]) and np.array_equal(Cr["e"], C["e"])
+    assert np.array_equal(oracle.classify_contacts(vptr, _rot90(vxy), Cr, 0.35), cls)
+    C2 = oracle.detect_contacts(vptr, 2.0 * vxy, 0.7)
+    assert np.array_equal(oracle.classify_contacts(vptr, 2.0 * vxy, C2, 0.35), cls)
+    # the generator's layout contacts (ends of shared, hence antiparallel, brick edges): all kept, the
+    # interior ones VE and those at an edge end VV1 (parallel edges, P:72)
+    pos = np.searchsorted(_keys(C), _keys(P.contacts))
+    assert np.array_equal(cls[pos], C["type"][pos])
+    # monotone in the tolerance: a larger angle tolerance abandons no more records
+    cls_big = oracle.classify_contacts(vptr, vxy, C, 0.6)
+    assert ((cls >= 0) <= (cls_big >= 0)).all()
+    Cc = oracle.classified_contacts(vptr, vxy, C, 0.35)
+    assert np.array_equal(np.sort(Cc["type"], kind="stable"), Cc["type"])
+    assert Cc["type"].size == (cls >= 0).sum()
+
+
+def test_angle_classes_brute_force_angles():
+    """Cross-check O-10 against a differently computed statement of the same rule (angles by
+    arctan2, not squared products): the decisions agree wherever the margin exceeds 1e-9 rad."""
+    P = make_slope(preset(400, seed=1047))
+    vptr, vxy, _ = _geom(P)
+    C = oracle.detect_contacts(vptr, vxy, 0.35)
+    cls = oracle.classify_contacts(vptr, vxy, C, 0.35)
+    th = np.arcsin(0.35)
+    agree = 0
+    for k in range(C["i"].size):
+        i, v, j, e = (int(C[f][k]) for f in ("i", "v", "j", "e"))
+        a0, a1 = vptr[i], vptr[i + 1]
+        P0 = vxy[v]
+        A = vxy[v - 1 if v > a0 else a1 - 1] - P0
+        B = vxy[v + 1 if v + 1 < a1 else a0] - P0
+        q2 = e + 1 if e + 1 < vptr[j + 1] else vptr[j]
+        d = vxy[q2] - vxy[e]
+        nrm = np.arctan2(-d[0], d[1])                         # direction of the outward normal
+        def elev(x):                                          # angle of x above the edge line (toward N)
+            ang = np.arctan2(x[1], x[0]) - nrm
+            return np.pi / 2 - abs((ang + np.pi) % (2 * np.pi) - np.pi)
+        def par(x):                                           # angle between x and the edge line
+            ang = abs((np.arctan2(x[1], x[0]) - np.arctan2(d[1], d[0])) % np.pi)
+            return min(ang, np.pi - ang)
+        turn = np.arctan2(A[0] * B[1] - A[1] * B[0], A @ B)
+        margins = [abs(elev(A) + th), abs(elev(B) + th), abs(turn)]
+        if min(margins) < 1e-9:
+            continue
+        ok = turn < 0 and elev(A) >= -th and elev(B) >= -th
+        want = -1 if not ok else (0 if C["type"][k] == 0 else None)
+        if want is None:
+            pm = [abs(par(A) - th), abs(par(B) - th)]
+            if min(pm) < 1e-9:
+                continue
+            want = 1 if (par(A) <= th or par(B) <= th) else 2
+        assert cls[k] == want, (k, cls[k], want)
+        agree += 1
+    assert agree > 0.99 * C["i"].size

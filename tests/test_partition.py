@@ -14,7 +14,7 @@ import torch.distributed as dist
 import torch.multiprocessing as mp
 
 import oracle
-from paper_conf_ipps_xiaohmxw17_b200.partition import row_bounds, local_from_slope, owner_of
+from partition_ref import row_bounds, local_from_slope, owner_of
 from synth import make_slope, preset
 
 

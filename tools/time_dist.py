@@ -8,21 +8,21 @@ import torch
 import paper_conf_ipps_xiaohmxw17_b200 as dda
 if os.environ.get("DDA_LIB_PATH"):          # A/B against another build of the library
     dda.LIB_PATH = os.environ["DDA_LIB_PATH"]
-from paper_conf_ipps_xiaohmxw17_b200.partition import row_bounds, local_from_slope
 from synth import make_slope, preset
 n = int(sys.argv[1]) if len(sys.argv) > 1 else 1_000_000
 P = make_slope(preset(n, seed=1005))
 out = {}
 for nparts in (1, 2):
-    b = row_bounds(P.n, nparts)
+    b = dda.row_bounds(P.n, nparts)
     comm = dda.Comm.loopback(nparts)
+    t = dda.problem_to_device(P)
     Fs, keep = [], []
     for r in range(nparts):
-        lp = local_from_slope(P, b, r)
-        K = dda.build_local(lp)
-        comm.attach(r, K, lp)
-        keep.append((K, lp))
-        Fs.append(torch.from_numpy(P.F[6 * lp.r0: 6 * lp.r1].copy()).cuda())
+        r0, r1 = int(b[r]), int(b[r + 1])
+        K = comm.build_matrix_dist(r, P.n, b, t["kdiag"][r0:r1].contiguous(), t["bi"], t["bj"], t["pen"], t["e"],
+                                   t["g"])
+        keep.append(K)
+        Fs.append(t["F"][6 * r0: 6 * r1].contiguous())
     ms = []
     for rep in range(4):
         a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
