@@ -77,7 +77,6 @@ struct GArgs {           // constant for a (matrix, preconditioner): baked into 
     int use_cond;        // 0 only for the internal phase-timing hook (kernels launched outside the graph)
     unsigned long long* trace;   // k_sp_loop timeline [iter][cta][4] (%globaltimer), null = off (internal hook)
     int trace_iters;
-    int* ctr;            // k_sp_loop<.., DYN>: phase-A group counters [2] (iteration parity), zero at launch
 };
 
 __device__ __forceinline__ unsigned long long gtimer() {
@@ -803,7 +802,7 @@ __device__ __forceinline__ void grid_allsum(const GArgs& a, cg::grid_group& grid
     cta_barrier();
 }
 
-template <int MINB, bool DYN>
+template <int MINB>
 __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_loop(const GArgs a) {
     cg::grid_group grid = cg::this_grid();
     State* st = a.st;
@@ -846,10 +845,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_loop(const GArgs a) {
                 acc += pv.x * y0 + pv.y * y1;
             }
         };
-        if (DYN)
-            for_rows_cd<SPMV_OFFDIAG, 5>(A, w0, W, a.ctr + (k & 1), xf, lane, rowA);
-        else
-            for_rows_c<SPMV_OFFDIAG, 5>(A, w0, W, xf, lane, rowA);
+        for_rows_c<SPMV_OFFDIAG, 5>(A, w0, W, xf, lane, rowA);
         if (tr) tr[1] = gtimer();
         double sv[1] = {acc}, stot[1];
         grid_allsum<1>(a, grid, 0, sv, stot);
@@ -858,9 +854,6 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_loop(const GArgs a) {
         pend = 0;
         if (!(sigma > 0.0) || !isfinite(sigma)) { status = DDA_ERR_BREAKDOWN; break; }   // reading Z19
         alpha = rho / sigma;
-        // the other parity's group counter was last used by phase A of iteration k-1 (before barrier
-        // A of k-1) and is next used by phase A of k+1 (after barrier B of k): reset it here
-        if (DYN && blockIdx.x == 0 && threadIdx.x == 0) a.ctr[(k + 1) & 1] = 0;
         // phase B: r~ -= alpha q; rho' = |r~|^2 and the lower bound sum_i w_i |r~_i|^2 of |L r~|^2
         double rz = 0.0, lb = 0.0;
         for (int grp = w0; grp < ngrp; grp += 2 * W) {
@@ -1177,7 +1170,6 @@ int occ_grid(const void* k, int minb_cap) {
 // scaled-engine loop: 1 = persistent cooperative kernel, 0 = CUDA-graph while loop, -1 = from
 // DDA_SCALED_LOOP (default persistent); set by the internal hook dda__set_scaled_loop
 int g_scaled_loop = -1;
-int g_dyn_tail = env_int("DDA_DYN_TAIL", 1);   // k_sp_loop phase A: dynamic tail (for_rows_cd) or static map
 unsigned long long* g_trace = nullptr;   // k_sp_loop timeline (internal hook dda__set_loop_trace)
 int g_trace_iters = 0;
 
@@ -1236,8 +1228,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     // scaled SSOR-AI exists as a persistent kernel only (k_sp_ssor)
     bool persist = scaled && (g_scaled_loop == 1 || pc == DDA_PC_SSOR_AI);
     const void* persist_kernel = pc == DDA_PC_SSOR_AI ? reinterpret_cast<const void*>(k_sp_ssor)
-                                                      : (g_dyn_tail ? reinterpret_cast<const void*>(k_sp_loop<3, true>)
-                                                                    : reinterpret_cast<const void*>(k_sp_loop<3, false>));
+                                                      : reinterpret_cast<const void*>(k_sp_loop<3>);
     if (persist) {
         // The persistent kernels need every CTA co-resident (cooperative launch).  If not even one CTA
         // per SM fits (e.g. a smaller shared-memory carve-out forced by the caller's context), fall
@@ -1301,7 +1292,6 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         char* tail = reinterpret_cast<char*>(a.part + 4 * (size_t)Gmax);
         a.ca = reinterpret_cast<CallArgs*>(tail);
         a.st = reinterpret_cast<State*>(tail + ((sizeof(CallArgs) + 15) / 16) * 16);
-        a.ctr = reinterpret_cast<int*>(reinterpret_cast<char*>(a.st) + ((sizeof(State) + 15) / 16) * 16);
         a.pc = (int)pc;
         a.out = reinterpret_cast<int*>(reinterpret_cast<char*>(K->scratch) + 128);
         a.use_cond = 1;
@@ -1406,7 +1396,6 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     }
     // ---- the device-side loop (its kernel launches are counted below from the iteration count)
     if (G->G_persist) {
-        DDA_CK(cudaMemsetAsync(a.ctr, 0, 2 * sizeof(int), st));
         a.trace = g_trace;
         a.trace_iters = g_trace_iters;
         void* kargs[] = {reinterpret_cast<void*>(&a)};
@@ -1576,7 +1565,3 @@ extern "C" int dda__time_ks_variants(dda_matrix_t K, const double* F, double* d,
     cudaEventDestroy(e0); cudaEventDestroy(e1);
     return cudaGetLastError() == cudaSuccess ? 0 : -3;
 }
-
-// internal A/B hook: k_sp_loop phase A with the dynamic tail (1) or the static map (0), from the
-// next solve on
-extern "C" void dda__set_dyn_tail(int v) { dda::g_dyn_tail = v; }

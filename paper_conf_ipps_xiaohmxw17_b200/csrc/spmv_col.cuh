@@ -244,44 +244,4 @@ __device__ __forceinline__ void for_rows_c(const BsrView& A, int w, int W, const
     }
 }
 
-// Row loop with a dynamic tail: steps 0..S-1 are the static map of for_rows_c (warp w takes
-// ten-row group w + s W), then the remaining groups (S W .. ngroups-1, in increasing order) are
-// handed out one at a time from the counter *ctr (zero on entry; lane 0 grabs, the warp
-// broadcasts).  S = floor(ngroups / W) - 1, so about one step's worth of groups is dynamic: the
-// warps that finish their static steps first take them, instead of 18% of the warps running a
-// whole extra step while the others wait at the next grid barrier.  Groups are still taken in
-// increasing row order (the transposed re-reads keep hitting L2).  The next group is fetched one
-// row ahead, so the atomic's latency hides behind the current row.
-template <int MODE, int V = 4, class XLoad, class Body>
-__device__ __forceinline__ void for_rows_cd(const BsrView& A, int w, int W, int* ctr, const XLoad& xload, int lane,
-                                            const Body& body) {
-    const int h = cgrp_of(lane);
-    const bool lane_ok = lane < 30;
-    const int ngrp = (A.n + 9) / 10;
-    int S = ngrp / W - 1;
-    if (S < 0) S = 0;
-    const int g0 = S * W;
-    auto grab = [&]() -> int {
-        int t = 0;
-        if (lane == 0) t = atomicAdd(ctr, 1);
-        return g0 + __shfl_sync(0xffffffffu, t, 0);
-    };
-    int g = S > 0 ? w : grab();
-    RowBounds nxt = row_bounds<MODE>(A, 10 * g + h, lane_ok && g < ngrp);
-    for (int step = 0; g < ngrp; ++step) {
-        const int gn = step + 1 < S ? w + (step + 1) * W : grab();
-        const int i = 10 * g + h;
-        const bool ok = lane_ok && i < A.n;
-        const RowBounds cur = nxt;
-        nxt = row_bounds<MODE>(A, 10 * gn + h, lane_ok && gn < ngrp);
-        double y0, y1;
-        if (V == 5)
-            spmv_row_c5<MODE>(A, i, ok, cur, xload, lane, y0, y1);
-        else
-            spmv_row_c4<MODE>(A, i, ok, cur, xload, lane, y0, y1);
-        body(i, ok, y0, y1);
-        g = gn;
-    }
-}
-
 }  // namespace dda
