@@ -285,6 +285,42 @@ dda_status_t dda_rcm_order(int32_t n_blocks, int64_t n_springs, const int32_t *b
                            int32_t *perm);
 
 /*
+ * NEXT-2 — the same order applied INSIDE the library: arguments and errors as dda_build_matrix
+ * (bi, bj device, caller's numbering).  The matrix is assembled in the RCM numbering of the contact
+ * graph (computed on the host from a copy of bi, bj: once per contact structure); every entry point
+ * keeps the caller's numbering by permuting at the boundary: dda_spmv / dda_spmv_full / dda_pcg_solve
+ * / dda_precond_apply (vectors gathered in and scattered out: 48 B per row each way, once per call —
+ * a PCG solve permutes F, d0 and d, not its iterations), dda_update_values (kdiag gathered),
+ * dda_bj_setup (D^{-1} and the failing block id in the caller's numbering), dda_matrix_export (the
+ * canonical arrays of the caller's numbering, rebuilt on the host; values bit-identical to
+ * dda_build_matrix's).  Block-Jacobi (and plain CG) do not depend on the order; SSOR-AI's triangular
+ * split and ILU(0)'s incomplete factor are those of the internal order.  Not accepted by
+ * dda_dist_attach.  Synchronising.
+ */
+dda_status_t dda_build_matrix_reordered(int32_t n_blocks, const double *kdiag, int64_t n_springs, const int32_t *bi,
+                                        const int32_t *bj, const double *pen, const double *e, const double *g,
+                                        void *stream, dda_matrix_t *out);
+
+/*
+ * NEXT-2 ablation — the paper's HSBCSR two-stage SpMV (§IV.B; Figs. 6-9), for the
+ * comparison of P:222 (2.8x over cuSPARSE on the K40) next to dda_spmv on B200.
+ * dda_hsbcsr_build copies K (not a reordered one) into the half-slice layout: d-data [6][dstride]
+ * and nd-data-up [6][ustride], where slice r holds row r (6 doubles) of every diagonal / upper block
+ * in block order and each slice is padded to a multiple of 32 doubles (reading Z13), so entry
+ * (block b, row r, column c) is at stride * r + 6 b + c.  dda_hsbcsr_spmv computes y = K x in two
+ * stages: (1) per upper block b = (i, j), up-res[b] = V_b x_j and low-res[b] = V_b^T x_i; (2) per row,
+ * D_i x_i + the up-res of its row + the low-res of its lower row through row-low-p (= low_to_up).
+ * x, y device [6n], no alias; stream-ordered; same tolerance as dda_spmv.  dda_hsbcsr_export copies
+ * the two slice arrays to host buffers (either may be NULL) and the two strides (host int64 [2]).
+ * The handle reads K's index arrays: K must outlive it.
+ */
+typedef struct dda_hsbcsr *dda_hsbcsr_t;
+dda_status_t dda_hsbcsr_build(dda_matrix_t K, void *stream, dda_hsbcsr_t *out);
+dda_status_t dda_hsbcsr_spmv(dda_hsbcsr_t H, const double *x, double *y, void *stream);
+dda_status_t dda_hsbcsr_export(dda_hsbcsr_t H, double *d_data, double *nd_data_up, int64_t *strides);
+void dda_hsbcsr_free(dda_hsbcsr_t H);
+
+/*
  * NEXT-3 — contact detection on the GPU (§III.B): the narrow phase's distance
  * judgment and its VE / VV classification, and the springs of the VE contacts that feed
  * dda_build_matrix (P:96 contact edge ratio).

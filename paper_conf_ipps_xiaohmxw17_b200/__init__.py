@@ -31,7 +31,9 @@ ABI_SYMBOLS = ("dda_build_matrix", "dda_update_values", "dda_matrix_info", "dda_
                "dda_memory_release", "dda_memory_cached", "dda_detect_contacts", "dda_contacts_info",
                "dda_contacts_export", "dda_contact_springs", "dda_contacts_free", "dda_build_matrix_dist",
                "dda_dist_info", "dda_classify_contacts", "dda_contacts_classes",
-               "dda_contact_init", "dda_contact_loads", "dda_contact_check", "dda_open_close")
+               "dda_contact_init", "dda_contact_loads", "dda_contact_check", "dda_open_close",
+               "dda_build_matrix_reordered", "dda_hsbcsr_build", "dda_hsbcsr_spmv", "dda_hsbcsr_export",
+               "dda_hsbcsr_free")
 
 _lib = None
 
@@ -55,6 +57,16 @@ def lib() -> C.CDLL:
         st = C.c_int
         L.dda_build_matrix.argtypes = [I32, P, I64, P, P, P, P, P, P, C.POINTER(P)]
         L.dda_build_matrix.restype = st
+        L.dda_build_matrix_reordered.argtypes = [I32, P, I64, P, P, P, P, P, P, C.POINTER(P)]
+        L.dda_build_matrix_reordered.restype = st
+        L.dda_hsbcsr_build.argtypes = [P, P, C.POINTER(P)]
+        L.dda_hsbcsr_build.restype = st
+        L.dda_hsbcsr_spmv.argtypes = [P, P, P, P]
+        L.dda_hsbcsr_spmv.restype = st
+        L.dda_hsbcsr_export.argtypes = [P, P, P, P]
+        L.dda_hsbcsr_export.restype = st
+        L.dda_hsbcsr_free.argtypes = [P]
+        L.dda_hsbcsr_free.restype = None
         L.dda_update_values.argtypes = [P, P, I64, P, P, P, P]
         L.dda_update_values.restype = st
         L.dda_matrix_info.argtypes = [P, C.POINTER(I32), C.POINTER(I64)]
@@ -289,17 +301,58 @@ class Matrix:
                "dda_update_values")
 
 
-def build_matrix(kdiag, bi, bj, pen, e, g, stream=None) -> Matrix:
-    """A1: assemble K from diagonal terms [n,6,6] and springs (bi, bj, pen, e[m,6], g[m,6])."""
+class HSBCSR:
+    """The paper's HSBCSR two-stage SpMV (dda_hsbcsr_*, NEXT-2 ablation) over a built Matrix."""
+
+    def __init__(self, K: "Matrix", stream=None):
+        self.K = K                       # the handle reads K's index arrays
+        h = C.c_void_p()
+        _check(lib().dda_hsbcsr_build(K.handle, C.c_void_p(_stream(stream)), C.byref(h)), "dda_hsbcsr_build")
+        self._h = h
+
+    def spmv(self, x, y=None, stream=None):
+        torch = _torch()
+        y = torch.empty_like(x) if y is None else y
+        N = 6 * self.K.n
+        _check(lib().dda_hsbcsr_spmv(self._h, _dev(x, torch.float64, (N,), "x"), _dev(y, torch.float64, (N,), "y"),
+                                     C.c_void_p(_stream(stream))), "dda_hsbcsr_spmv")
+        return y
+
+    def export(self):
+        """(d-data [6, dstride], nd-data-up [6, ustride]) host arrays."""
+        strides = np.zeros(2, np.int64)
+        _check(lib().dda_hsbcsr_export(self._h, None, None, strides.ctypes.data_as(C.c_void_p)), "dda_hsbcsr_export")
+        dd = np.zeros((6, int(strides[0])))
+        nd = np.zeros((6, max(int(strides[1]), 1)))
+        _check(lib().dda_hsbcsr_export(self._h, dd.ctypes.data_as(C.c_void_p), nd.ctypes.data_as(C.c_void_p),
+                                       strides.ctypes.data_as(C.c_void_p)), "dda_hsbcsr_export")
+        return dd, nd[:, :int(strides[1])]
+
+    def free(self):
+        if self._h is not None and _lib is not None:
+            _lib.dda_hsbcsr_free(self._h)
+        self._h = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def build_matrix(kdiag, bi, bj, pen, e, g, stream=None, reorder=False) -> Matrix:
+    """A1: assemble K from diagonal terms [n,6,6] and springs (bi, bj, pen, e[m,6], g[m,6]).
+    reorder=True: dda_build_matrix_reordered (internal RCM order, caller's numbering at the ABI)."""
     torch = _torch()
     n = int(kdiag.shape[0])
     m = int(bi.shape[0])
     h = C.c_void_p()
-    st = lib().dda_build_matrix(n, _dev(kdiag, torch.float64, (n, 6, 6), "kdiag"), m,
+    fn = lib().dda_build_matrix_reordered if reorder else lib().dda_build_matrix
+    st = fn(n, _dev(kdiag, torch.float64, (n, 6, 6), "kdiag"), m,
                                 _dev(bi, torch.int32, (m,), "bi"), _dev(bj, torch.int32, (m,), "bj"),
                                 _dev(pen, torch.float64, (m,), "pen"), _dev(e, torch.float64, (m, 6), "e"),
                                 _dev(g, torch.float64, (m, 6), "g"), C.c_void_p(_stream(stream)), C.byref(h))
-    _check(st, "dda_build_matrix")
+    _check(st, "dda_build_matrix_reordered" if reorder else "dda_build_matrix")
     return Matrix(h)
 
 

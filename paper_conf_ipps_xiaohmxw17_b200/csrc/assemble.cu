@@ -240,6 +240,8 @@ cudaError_t dmalloc(T** p, size_t count, cudaStream_t st) {
     return dev_alloc(reinterpret_cast<void**>(p), count ? count * sizeof(T) : 16, st);
 }
 
+}  // namespace
+
 dda_status_t run_values(dda_matrix* K, const double* kdiag, const double* pen, const double* e, const double* g,
                         cudaStream_t st) {
     if (K->nnzb > 0) {
@@ -260,8 +262,6 @@ dda_status_t run_values(dda_matrix* K, const double* kdiag, const double* pen, c
     return DDA_OK;
 }
 
-}  // namespace
-
 dda_status_t cuda_fail(cudaError_t e);
 
 }  // namespace dda
@@ -281,7 +281,7 @@ extern "C" void dda_matrix_free(dda_matrix_t K) {
     void* ptrs[] = {K->row_ptr, K->col_idx, K->low_ptr, K->low_row, K->low_to_up, K->urow, K->diag, K->upper,
                     K->perm, K->seg, K->dperm, K->dstart, K->orient, K->dinv, K->ws, K->scratch,
                     K->ilu_up, K->ilu_inv, K->ilu_flags, K->ilu_order, K->full_ptr, K->full_col, K->full_val,
-                    K->lfac, K->sfac, K->bj_w, K->sc_upper};
+                    K->lfac, K->sfac, K->bj_w, K->sc_upper, K->rperm, K->rinv, K->rtmp};
     for (void* p : ptrs)
         if (p) dev_free(p);
     cudaSetDevice(prev);
@@ -455,7 +455,8 @@ extern "C" dda_status_t dda_update_values(dda_matrix_t K, const double* kdiag, i
     if (!K || !kdiag || m != K->m) return DDA_ERR_ARG;
     if (m > 0 && (!pen || !e || !g)) return DDA_ERR_ARG;
     if (m > 0 && ((reinterpret_cast<uintptr_t>(e) | reinterpret_cast<uintptr_t>(g)) & 15)) return DDA_ERR_ARG;
-    return run_values(K, kdiag, pen, e, g, reinterpret_cast<cudaStream_t>(stream));
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    return K->rperm ? ro_update_values(K, kdiag, pen, e, g, st) : run_values(K, kdiag, pen, e, g, st);
 }
 
 extern "C" dda_status_t dda_matrix_info(dda_matrix_t K, int32_t* n, int64_t* nnzb) {
@@ -468,6 +469,12 @@ extern "C" dda_status_t dda_matrix_info(dda_matrix_t K, int32_t* n, int64_t* nnz
 extern "C" dda_status_t dda_matrix_export(dda_matrix_t K, int32_t* row_ptr, int32_t* col_idx, int32_t* low_ptr,
                                           int32_t* low_row, int32_t* low_to_up, double* diag, double* upper) {
     if (!K) return DDA_ERR_ARG;
+    if (K->rperm) return ro_export(K, row_ptr, col_idx, low_ptr, low_row, low_to_up, diag, upper);
+    return export_internal(K, row_ptr, col_idx, low_ptr, low_row, low_to_up, diag, upper);
+}
+
+dda_status_t dda::export_internal(dda_matrix* K, int32_t* row_ptr, int32_t* col_idx, int32_t* low_ptr,
+                                  int32_t* low_row, int32_t* low_to_up, double* diag, double* upper) {
     const size_t n1 = (size_t)K->n + 1, z = (size_t)K->nnzb;
     DDA_CK(cudaDeviceSynchronize());
     if (row_ptr) DDA_CK(cudaMemcpy(row_ptr, K->row_ptr, n1 * sizeof(int32_t), cudaMemcpyDeviceToHost));

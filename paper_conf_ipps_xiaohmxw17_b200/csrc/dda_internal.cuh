@@ -151,6 +151,11 @@ struct dda_matrix {
     double* full_val = nullptr;
     int64_t graph_iters = 0;        // loop-body launches issued inside graphs (launch accounting)
     int last_checks = 0;            // scaled engine: exact stopping tests in the last solve
+    // NEXT-2 internal block order (dda_build_matrix_reordered): the arrays above are in the internal
+    // (RCM) numbering; rperm[new] = user id, rinv[user] = new; vectors are permuted at the ABI
+    int32_t* rperm = nullptr;
+    int32_t* rinv = nullptr;
+    double* rtmp = nullptr;         // [3][6n] permuted vector scratch
 };
 
 // contact records of dda_detect_contacts (contact.cu) and the open-close state (openclose.cu)
@@ -180,6 +185,25 @@ dda_status_t build_matrix_impl(int32_t n, const double* kdiag, int64_t m, const 
                                const double* pen, const double* e, const double* g, cudaStream_t stream,
                                cudaEvent_t values_ready, dda_matrix_t* out);   // S_i V_ij S_j^T (needs lfac / sfac of every row)
 dda_status_t ilu_setup(dda_matrix* K, cudaStream_t st, int32_t* bad_block);
+dda_status_t bj_setup(dda_matrix* K, cudaStream_t st, int32_t* bad_block, double* full);
+dda_status_t run_values(dda_matrix* K, const double* kdiag, const double* pen, const double* e, const double* g,
+                        cudaStream_t st);
+dda_status_t spmv_full(dda_matrix* K, const double* x, double* y, cudaStream_t st);
+dda_status_t precond_apply(dda_matrix* K, dda_precond_t pc, double omega, const double* r, double* z, cudaStream_t st);
+dda_status_t pcg_entry(dda_matrix* K, const double* F, const double* d0, double* d, double tol, int32_t maxit,
+                       dda_precond_t pc, double omega, int32_t* iters, double* rel_res, cudaStream_t st);
+dda_status_t export_internal(dda_matrix* K, int32_t* row_ptr, int32_t* col_idx, int32_t* low_ptr, int32_t* low_row,
+                             int32_t* low_to_up, double* diag, double* upper);
+// reordered matrices (reorder.cu): the same operations in the caller's numbering
+dda_status_t ro_spmv(dda_matrix* K, const double* x, double* y, cudaStream_t st, bool full);
+dda_status_t ro_pcg(dda_matrix* K, const double* F, const double* d0, double* d, double tol, int32_t maxit,
+                    dda_precond_t pc, double omega, int32_t* iters, double* rel_res, cudaStream_t st);
+dda_status_t ro_precond(dda_matrix* K, dda_precond_t pc, double omega, const double* r, double* z, cudaStream_t st);
+dda_status_t ro_bj_setup(dda_matrix* K, double* dinv_full, int32_t* bad_block, cudaStream_t st);
+dda_status_t ro_update_values(dda_matrix* K, const double* kdiag, const double* pen, const double* e, const double* g,
+                              cudaStream_t st);
+dda_status_t ro_export(dda_matrix* K, int32_t* row_ptr, int32_t* col_idx, int32_t* low_ptr, int32_t* low_row,
+                       int32_t* low_to_up, double* diag, double* upper);
 dda_status_t ilu_apply(dda_matrix* K, const double* r, double* z, double* y, double* yh, cudaStream_t st);
 int ilu_grid();
 int comm_nparts(const dda_comm* c);                 // partitions of the communicator (NCCL: ranks)

@@ -598,6 +598,7 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
                                         const int32_t* send_counts, const int32_t* send_idx,
                                         const int32_t* recv_counts, void* stream) {
     if (!c || !K || !send_counts || !recv_counts) return DDA_ERR_ARG;
+    if (K->rperm) return DDA_ERR_ARG;            // partitions are built in their own local numbering
     const int P = c->nranks;
     const int slot = c->loopback ? part : 0;
     if (slot < 0 || slot >= (int)c->parts.size() || n_own < 1 || n_own > K->n) return DDA_ERR_ARG;

@@ -520,6 +520,13 @@ extern "C" dda_status_t dda_pcg_solve(dda_matrix_t K, const double* F, const dou
                                       double* rel_res, void* stream) {
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (!K) return DDA_ERR_ARG;
+    if (K->rperm) return dda::ro_pcg(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, st);
+    return dda::pcg_entry(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, st);
+}
+
+dda_status_t dda::pcg_entry(dda_matrix* K, const double* F, const double* d0, double* d, double tol, int32_t maxit,
+                            dda_precond_t pc, double omega, int32_t* iters, double* rel_res, cudaStream_t st) {
+    if (!K) return DDA_ERR_ARG;
     const int engine = pcg_engine(K, pc);
     if (engine == 1) return pcg_solve(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, st);
     if (iters) *iters = 0;

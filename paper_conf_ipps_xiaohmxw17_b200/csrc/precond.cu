@@ -219,13 +219,20 @@ using namespace dda;
 
 extern "C" dda_status_t dda_bj_setup(dda_matrix_t K, double* dinv_full, int32_t* bad_block, void* stream) {
     if (!K) return DDA_ERR_ARG;
-    return bj_setup(K, reinterpret_cast<cudaStream_t>(stream), bad_block, dinv_full);
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    if (K->rperm) return ro_bj_setup(K, dinv_full, bad_block, st);
+    return bj_setup(K, st, bad_block, dinv_full);
 }
 
 extern "C" dda_status_t dda_precond_apply(dda_matrix_t K, dda_precond_t pc, double omega, const double* r, double* z,
                                           void* stream) {
     if (!K || !r || !z || r == z) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    return K->rperm ? ro_precond(K, pc, omega, r, z, st) : dda::precond_apply(K, pc, omega, r, z, st);
+}
+
+dda_status_t dda::precond_apply(dda_matrix* K, dda_precond_t pc, double omega, const double* r, double* z,
+                                cudaStream_t st) {
     const size_t N = 6 * (size_t)K->n;
     if (pc == DDA_PC_NONE) {
         DDA_CK(cudaMemcpyAsync(z, r, N * sizeof(double), cudaMemcpyDeviceToDevice, st));

@@ -144,10 +144,7 @@ dda_status_t spmv(dda_matrix* K, const double* x, double* y, cudaStream_t s) {
 }  // namespace dda
 
 // configs[3]: full-storage BSR6 SpMV (every off-diagonal block stored twice), built on first use
-extern "C" dda_status_t dda_spmv_full(dda_matrix_t K, const double* x, double* y, void* stream) {
-    using namespace dda;
-    if (!K || !x || !y || x == y) return DDA_ERR_ARG;
-    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+dda_status_t dda::spmv_full(dda_matrix* K, const double* x, double* y, cudaStream_t st) {
     if (!K->full_ptr) {
         // allocate into locals and publish only when all three exist (a partial expansion must not
         // be taken for a built one on the next call)
@@ -183,7 +180,14 @@ extern "C" dda_status_t dda_spmv_full(dda_matrix_t K, const double* x, double* y
     return DDA_OK;
 }
 
+extern "C" dda_status_t dda_spmv_full(dda_matrix_t K, const double* x, double* y, void* stream) {
+    if (!K || !x || !y || x == y) return DDA_ERR_ARG;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    return K->rperm ? dda::ro_spmv(K, x, y, st, true) : dda::spmv_full(K, x, y, st);
+}
+
 extern "C" dda_status_t dda_spmv(dda_matrix_t K, const double* x, double* y, void* stream) {
     if (!K || !x || !y || x == y) return DDA_ERR_ARG;
-    return dda::spmv(K, x, y, reinterpret_cast<cudaStream_t>(stream));
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    return K->rperm ? dda::ro_spmv(K, x, y, st, false) : dda::spmv(K, x, y, st);
 }

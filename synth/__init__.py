@@ -7,7 +7,7 @@ diagonal terms and contact springs — from a seeded jittered-brick slope model
 its arrays; neither imports the other.
 """
 from .slope import (SlopeConfig, SlopeProblem, make_slope, preset, PRESETS,
-                    random_vector, warm_start)
+                    random_vector, warm_start, case1_like)
 
 __all__ = ["SlopeConfig", "SlopeProblem", "make_slope", "preset", "PRESETS",
-           "random_vector", "warm_start"]
+           "random_vector", "warm_start", "case1_like"]

@@ -330,3 +330,39 @@ def warm_start(d_ref: np.ndarray, seed: int, rel: float = 1e-3) -> np.ndarray:
     """Warm start d0 = d_ref * (1 + rel * N(0,1)) (ambiguity Z5)."""
     r = np.random.default_rng(seed).standard_normal(d_ref.shape)
     return d_ref * (1.0 + rel * r)
+
+
+def case1_like(seed: int = 1046, n_blocks: int = 4361, n_offdiag: int = 18731):
+    """A matrix input with the block counts of the paper's case 1 (4361 diagonal and 18731
+    upper off-diagonal sub-matrices, u = 4.3, denser than a brick wall's u ~ 3): the jittered slope
+    truncated to its first n_blocks blocks (springs between kept blocks only), plus one extra random
+    spring (random e, g of the slope's scale, the slope's normal penalty) on distinct new block pairs
+    (i, j), 2 <= j - i <= 3 * course length, drawn until there are exactly n_offdiag coupled pairs.
+    Input generation only; returns (n, kdiag, bi, bj, pen, e, g, F)."""
+    P = make_slope(preset(int(n_blocks * 1.05), seed=seed))
+    assert P.n >= n_blocks
+    keep = (P.bi < n_blocks) & (P.bj < n_blocks)
+    bi, bj = P.bi[keep].astype(np.int64), P.bj[keep].astype(np.int64)
+    pen, e, g = P.pen[keep], P.e[keep], P.g[keep]
+    pairs = set(zip(np.minimum(bi, bj).tolist(), np.maximum(bi, bj).tolist()))
+    assert len(pairs) <= n_offdiag
+    rng = np.random.default_rng(seed + 1)
+    L = int(np.bincount(P.course[:n_blocks]).max())
+    scale_e, scale_g = float(np.abs(e).mean()), float(np.abs(g).mean())
+    new_i, new_j = [], []
+    while len(pairs) < n_offdiag:
+        i = int(rng.integers(0, n_blocks - 2))
+        j = i + int(rng.integers(2, 3 * L + 1))
+        if j >= n_blocks or (i, j) in pairs:
+            continue
+        pairs.add((i, j))
+        new_i.append(i)
+        new_j.append(j)
+    k = len(new_i)
+    bi = np.concatenate([bi, new_i]).astype(np.int32)
+    bj = np.concatenate([bj, new_j]).astype(np.int32)
+    pen = np.concatenate([pen, np.full(k, float(P.pen.max()) / 1.2)])
+    e = np.ascontiguousarray(np.concatenate([e, rng.normal(0.0, scale_e, (k, 6))]))
+    g = np.ascontiguousarray(np.concatenate([g, rng.normal(0.0, scale_g, (k, 6))]))
+    F = np.ascontiguousarray(P.F[:6 * n_blocks])
+    return n_blocks, np.ascontiguousarray(P.kdiag[:n_blocks]), bi, bj, pen, e, g, F
