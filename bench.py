@@ -302,6 +302,8 @@ def main():
     ap.add_argument("--cpu-iter-sample", type=int, default=8, help="oracle PCG iterations timed (cpu_baseline)")
     ap.add_argument("--ref-iter-sample", type=int, default=4, help="oracle PCG iterations timed per reference step")
     ap.add_argument("--clock-period", type=float, default=0.05, help="NVML clock sampling period (s)")
+    ap.add_argument("--force-dist", action="store_true",
+                    help="run the partitioned (NCCL) path even at N = 1 (a check of the N > 1 code path)")
     args = ap.parse_args()
     if args.warmup < 3:
         print("warning: --warmup < 3 violates the timing rules; using 3", file=sys.stderr)
@@ -327,7 +329,12 @@ def main():
     from synth import make_slope, preset
 
     P = make_slope(preset(args.blocks, seed=1005))
-    if world > 1:
+    if world > 1 or args.force_dist:
+        if world == 1:
+            import torch.distributed as dist
+            os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+            os.environ.setdefault("MASTER_PORT", "29511")
+            dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", local))
         run_dist(args, P, world, rank, local)
         return
     t = dda.problem_to_device(P)
@@ -532,15 +539,30 @@ def run_dist(args, P, world, rank, local):
     pcg = statistics.mean(e[1].elapsed_time(e[2]) for e in evs)
     K, iters, rel_res, status = res[-1]
     assert status == dda.OK and rel_res <= 1.01e-10, (status, rel_res)
-    # v3 (block-Jacobi): the scaled engine per rank, 300u + 448 algorithmic bytes per own row and
-    # iteration as on one GPU; u over the rank's own rows
+    # v4 (block-Jacobi): the scaled engine per rank, 300u + 496 algorithmic bytes per own row and
+    # iteration (phase A 300u + 152, phase B 344); u over the rank's own rows
     info = comm.info(0, nparts=world)
     u = K.nnzb / max(n_own, 1)
-    local_bytes = n_own * (300.0 * u + 448.0) * iters
+    local_bytes = n_own * (300.0 * u + 496.0) * iters
     ach = local_bytes / (pcg * 1e-3) / 1e9
     tt = torch.tensor([ms, pcg, asm], device="cuda")
     dist.all_reduce(tt, op=dist.ReduceOp.MAX)
     ms, pcg_max, asm_max = (float(v) for v in tt.tolist())
+    # comm / compute split: one extra (untimed) solve with CUDA events between the steps of every
+    # iteration (halo exchange, phase A, allreduce, phase B; DDA_DIST_PROFILE=1), max over ranks
+    import ctypes as _C
+    os.environ["DDA_DIST_PROFILE"] = "1"
+    comm.pcg_solve([t["F"]], tol=1e-10, maxit=10000, precond=args.precond)
+    os.environ.pop("DDA_DIST_PROFILE")
+    prof = (_C.c_double * 4)()
+    fprof = dda.lib().dda__dist_profile
+    fprof.argtypes = [_C.c_void_p, _C.c_void_p]
+    fprof(comm._h, prof)
+    tp = torch.tensor(list(prof), device="cuda")
+    dist.all_reduce(tp, op=dist.ReduceOp.MAX)
+    split = {"halo_ms": float(tp[0]), "phaseA_ms": float(tp[1]), "allreduce_ms": float(tp[2]),
+             "phaseB_ms": float(tp[3]), "note": "per solve, summed over iterations, max over ranks; one profiled "
+                                                "(event-instrumented, untimed) solve"}
     # e2e: pinned host local inputs -> device, assemble, solve, d -> host (max over ranks)
     e2e = None
     if not args.no_e2e:
@@ -578,9 +600,11 @@ def run_dist(args, P, world, rank, local):
                                "dda_pcg_solve_dist",
                        "l2": "inputs larger than L2 per rank at 1M/N; no flush"},
             "phases_ms": {"assemble_max": asm_max, "pcg_max": pcg_max, "pcg_iters": iters,
-                          "pcg_us_per_iter": 1000.0 * pcg_max / max(iters, 1), "true_rel_res": rel_res},
-            "roofline": {"kernel": "rank 0: dist v3 scaled engine (k_v3_a fused p-update + Ks SpMV, k_v3_b, "
-                                   "one-thread scalar kernels; NCCL halo of r~ and p, device-buffer allreduces)",
+                          "pcg_us_per_iter": 1000.0 * pcg_max / max(iters, 1), "true_rel_res": rel_res,
+                          "comm_compute_split": split},
+            "roofline": {"kernel": "rank 0: dist v4 scaled engine (k_v4_a Ks SpMV + sigma / r~.q / q.q, k_v4_b "
+                                   "r~, p, x updates + stopping sums; one NCCL halo of p and one 6-double "
+                                   "allreduce per iteration)",
                          "bound": "hbm",
                          "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
                          "traffic": None, "peak_source": peak_src, "per": "GPU (rank 0)"},

@@ -473,6 +473,233 @@ __global__ void __launch_bounds__(DDA_THREADS) k_v3_final(int n, double* d, cons
     }
 }
 
+// ---- v4: one halo and one allreduce per iteration
+//
+// Iteration k on each partition (own rows), with p_k of own and halo rows in place:
+//   A_k  q = Ks p_k; partials sigma = p.q, r~.q, q.q                       -> scal[0..2]
+//   allreduce scal[0..5]   (slots 3..5 were written by B_{k-1}: |r~_k|^2, the w-bound, |L r~_k|^2)
+//   B_k  (every CTA derives the same scalars from the reduced sums)
+//        stopping test on r~_k (reading Z1 with the w-bound of the single-GPU engine; the exact
+//        |L r~_k|^2 was computed speculatively by B_{k-1} once the bound came within a factor 4 of
+//        the threshold; if it is missing, B_k only computes it and the next pass repeats A_k, B_k);
+//        alpha = rho_k / sigma with the exact rho_k = |r~_k|^2; beta = rho^_{k+1} / rho_k with
+//        rho^_{k+1} = rho_k - 2 alpha r~.q + alpha^2 q.q (the recurrence: rho_{k+1} itself is
+//        only reduced in the next allreduce);
+//        r~' = r~ - alpha q, p_{k+1} = r~' + beta p_k, x += alpha p_k; partials of r~'  -> scal[3..5]
+//   halo  of p_{k+1} (pack + one grouped send / receive)
+// Partial sums: every CTA writes its partials, the last CTA to arrive (ticket) adds them in CTA
+// order and writes the partition's slots: no separate reduction launch.  Per iteration: 3 kernels
+// (pack, A, B) and 2 NCCL calls (the halo group, the allreduce).
+struct S4 {
+    double rho, bnorm, tol, rr;
+    double alpha, beta, rho_hat;
+    int k, maxit, done, status, iters, checks, spec, retry;
+};
+
+// CTA partials -> part[k * G + cta]; the last CTA to arrive (ticket) writes out[k] = the sum over CTAs
+// in CTA order and returns true (in every thread of that CTA), after all other CTAs have finished
+template <int NV>
+__device__ __forceinline__ bool last_cta_sum(double (&v)[NV], double* part, int G, unsigned* ticket, double* out) {
+    __shared__ double red[NV][WPB];
+    __shared__ bool last;
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+#pragma unroll
+    for (int k = 0; k < NV; ++k) v[k] = warp_sum(v[k]);
+    if (lane == 0) {
+#pragma unroll
+        for (int k = 0; k < NV; ++k) red[k][wib] = v[k];
+    }
+    cta_barrier();
+    if (threadIdx.x == 0) {
+#pragma unroll
+        for (int k = 0; k < NV; ++k) {
+            double s = 0.0;
+            for (int w = 0; w < WPB; ++w) s += red[k][w];
+            part[k * G + blockIdx.x] = s;
+        }
+        __threadfence();
+        last = atomicAdd(ticket, 1u) == (unsigned)G - 1;
+    }
+    cta_barrier();
+    if (!last) return false;
+    __threadfence();
+    // the whole last CTA adds the G partials: strided per thread, then a fixed-shape tree
+    __shared__ double tr[NV][DDA_THREADS];
+#pragma unroll
+    for (int k = 0; k < NV; ++k) {
+        double s = 0.0;
+        for (int j = threadIdx.x; j < G; j += DDA_THREADS) s += __ldcg(part + k * G + j);
+        tr[k][threadIdx.x] = s;
+    }
+    cta_barrier();
+    for (int h = DDA_THREADS / 2; h > 0; h >>= 1) {
+        if (threadIdx.x < h) {
+#pragma unroll
+            for (int k = 0; k < NV; ++k) tr[k][threadIdx.x] += tr[k][threadIdx.x + h];
+        }
+        cta_barrier();
+    }
+    if (threadIdx.x < NV) out[threadIdx.x] = tr[threadIdx.x][0];
+    if (threadIdx.x == 0) *ticket = 0u;
+    return true;
+}
+
+// A_k: q = Ks p_k over own rows (p_k own + halo in P), partials sigma, r~.q, q.q -> scal[0..2]
+__global__ void __launch_bounds__(DDA_THREADS, 3) k_v4_a(BsrView A, const double* __restrict__ rt,
+                                                         const double* __restrict__ P, double* __restrict__ q,
+                                                         const S4* st, double* part, unsigned* ticket,
+                                                         double* scal) {
+    if (st->done) return;
+    const int lane = threadIdx.x & 31;
+    const XLdC xf{P};
+    double s0 = 0.0, s1 = 0.0, s2 = 0.0;
+    for_rows_c<SPMV_OFFDIAG, 5>(A, blockIdx.x * WPB + (threadIdx.x >> 5), gridDim.x * WPB, xf, lane,
+                                [&](int i, bool ok, double y0, double y1) {
+                                    if (ok) {
+                                        const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
+                                        const double2 pv = xf(i, ccol_of(lane));
+                                        y0 += pv.x;
+                                        y1 += pv.y;
+                                        *reinterpret_cast<double2*>(q + o) = make_double2(y0, y1);
+                                        const double2 rv = __ldg(reinterpret_cast<const double2*>(rt + o));
+                                        s0 += pv.x * y0 + pv.y * y1;
+                                        s1 += rv.x * y0 + rv.y * y1;
+                                        s2 += y0 * y0 + y1 * y1;
+                                    }
+                                });
+    double v[3] = {s0, s1, s2};
+    last_cta_sum<3>(v, part, gridDim.x, ticket, scal);
+}
+
+// B_k (see above); red = the allreduced scal[0..5].  Every CTA reads the state at entry and takes the
+// same decisions; only the last CTA (after all others have arrived) writes the state.
+__global__ void __launch_bounds__(DDA_THREADS) k_v4_b(int n, double* rt, double* P, const double* __restrict__ q,
+                                                      double* x, const double* __restrict__ w,
+                                                      const double* __restrict__ lfac, S4* st, const double* red,
+                                                      double* part, unsigned* ticket, double* scal) {
+    if (st->done) return;
+    const int k = st->k;
+    const int spec = st->spec;
+    const double thr = st->tol * st->bnorm;
+    // ---- the stopping test on r~_k (k = 0: decided at setup)
+    bool need_exact = false, stop = false;
+    double rho = st->rho;
+    if (k > 0) {
+        rho = red[3];
+        if (rho == 0.0) stop = true;
+        else if (isfinite(rho) && !(0.999 * red[4] > thr * thr)) {       // the bound allows convergence
+            if (spec) stop = sqrt(red[5]) <= thr;
+            else need_exact = true;
+        }
+    }
+    const double sigma = red[0];
+    const bool breakdown = !stop && !need_exact &&
+                           (!(sigma > 0.0) || !isfinite(sigma) || !(rho > 0.0) || !isfinite(rho));
+    const bool maxed = !stop && !need_exact && !breakdown && k >= st->maxit;
+    const bool finish = stop || breakdown || maxed;
+    const bool update = !finish && !need_exact;
+    const double alpha = rho / sigma;
+    const double rho_hat = rho - 2.0 * alpha * red[1] + alpha * alpha * red[2];
+    const double beta = rho_hat / rho;
+    // the exact norm of the NEXT residual is computed speculatively once the bound is within 4x
+    const bool spec_next = !(0.999 * red[4] > 16.0 * thr * thr);
+    const int lane = threadIdx.x & 31, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    double rz = 0.0, lb = 0.0, rl = 0.0;
+    if (!finish) {
+        const bool exact = need_exact || spec_next;
+        for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+            const Row5 R = row5(grp, lane, n);
+            double rv = 0.0;
+            if (R.valid) {
+                rv = rt[R.idx];
+                if (update) {          // r~' = r~ - alpha q, p' = r~' + beta p, x += alpha p
+                    const double pk = P[R.idx];
+                    rv = rv - alpha * q[R.idx];
+                    rt[R.idx] = rv;
+                    P[R.idx] = fma(beta, pk, rv);
+                    x[R.idx] = x[R.idx] + alpha * pk;
+                }
+                rz += rv * rv;
+                lb += __ldg(w + R.i) * (rv * rv);
+            }
+            if (exact) {               // uniform branch: every lane shuffles
+                const double o0 = tri_apply(lfac, R, rv, false);
+                const double o = R.valid ? o0 : 0.0;
+                rl += o * o;
+            }
+        }
+    }
+    // need_exact: r~_k is unchanged and its |r~|^2 and bound are recomputed bit-identically, so the
+    // next pass (A_k again, then B_k) finds the same sums plus the exact norm
+    double v[3] = {rz, lb, rl};
+    if (last_cta_sum<3>(v, part, gridDim.x, ticket, scal + 3) && threadIdx.x == 0) {
+        if (finish) {
+            st->done = 1;
+            st->status = stop ? DDA_OK : (breakdown ? DDA_ERR_BREAKDOWN : DDA_ERR_NO_CONVERGENCE);
+            st->iters = k;
+            if (k > 0 && spec && !(0.999 * red[4] > thr * thr)) { st->checks = st->checks + 1; st->rr = red[5]; }
+        } else if (need_exact) {
+            st->spec = 1;
+            st->retry = st->retry + 1;
+        } else {
+            if (k > 0 && spec && !(0.999 * red[4] > thr * thr)) { st->checks = st->checks + 1; st->rr = red[5]; }
+            st->alpha = alpha;
+            st->beta = beta;
+            st->rho_hat = rho_hat;
+            st->rho = rho;
+            st->k = k + 1;
+            st->iters = k + 1;
+            st->spec = spec_next ? 1 : 0;
+        }
+    }
+}
+
+// r = F - q (or F); r~ = S r -> rt and P (p_0); x = L^T d0 (or 0) -> d; scal[3] = |r~|^2, scal[4] =
+// the w-bound, scal[5] = |r|^2 (the exact test of r~_0), scal[6] = FF
+__global__ void __launch_bounds__(DDA_THREADS) k_v4_init(int n, const double* __restrict__ F,
+                                                         const double* __restrict__ q, const double* d0, double* d,
+                                                         const double* __restrict__ sfac,
+                                                         const double* __restrict__ lfac,
+                                                         const double* __restrict__ w, double* rt, double* P,
+                                                         double* part, unsigned* ticket, double* scal) {
+    const int lane = threadIdx.x & 31, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    double FF = 0, rr = 0, rz = 0, lb = 0;
+    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        double fv = 0.0, rv = 0.0, dv = 0.0;
+        if (R.valid) {
+            fv = F[R.idx];
+            rv = q ? fv - q[R.idx] : fv;
+            if (d0) dv = d0[R.idx];
+        }
+        FF += fv * fv;
+        rr += rv * rv;
+        const double t0 = tri_apply(sfac, R, rv, false);
+        const double t = R.valid ? t0 : 0.0;
+        const double x0 = tri_apply(lfac, R, dv, true);
+        if (R.valid) {
+            rt[R.idx] = t;
+            P[R.idx] = t;
+            d[R.idx] = d0 ? x0 : 0.0;
+            lb += __ldg(w + R.i) * (t * t);
+        }
+        rz += t * t;
+    }
+    double v[4] = {rz, lb, rr, FF};
+    last_cta_sum<4>(v, part, gridDim.x, ticket, scal + 3);
+}
+
+// d = S^T x (own rows; every x update was applied in B)
+__global__ void __launch_bounds__(DDA_THREADS) k_v4_final(int n, double* d, const double* __restrict__ sfac) {
+    const int lane = threadIdx.x & 31, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        const double xv = R.valid ? d[R.idx] : 0.0;
+        const double dv = tri_apply(sfac, R, xv, true);
+        if (R.valid) d[R.idx] = dv;
+    }
+}
+
 int grid_of(const void* k, int cap_per_sm) {
     int per = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k, DDA_THREADS, 0);
@@ -502,11 +729,14 @@ struct DistPart {
     void* dst = nullptr;         // device DState (v2)
     const double** scal_ptrs = nullptr;   // device [P] (loopback: every partition's scal)
     double *rt = nullptr, *pA = nullptr, *pB = nullptr;   // v3: r~, p ping-pong over local rows (own + halo)
+    unsigned* ticket = nullptr;  // v4: last-CTA ticket of the partial sums
     int G_spmv = 0, G_vec = 0, G_spmv2 = 0, G_a3 = 0;
 };
 
 struct dda_comm {
     bool loopback = false;
+    int last_checks = 0;         // v4: exact stopping tests of the last solve
+    double prof_ms[4] = {0, 0, 0, 0};   // v4 with DDA_DIST_PROFILE=1: halo, A, allreduce, B (summed, ms)
     int nranks = 1, rank = 0;    // NCCL: world; loopback: nranks = partitions, rank unused
     ncclComm_t nccl = nullptr;
     std::vector<DistPart> parts;
@@ -607,7 +837,7 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     if (D.K) {                                   // re-attach (e.g. a rebuilt matrix): release the old buffers
         cudaStreamSynchronize(st);
         void* ptrs[] = {D.send_idx, D.sendbuf, D.x, D.q, D.r, D.z, D.part, D.scal, D.red, D.dst,
-                        (void*)D.scal_ptrs, D.rt, D.pA, D.pB};
+                        (void*)D.scal_ptrs, D.rt, D.pA, D.pB, D.ticket};
         for (void* v : ptrs)
             if (v) dev_free(v);
         D = DistPart();
@@ -658,10 +888,16 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.q), no6 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.r), no6 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.z), no6 * sizeof(double), st));
-    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.part), 3 * (size_t)Gm * sizeof(double), st));
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.part), 4 * (size_t)Gm * sizeof(double), st));
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.ticket), sizeof(unsigned), st));
+    DDA_CK(cudaMemsetAsync(D.ticket, 0, sizeof(unsigned), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.scal), 8 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.red), 8 * sizeof(double), st));
-    DDA_CK(dev_alloc(&D.dst, sizeof(DState) > sizeof(SState) ? sizeof(DState) : sizeof(SState), st));
+    {
+        size_t ds = sizeof(DState) > sizeof(SState) ? sizeof(DState) : sizeof(SState);
+        if (sizeof(S4) > ds) ds = sizeof(S4);
+        DDA_CK(dev_alloc(&D.dst, ds, st));
+    }
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.rt), nl6 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.pA), nl6 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.pB), nl6 * sizeof(double), st));
@@ -761,6 +997,28 @@ dda_status_t allreduce_host(dda_comm* c, int nv, double* out, cudaStream_t st) {
     DistPart& D = c->parts[0];
     if (c->nranks > 1) DDA_NCCL(ncclAllReduce(D.scal, D.scal, nv, ncclDouble, ncclSum, c->nccl, st));
     DDA_CK(cudaMemcpyAsync(out, D.scal, nv * sizeof(double), cudaMemcpyDeviceToHost, st));
+    DDA_CK(cudaStreamSynchronize(st));
+    return DDA_OK;
+}
+
+// the sum over all partitions / ranks of D.scal[off .. off+nv), to the host; D.scal is not modified
+// (the NCCL sum goes to D.red)
+dda_status_t allreduce_host_at(dda_comm* c, int off, int nv, double* out, cudaStream_t st) {
+    for (int k = 0; k < nv; ++k) out[k] = 0.0;
+    if (c->loopback) {
+        std::vector<double> tmp(nv * c->parts.size());
+        for (size_t p = 0; p < c->parts.size(); ++p)
+            DDA_CK(cudaMemcpyAsync(tmp.data() + p * nv, c->parts[p].scal + off, nv * sizeof(double),
+                                   cudaMemcpyDeviceToHost, st));
+        DDA_CK(cudaStreamSynchronize(st));
+        for (size_t p = 0; p < c->parts.size(); ++p)
+            for (int k = 0; k < nv; ++k) out[k] += tmp[p * nv + k];
+        return DDA_OK;
+    }
+    DistPart& D = c->parts[0];
+    if (c->nranks > 1) DDA_NCCL(ncclAllReduce(D.scal + off, D.red, nv, ncclDouble, ncclSum, c->nccl, st));
+    else DDA_CK(cudaMemcpyAsync(D.red, D.scal + off, nv * sizeof(double), cudaMemcpyDeviceToDevice, st));
+    DDA_CK(cudaMemcpyAsync(out, D.red, nv * sizeof(double), cudaMemcpyDeviceToHost, st));
     DDA_CK(cudaStreamSynchronize(st));
     return DDA_OK;
 }
@@ -947,6 +1205,126 @@ dda_status_t dist_scaled_solve(dda_comm* c, const double* const* F, const double
     return DDA_OK;
 }
 
+// v4 solve (BJ, scaled engine per partition, one halo + one allreduce per iteration)
+dda_status_t dist_v4_solve(dda_comm* c, const double* const* F, const double* const* d0, double* const* d,
+                           double tol, int32_t maxit, dda_status_t* status, int* it, bool* zero, double* bnorm_out,
+                           int* checks_out, cudaStream_t st) {
+    *zero = false;
+    *it = 0;
+    DDA_TRY(halo_exchange_w(c, st, 4, kDinv));             // S_j of the halo rows
+    for (DistPart& D : c->parts) {
+        D.K->scaled_valid = false;
+        DDA_TRY(scaled_setup(D.K, st));
+    }
+    const bool have_d0 = d0 != nullptr;
+    if (have_d0) {                                          // q = K d0 over own rows (unscaled)
+        for (size_t p = 0; p < c->parts.size(); ++p) {
+            DistPart& D = c->parts[p];
+            if (d0[p]) DDA_CK(cudaMemcpyAsync(D.x, d0[p], 6 * sizeof(double) * D.n_own, cudaMemcpyDeviceToDevice, st));
+            else DDA_CK(cudaMemsetAsync(D.x, 0, 6 * sizeof(double) * D.n_own, st));
+        }
+        DDA_TRY(halo_exchange(c, st));
+        DDA_TRY(spmv_parts(c, false, st));
+    }
+    for (size_t p = 0; p < c->parts.size(); ++p) {
+        DistPart& D = c->parts[p];
+        k_v4_init<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, F[p], have_d0 ? D.q : nullptr,
+                                                   have_d0 ? d0[p] : nullptr, d[p], D.K->sfac, D.K->lfac,
+                                                   D.K->bj_w, D.rt, D.pA, D.part, D.ticket, D.scal);
+        DDA_LAUNCHED();
+    }
+    double s4[4];
+    DDA_TRY(allreduce_host_at(c, 3, 4, s4, st));
+    const double rho = s4[0], rr = s4[2], FF = s4[3], bnorm = std::sqrt(FF);
+    *bnorm_out = bnorm;
+    if (FF == 0.0) {                                        // reading Z2
+        for (size_t p = 0; p < c->parts.size(); ++p)
+            DDA_CK(cudaMemsetAsync(d[p], 0, 6 * sizeof(double) * c->parts[p].n_own, st));
+        DDA_CK(cudaStreamSynchronize(st));
+        *zero = true;
+        *status = DDA_OK;
+        return DDA_OK;
+    }
+    S4 h{};
+    h.rho = rho; h.bnorm = bnorm; h.tol = tol; h.rr = rr; h.maxit = maxit;
+    h.status = DDA_ERR_NO_CONVERGENCE;
+    if (std::sqrt(rr) <= tol * bnorm) { h.status = DDA_OK; h.done = 1; }
+    else if (!(rho > 0.0) || !std::isfinite(rho)) { h.status = DDA_ERR_BREAKDOWN; h.done = 1; }
+    else if (maxit <= 0) { h.done = 1; }
+    std::vector<const double*> sp;
+    for (DistPart& D : c->parts) sp.push_back(D.scal);
+    for (DistPart& D : c->parts) {
+        DDA_CK(cudaMemcpyAsync(D.dst, &h, sizeof h, cudaMemcpyHostToDevice, st));
+        if (c->loopback)
+            DDA_CK(cudaMemcpyAsync(D.scal_ptrs, sp.data(), sp.size() * sizeof(double*), cudaMemcpyHostToDevice, st));
+    }
+    int chunk = 8;
+    if (const char* e = getenv("DDA_DIST_CHUNK")) chunk = atoi(e) > 0 ? atoi(e) : 8;
+    S4 out = h;
+    // DDA_DIST_PROFILE=1: CUDA events between the four steps of every iteration (a diagnostic solve:
+    // the comm / compute split of bench.py's N > 1 line), summed per step
+    const char* pe = getenv("DDA_DIST_PROFILE");
+    const bool prof = pe && pe[0] == '1';
+    std::vector<cudaEvent_t> ev;
+    std::vector<int> ev_step;
+    for (int q = 0; q < 4; ++q) c->prof_ms[q] = 0.0;
+    auto mark = [&](int step) {
+        if (!prof) return;
+        cudaEvent_t e;
+        cudaEventCreate(&e);
+        cudaEventRecord(e, st);
+        ev.push_back(e);
+        ev_step.push_back(step);
+    };
+    // passes: maxit iterations + the pass that finds the final test + the rare exact-test retries
+    for (int k = 0; !out.done && k < maxit + 64; k += chunk) {
+        for (int ci = 0; ci < chunk; ++ci) {
+            mark(-1);
+            DDA_TRY(halo_exchange_w(c, st, 2, 6));                                   // p_k
+            mark(0);
+            for (DistPart& D : c->parts) {
+                k_v4_a<<<D.G_a3, DDA_THREADS, 0, st>>>(own_view_sc(D), D.rt, D.pA, D.q,
+                                                        reinterpret_cast<S4*>(D.dst), D.part, D.ticket, D.scal);
+                DDA_LAUNCHED();
+            }
+            mark(1);
+            DDA_TRY(allreduce_dev(c, 6, st));
+            mark(2);
+            for (size_t p = 0; p < c->parts.size(); ++p) {
+                DistPart& D = c->parts[p];
+                k_v4_b<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, D.rt, D.pA, D.q, d[p], D.K->bj_w, D.K->lfac,
+                                                        reinterpret_cast<S4*>(D.dst), D.red, D.part, D.ticket,
+                                                        D.scal);
+                DDA_LAUNCHED();
+            }
+            mark(3);
+        }
+        DDA_CK(cudaMemcpyAsync(&out, c->parts[0].dst, sizeof out, cudaMemcpyDeviceToHost, st));
+        DDA_CK(cudaStreamSynchronize(st));
+        if (prof) {
+            for (size_t q = 1; q < ev.size(); ++q) {
+                if (ev_step[q] < 0) continue;
+                float ms = 0.0f;
+                cudaEventElapsedTime(&ms, ev[q - 1], ev[q]);
+                c->prof_ms[ev_step[q]] += ms;
+            }
+            for (cudaEvent_t e : ev) cudaEventDestroy(e);
+            ev.clear();
+            ev_step.clear();
+        }
+    }
+    for (size_t p = 0; p < c->parts.size(); ++p) {          // d = S^T x
+        DistPart& D = c->parts[p];
+        k_v4_final<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, d[p], D.K->sfac);
+        DDA_LAUNCHED();
+    }
+    DDA_CK(cudaStreamSynchronize(st));
+    *status = out.done ? (dda_status_t)out.status : DDA_ERR_NO_CONVERGENCE;
+    *it = out.iters;
+    *checks_out = out.checks;
+    return DDA_OK;
+}
+
 }  // namespace
 
 extern "C" dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double* const* F, const double* const* d0,
@@ -962,14 +1340,19 @@ extern "C" dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double* const* F,
         if (!D.K) return DDA_ERR_ARG;
     if (use_bj)
         for (DistPart& D : c->parts) DDA_TRY(bj_setup_rows(D.K, D.n_own, st, nullptr));
-    // v3 (default for block-Jacobi): the scaled engine per partition; DDA_DIST_SCALED=0 selects v2
+    // v4 (default for block-Jacobi): one halo + one allreduce per iteration; DDA_DIST_VERSION=3 selects
+    // v3 (two halos, three allreduces); DDA_DIST_SCALED=0 selects the unscaled v2
     const char* dse = getenv("DDA_DIST_SCALED");
+    const char* dve = getenv("DDA_DIST_VERSION");
+    const bool v3 = dve && dve[0] == '3';
     if (use_bj && !(dse && dse[0] == '0')) {
         dda_status_t status = DDA_ERR_NO_CONVERGENCE;
-        int it = 0;
+        int it = 0, checks = 0;
         bool zero = false;
         double bnorm = 0.0;
-        DDA_TRY(dist_scaled_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, st));
+        if (v3) DDA_TRY(dist_scaled_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, st));
+        else DDA_TRY(dist_v4_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, &checks, st));
+        c->last_checks = checks;
         if (zero) return DDA_OK;
         // true residual ||F - K d|| / ||F|| (unscaled, over the partitions)
         for (size_t p = 0; p < c->parts.size(); ++p) {
@@ -1100,4 +1483,11 @@ extern "C" dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double* const* F,
     if (iters) *iters = it;
     if (rel_res) *rel_res = std::sqrt(res) / bnorm;
     return status;
+}
+
+// internal hook: the step times of the last profiled v4 solve (DDA_DIST_PROFILE=1): halo, A, allreduce, B
+extern "C" int dda__dist_profile(dda_comm_t c, double* ms4) {
+    if (!c || !ms4) return -1;
+    for (int q = 0; q < 4; ++q) ms4[q] = c->prof_ms[q];
+    return c->last_checks;
 }

@@ -60,14 +60,17 @@ def test_spmv_dist_loopback(dda, prob, nparts):
     assert (np.abs(y - yo) <= 1e-12 * bound).all()
 
 
-@pytest.fixture(params=["v3", "v2"])
+@pytest.fixture(params=["v4", "v3", "v2"])
 def dist_version(request, monkeypatch):
-    """v3 = the scaled block-Jacobi engine per partition (default); v2 = the unscaled loop
-    (DDA_DIST_SCALED=0, read by the library on every solve)."""
+    """v4 = the scaled block-Jacobi engine per partition with one halo and one allreduce per
+    iteration (default); v3 = the same engine with two halos and three allreduces
+    (DDA_DIST_VERSION=3); v2 = the unscaled loop (DDA_DIST_SCALED=0).  Read on every solve."""
+    monkeypatch.delenv("DDA_DIST_SCALED", raising=False)
+    monkeypatch.delenv("DDA_DIST_VERSION", raising=False)
     if request.param == "v2":
         monkeypatch.setenv("DDA_DIST_SCALED", "0")
-    else:
-        monkeypatch.delenv("DDA_DIST_SCALED", raising=False)
+    elif request.param == "v3":
+        monkeypatch.setenv("DDA_DIST_VERSION", "3")
     return request.param
 
 

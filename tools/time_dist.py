@@ -12,7 +12,7 @@ from synth import make_slope, preset
 n = int(sys.argv[1]) if len(sys.argv) > 1 else 1_000_000
 P = make_slope(preset(n, seed=1005))
 out = {}
-for nparts in (1, 2):
+for nparts in (1, 2, 4):
     b = dda.row_bounds(P.n, nparts)
     comm = dda.Comm.loopback(nparts)
     t = dda.problem_to_device(P)
@@ -23,14 +23,22 @@ for nparts in (1, 2):
                                    t["g"])
         keep.append(K)
         Fs.append(t["F"][6 * r0: 6 * r1].contiguous())
-    ms = []
-    for rep in range(4):
-        a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record()
-        ds, it, rr, st = comm.pcg_solve(Fs)
-        e.record(); torch.cuda.synchronize()
-        if rep: ms.append(a.elapsed_time(e))
-    out[nparts] = {"iters": it, "rel_res": rr, "status": st, "ms": statistics.median(ms),
-                   "us_per_iter": 1000 * statistics.median(ms) / it}
+    for ver in ("4", "3"):
+        os.environ["DDA_DIST_VERSION"] = ver
+        ms = []
+        for rep in range(4):
+            a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            ds, it, rr, st = comm.pcg_solve(Fs)
+            e.record(); torch.cuda.synchronize()
+            if rep: ms.append(a.elapsed_time(e))
+        out[f"P{nparts}_v{ver}"] = {"iters": it, "rel_res": rr, "status": st, "ms": statistics.median(ms),
+                                    "us_per_iter": 1000 * statistics.median(ms) / it}
     comm.free()
+# the single-GPU scaled engine on the same system, for reference
+Kg = dda.build_matrix(t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+Kg.pcg_solve(t["F"])
+a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+a.record(); _, it1, _, _ = Kg.pcg_solve(t["F"]); e.record(); torch.cuda.synchronize()
+out["single_gpu"] = {"iters": it1, "ms": a.elapsed_time(e), "us_per_iter": 1000 * a.elapsed_time(e) / it1}
 print(json.dumps({"n": P.n, "chunk": os.environ.get("DDA_DIST_CHUNK", "8"), "loopback": out}), flush=True)
