@@ -477,7 +477,7 @@ __global__ void __launch_bounds__(DDA_THREADS) k_v3_final(int n, double* d, cons
 //
 // Iteration k on each partition (own rows), with p_k of own and halo rows in place:
 //   A_k  q = Ks p_k; partials sigma = p.q, r~.q, q.q                       -> scal[0..2]
-//   allreduce scal[0..5]   (slots 3..5 were written by B_{k-1}: |r~_k|^2, the w-bound, |L r~_k|^2)
+//   allreduce scal[0..5]   (slots 3..5: B_{k-1}'s |r~_k|^2, w-bound, |L r~_k|^2, moved from 8..10 by A_k)
 //   B_k  (every CTA derives the same scalars from the reduced sums)
 //        stopping test on r~_k (reading Z1 with the w-bound of the single-GPU engine; the exact
 //        |L r~_k|^2 was computed speculatively by B_{k-1} once the bound came within a factor 4 of
@@ -544,14 +544,29 @@ __device__ __forceinline__ bool last_cta_sum(double (&v)[NV], double* part, int 
     return true;
 }
 
-// A_k: q = Ks p_k over own rows (p_k own + halo in P), partials sigma, r~.q, q.q -> scal[0..2]
-__global__ void __launch_bounds__(DDA_THREADS, 3) k_v4_a(BsrView A, const double* __restrict__ rt,
-                                                         const double* __restrict__ P, double* __restrict__ q,
-                                                         const S4* st, double* part, unsigned* ticket,
-                                                         double* scal) {
+// v5 (loopback): halo rows read straight from the owner partition's p (a pointer per halo row into
+// the owner's own rows) instead of a packed copy — the peer-load halo an NVLink-mapped multi-GPU
+// version performs over peer memory
+struct XPeer {
+    const double* __restrict__ x;             // own rows
+    const double* const* __restrict__ hsrc;   // [n_halo] the owner's row
+    int n_own;
+    using Raw = double2;
+    __device__ __forceinline__ Raw raw(int vec, int pair) const {
+        const double* row = vec < n_own ? x + 6 * (size_t)vec : hsrc[vec - n_own];
+        return __ldg(reinterpret_cast<const double2*>(row + 2 * pair));
+    }
+    __device__ __forceinline__ double2 cook(const Raw& r) const { return r; }
+    __device__ __forceinline__ double2 operator()(int vec, int pair) const { return raw(vec, pair); }
+};
+
+// A_k: q = Ks p_k over own rows (p_k own + halo through XL), partials sigma, r~.q, q.q -> scal[0..2]
+template <class XL>
+__global__ void __launch_bounds__(DDA_THREADS, 3) k_v4_a(BsrView A, const double* __restrict__ rt, const XL xf,
+                                                         double* __restrict__ q, const S4* st, double* part,
+                                                         unsigned* ticket, double* scal) {
     if (st->done) return;
     const int lane = threadIdx.x & 31;
-    const XLdC xf{P};
     double s0 = 0.0, s1 = 0.0, s2 = 0.0;
     for_rows_c<SPMV_OFFDIAG, 5>(A, blockIdx.x * WPB + (threadIdx.x >> 5), gridDim.x * WPB, xf, lane,
                                 [&](int i, bool ok, double y0, double y1) {
@@ -568,16 +583,31 @@ __global__ void __launch_bounds__(DDA_THREADS, 3) k_v4_a(BsrView A, const double
                                     }
                                 });
     double v[3] = {s0, s1, s2};
-    last_cta_sum<3>(v, part, gridDim.x, ticket, scal);
+    if (last_cta_sum<3>(v, part, gridDim.x, ticket, scal) && threadIdx.x < 3)
+        scal[3 + threadIdx.x] = scal[8 + threadIdx.x];    // B_{k-1}'s partials (written to 8..10)
 }
 
 // B_k (see above); red = the allreduced scal[0..5].  Every CTA reads the state at entry and takes the
 // same decisions; only the last CTA (after all others have arrived) writes the state.
+// red: the allreduced sums, or (red_all != null, v5) the sums of the partitions' slots red_all[p][0..5]
+// taken here in partition order: the one-shot allreduce, identical in every CTA of every partition
 __global__ void __launch_bounds__(DDA_THREADS) k_v4_b(int n, double* rt, double* P, const double* __restrict__ q,
                                                       double* x, const double* __restrict__ w,
-                                                      const double* __restrict__ lfac, S4* st, const double* red,
-                                                      double* part, unsigned* ticket, double* scal) {
+                                                      const double* __restrict__ lfac, S4* st, const double* red_in,
+                                                      const double* const* red_all, int nparts, double* part,
+                                                      unsigned* ticket, double* scal) {
     if (st->done) return;
+    __shared__ double red_sh[6];
+    const double* red = red_in;
+    if (red_all) {
+        if (threadIdx.x < 6) {
+            double s = 0.0;
+            for (int p = 0; p < nparts; ++p) s += red_all[p][threadIdx.x];
+            red_sh[threadIdx.x] = s;
+        }
+        __syncthreads();
+        red = red_sh;
+    }
     const int k = st->k;
     const int spec = st->spec;
     const double thr = st->tol * st->bnorm;
@@ -631,8 +661,10 @@ __global__ void __launch_bounds__(DDA_THREADS) k_v4_b(int n, double* rt, double*
     }
     // need_exact: r~_k is unchanged and its |r~|^2 and bound are recomputed bit-identically, so the
     // next pass (A_k again, then B_k) finds the same sums plus the exact norm
+    // the partials of the next residual go to slots 8..10; the next A moves them to 3..5 once every
+    // B of this pass has read 3..5 (the loopback one-shot sum reads the other partitions' slots)
     double v[3] = {rz, lb, rl};
-    if (last_cta_sum<3>(v, part, gridDim.x, ticket, scal + 3) && threadIdx.x == 0) {
+    if (last_cta_sum<3>(v, part, gridDim.x, ticket, scal + 8) && threadIdx.x == 0) {
         if (finish) {
             st->done = 1;
             st->status = stop ? DDA_OK : (breakdown ? DDA_ERR_BREAKDOWN : DDA_ERR_NO_CONVERGENCE);
@@ -686,7 +718,7 @@ __global__ void __launch_bounds__(DDA_THREADS) k_v4_init(int n, const double* __
         rz += t * t;
     }
     double v[4] = {rz, lb, rr, FF};
-    last_cta_sum<4>(v, part, gridDim.x, ticket, scal + 3);
+    last_cta_sum<4>(v, part, gridDim.x, ticket, scal + 8);  // slots 8..11 (A_0 moves 8..10 to 3..5)
 }
 
 // d = S^T x (own rows; every x update was applied in B)
@@ -730,6 +762,8 @@ struct DistPart {
     const double** scal_ptrs = nullptr;   // device [P] (loopback: every partition's scal)
     double *rt = nullptr, *pA = nullptr, *pB = nullptr;   // v3: r~, p ping-pong over local rows (own + halo)
     unsigned* ticket = nullptr;  // v4: last-CTA ticket of the partial sums
+    std::vector<int> h_send_idx; // host copy of send_idx (v5 peer tables)
+    const double** hsrc = nullptr;   // v5: [n_halo] device pointers to the owners' rows of p
     int G_spmv = 0, G_vec = 0, G_spmv2 = 0, G_a3 = 0;
 };
 
@@ -796,7 +830,7 @@ extern "C" void dda_comm_free(dda_comm_t c) {
     cudaDeviceSynchronize();
     for (DistPart& p : c->parts) {
         void* ptrs[] = {p.send_idx, p.sendbuf, p.x, p.q, p.r, p.z, p.part, p.scal, p.red, p.dst,
-                        (void*)p.scal_ptrs, p.rt, p.pA, p.pB};
+                        (void*)p.scal_ptrs, p.rt, p.pA, p.pB, p.ticket, (void*)p.hsrc};
         for (void* v : ptrs)
             if (v) dev_free(v);
     }
@@ -837,7 +871,7 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     if (D.K) {                                   // re-attach (e.g. a rebuilt matrix): release the old buffers
         cudaStreamSynchronize(st);
         void* ptrs[] = {D.send_idx, D.sendbuf, D.x, D.q, D.r, D.z, D.part, D.scal, D.red, D.dst,
-                        (void*)D.scal_ptrs, D.rt, D.pA, D.pB, D.ticket};
+                        (void*)D.scal_ptrs, D.rt, D.pA, D.pB, D.ticket, (void*)D.hsrc};
         for (void* v : ptrs)
             if (v) dev_free(v);
         D = DistPart();
@@ -864,6 +898,7 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
         D.recv_off[q + 1] = D.recv_off[q] + D.recv_counts[q];
     }
     D.n_send = D.send_off[P];
+    if (D.n_send && send_idx) D.h_send_idx.assign(send_idx, send_idx + D.n_send);
     if (D.recv_off[P] != K->n - n_own) return DDA_ERR_ARG;   // halo rows = received rows
     if (D.n_send && !send_idx) return DDA_ERR_ARG;
     const size_t nl6 = 6 * (size_t)K->n, no6 = 6 * (size_t)n_own;
@@ -891,7 +926,7 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.part), 4 * (size_t)Gm * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.ticket), sizeof(unsigned), st));
     DDA_CK(cudaMemsetAsync(D.ticket, 0, sizeof(unsigned), st));
-    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.scal), 8 * sizeof(double), st));
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.scal), 16 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.red), 8 * sizeof(double), st));
     {
         size_t ds = sizeof(DState) > sizeof(SState) ? sizeof(DState) : sizeof(SState);
@@ -1234,7 +1269,7 @@ dda_status_t dist_v4_solve(dda_comm* c, const double* const* F, const double* co
         DDA_LAUNCHED();
     }
     double s4[4];
-    DDA_TRY(allreduce_host_at(c, 3, 4, s4, st));
+    DDA_TRY(allreduce_host_at(c, 8, 4, s4, st));
     const double rho = s4[0], rr = s4[2], FF = s4[3], bnorm = std::sqrt(FF);
     *bnorm_out = bnorm;
     if (FF == 0.0) {                                        // reading Z2
@@ -1258,6 +1293,28 @@ dda_status_t dist_v4_solve(dda_comm* c, const double* const* F, const double* co
         if (c->loopback)
             DDA_CK(cudaMemcpyAsync(D.scal_ptrs, sp.data(), sp.size() * sizeof(double*), cudaMemcpyHostToDevice, st));
     }
+    // v5 (loopback, default there; DDA_DIST_VERSION=4 keeps the copies): halo by peer loads, one-shot
+    // allreduce inside B.  The pointer tables follow the exchange plan: halo row recv_off[q] + t of p
+    // is q's own row send_idx_q[send_off_q[p] + t]
+    const char* dve = getenv("DDA_DIST_VERSION");
+    const bool peer = c->loopback && !(dve && dve[0] == '4');
+    if (peer) {
+        const int P = (int)c->parts.size();
+        for (int p = 0; p < P; ++p) {
+            DistPart& D = c->parts[p];
+            const int nh = D.n_local - D.n_own;
+            if (!D.hsrc) DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.hsrc), (nh + 1) * sizeof(double*), st));
+            std::vector<const double*> tab(nh + 1, nullptr);
+            for (int q = 0; q < P; ++q) {
+                if (q == p) continue;
+                const DistPart& S = c->parts[q];
+                for (int t = 0; t < D.recv_counts[q]; ++t)
+                    tab[D.recv_off[q] + t] = S.pA + 6 * (size_t)S.h_send_idx[S.send_off[p] + t];
+            }
+            DDA_CK(cudaMemcpyAsync(D.hsrc, tab.data(), (nh + 1) * sizeof(double*), cudaMemcpyHostToDevice, st));
+        }
+        DDA_CK(cudaStreamSynchronize(st));                  // the host table must outlive the copies
+    }
     int chunk = 8;
     if (const char* e = getenv("DDA_DIST_CHUNK")) chunk = atoi(e) > 0 ? atoi(e) : 8;
     S4 out = h;
@@ -1280,21 +1337,31 @@ dda_status_t dist_v4_solve(dda_comm* c, const double* const* F, const double* co
     for (int k = 0; !out.done && k < maxit + 64; k += chunk) {
         for (int ci = 0; ci < chunk; ++ci) {
             mark(-1);
-            DDA_TRY(halo_exchange_w(c, st, 2, 6));                                   // p_k
+            if (!peer) DDA_TRY(halo_exchange_w(c, st, 2, 6));                        // p_k
             mark(0);
             for (DistPart& D : c->parts) {
-                k_v4_a<<<D.G_a3, DDA_THREADS, 0, st>>>(own_view_sc(D), D.rt, D.pA, D.q,
-                                                        reinterpret_cast<S4*>(D.dst), D.part, D.ticket, D.scal);
+                if (peer) {
+                    const XPeer xf{D.pA, D.hsrc, D.n_own};
+                    k_v4_a<XPeer><<<D.G_a3, DDA_THREADS, 0, st>>>(own_view_sc(D), D.rt, xf, D.q,
+                                                                  reinterpret_cast<S4*>(D.dst), D.part, D.ticket,
+                                                                  D.scal);
+                } else {
+                    const XLdC xf{D.pA};
+                    k_v4_a<XLdC><<<D.G_a3, DDA_THREADS, 0, st>>>(own_view_sc(D), D.rt, xf, D.q,
+                                                                 reinterpret_cast<S4*>(D.dst), D.part, D.ticket,
+                                                                 D.scal);
+                }
                 DDA_LAUNCHED();
             }
             mark(1);
-            DDA_TRY(allreduce_dev(c, 6, st));
+            if (!peer) DDA_TRY(allreduce_dev(c, 6, st));
             mark(2);
             for (size_t p = 0; p < c->parts.size(); ++p) {
                 DistPart& D = c->parts[p];
                 k_v4_b<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, D.rt, D.pA, D.q, d[p], D.K->bj_w, D.K->lfac,
-                                                        reinterpret_cast<S4*>(D.dst), D.red, D.part, D.ticket,
-                                                        D.scal);
+                                                        reinterpret_cast<S4*>(D.dst), D.red,
+                                                        peer ? D.scal_ptrs : nullptr, (int)c->parts.size(),
+                                                        D.part, D.ticket, D.scal);
                 DDA_LAUNCHED();
             }
             mark(3);

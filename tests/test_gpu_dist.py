@@ -60,17 +60,18 @@ def test_spmv_dist_loopback(dda, prob, nparts):
     assert (np.abs(y - yo) <= 1e-12 * bound).all()
 
 
-@pytest.fixture(params=["v4", "v3", "v2"])
+@pytest.fixture(params=["v5", "v4", "v3", "v2"])
 def dist_version(request, monkeypatch):
-    """v4 = the scaled block-Jacobi engine per partition with one halo and one allreduce per
-    iteration (default); v3 = the same engine with two halos and three allreduces
+    """v5 = the v4 iteration with the halo read from the owners' rows (peer loads) and the allreduce
+    taken inside phase B (loopback default); v4 = one halo copy and one allreduce per iteration
+    (DDA_DIST_VERSION=4; the NCCL transport always runs it); v3 = two halos and three allreduces
     (DDA_DIST_VERSION=3); v2 = the unscaled loop (DDA_DIST_SCALED=0).  Read on every solve."""
     monkeypatch.delenv("DDA_DIST_SCALED", raising=False)
     monkeypatch.delenv("DDA_DIST_VERSION", raising=False)
     if request.param == "v2":
         monkeypatch.setenv("DDA_DIST_SCALED", "0")
-    elif request.param == "v3":
-        monkeypatch.setenv("DDA_DIST_VERSION", "3")
+    elif request.param in ("v3", "v4"):
+        monkeypatch.setenv("DDA_DIST_VERSION", request.param[1])
     return request.param
 
 

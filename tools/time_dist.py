@@ -23,7 +23,7 @@ for nparts in (1, 2, 4):
                                    t["g"])
         keep.append(K)
         Fs.append(t["F"][6 * r0: 6 * r1].contiguous())
-    for ver in ("4", "3"):
+    for ver in ("5", "4", "3"):
         os.environ["DDA_DIST_VERSION"] = ver
         ms = []
         for rep in range(4):
