@@ -412,6 +412,16 @@ void dda_contacts_free(dda_contacts_t C);
  *   (total), converged (1 / 0) and rel_res (last solve) are host outputs.  DDA_ERR_ARG for a set
  *   that is not classified and initialised (dda_contact_init).  Synchronising.
  */
+/*
+ * NEXT-3 contact transfer (§III.B; reading N3-4, the oracle's O-13): for every record k of the
+ * current set `cur`, state[k] (device int32 [cur count]) becomes prev_state[j] (device, [prev count])
+ * of the previous step's record j with the same (vertex v, edge e) pair, and keeps its value (e.g.
+ * the initial state of dda_contact_init) when there is none.  The previous records are radix-sorted
+ * by (v, e) and searched ("sorted search").  matched (host, may be NULL): records transferred.
+ * Synchronising.
+ */
+dda_status_t dda_contact_transfer(dda_contacts_t prev, const int32_t *prev_state, dda_contacts_t cur, int32_t *state,
+                                  int64_t *matched, void *stream);
 dda_status_t dda_contact_init(dda_contacts_t C, int32_t *state, void *stream);
 dda_status_t dda_contact_loads(dda_contacts_t C, const double *e, const double *g, const double *pen, const double *F,
                                double *out, void *stream);

@@ -70,6 +70,8 @@ def lib():
                                           C.c_double, P, P, P, P, P]
         L.orc_contact_springs.restype = C.c_int64
         L.orc_classify_contacts.argtypes = [C.c_int32, P, P, C.c_int64, P, P, P, P, P, C.c_double, P]
+        L.orc_contact_transfer.argtypes = [C.c_int64, P, P, P, C.c_int64, P, P, P, P]
+        L.orc_contact_transfer.restype = C.c_int64
         L.orc_contact_loads.argtypes = [C.c_int32, P, P, C.c_int64, P, P, P, P, P, P, P, P, P]
         L.orc_contact_check.argtypes = [C.c_int32, P, P, C.c_int64, P, P, P, P, P, P, P, P, C.c_double,
                                         C.c_double, C.c_double, C.c_double, P, P, P]
@@ -392,3 +394,15 @@ def open_close_loop(n, kdiag, F, vptr, vxy, cxy, Cc, p_n, shear_ratio, tan_phi, 
         if counts[1] + counts[2] + counts[4] + counts[5] == 0:
             return d, state, hist, True
     return d, state, hist, False
+
+
+def contact_transfer(prev, prev_state, cur, init_state):
+    """O-13: the states of the current records, transferred from the previous step's record with the
+    same (v, e), else the initial state.  Returns (state, matched)."""
+    pv, pe = np.ascontiguousarray(prev["v"], np.int32), np.ascontiguousarray(prev["e"], np.int32)
+    cv, ce = np.ascontiguousarray(cur["v"], np.int32), np.ascontiguousarray(cur["e"], np.int32)
+    ps = np.ascontiguousarray(prev_state, np.int32)
+    ini = np.ascontiguousarray(init_state, np.int32)
+    out = np.empty(max(cv.size, 1), np.int32)
+    matched = lib().orc_contact_transfer(pv.size, _p(pv), _p(pe), _p(ps), cv.size, _p(cv), _p(ce), _p(ini), _p(out))
+    return out[:cv.size], int(matched)

@@ -899,3 +899,26 @@ int orc_contact_loads(int32_t n, const int32_t *vptr, const double *vxy, int64_t
     }
     return ORC_OK;
 }
+
+/*
+ * O-13 (NEXT-3)  Contact transfer (§III.B: "each contact of the previous step will
+ * search the contacts of the current step; if their contact data are the same, then the contact
+ * status parameter ... of the previous step [is] transferred to the current step").  Reading N3-4:
+ * the contact data of a record are its (vertex v, edge e) pair (global vertex / edge ids, stable
+ * across steps); the transferred parameter is the open-close state.  For every current record k:
+ * state[k] = prev_state[j] for the previous record j with the same (v, e), else init[k] (the
+ * gap-based initial state of O-12).  Plain search over the previous records.  Returns the number of
+ * matched records.
+ */
+int64_t orc_contact_transfer(int64_t n_prev, const int32_t *pv, const int32_t *pe, const int32_t *pstate,
+                             int64_t n_cur, const int32_t *cv, const int32_t *ce, const int32_t *init,
+                             int32_t *state) {
+    int64_t matched = 0;
+    for (int64_t k = 0; k < n_cur; ++k) {
+        int32_t s = init[k];
+        for (int64_t j = 0; j < n_prev; ++j)
+            if (pv[j] == cv[k] && pe[j] == ce[k]) { s = pstate[j]; ++matched; break; }
+        state[k] = s;
+    }
+    return matched;
+}

@@ -33,7 +33,7 @@ ABI_SYMBOLS = ("dda_build_matrix", "dda_update_values", "dda_matrix_info", "dda_
                "dda_dist_info", "dda_classify_contacts", "dda_contacts_classes",
                "dda_contact_init", "dda_contact_loads", "dda_contact_check", "dda_open_close",
                "dda_build_matrix_reordered", "dda_hsbcsr_build", "dda_hsbcsr_spmv", "dda_hsbcsr_export",
-               "dda_hsbcsr_free")
+               "dda_hsbcsr_free", "dda_contact_transfer")
 
 _lib = None
 
@@ -132,6 +132,8 @@ def lib() -> C.CDLL:
         L.dda_classify_contacts.restype = st
         L.dda_contacts_classes.argtypes = [P, P, P, P, P]
         L.dda_contacts_classes.restype = st
+        L.dda_contact_transfer.argtypes = [P, P, P, P, P, P]
+        L.dda_contact_transfer.restype = st
         L.dda_contact_init.argtypes = [P, P, P]
         L.dda_contact_init.restype = st
         L.dda_contact_loads.argtypes = [P, P, P, P, P, P, P]
@@ -575,6 +577,15 @@ class Contacts:
         _check(lib().dda_contact_init(self._h, C.c_void_p(state.data_ptr()), C.c_void_p(_stream(stream))),
                "dda_contact_init")
         return state[:self.count]
+
+    def transfer_from(self, prev: "Contacts", prev_state, state, stream=None) -> int:
+        """dda_contact_transfer: state (CUDA int32 [count], in: initial, out: transferred) of this set
+        from the previous step's set and states; returns the number of transferred records."""
+        mt = C.c_int64()
+        _check(lib().dda_contact_transfer(prev._h, C.c_void_p(prev_state.data_ptr()), self._h,
+                                          C.c_void_p(state.data_ptr()), C.cast(C.byref(mt), C.c_void_p),
+                                          C.c_void_p(_stream(stream))), "dda_contact_transfer")
+        return int(mt.value)
 
     def loads(self, sp, pen, F=None, stream=None):
         """dda_contact_loads: F (or 0) + the gap load of the closed normal springs (CUDA [6n])."""

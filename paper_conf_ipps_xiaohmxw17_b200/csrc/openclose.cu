@@ -339,3 +339,74 @@ extern "C" dda_status_t dda_open_close(dda_matrix_t K, dda_contacts_t C, const d
     }
     return DDA_OK;
 }
+
+// ---- contact transfer (NEXT-3; reading N3-4; the oracle's O-13): the previous step's records
+// sorted by their (v, e) key (radix sort), then a binary search per current record ("sorted search")
+namespace dda {
+namespace {
+
+__global__ void k_tr_keys(int64_t m, const int32_t* __restrict__ v, const int32_t* __restrict__ e,
+                          uint64_t* __restrict__ key, int32_t* __restrict__ idx) {
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < m; k += (int64_t)gridDim.x * blockDim.x) {
+        key[k] = ((uint64_t)(uint32_t)v[k] << 32) | (uint32_t)e[k];
+        idx[k] = (int32_t)k;
+    }
+}
+
+__global__ void k_tr_search(int64_t m, const int32_t* __restrict__ v, const int32_t* __restrict__ e, int64_t mp,
+                            const uint64_t* __restrict__ skey, const int32_t* __restrict__ sidx,
+                            const int32_t* __restrict__ pstate, int32_t* __restrict__ state,
+                            unsigned long long* __restrict__ matched) {
+    unsigned long long cnt = 0;
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < m; k += (int64_t)gridDim.x * blockDim.x) {
+        const uint64_t key = ((uint64_t)(uint32_t)v[k] << 32) | (uint32_t)e[k];
+        int64_t lo = 0, hi = mp;
+        while (lo < hi) {
+            const int64_t mid = (lo + hi) >> 1;
+            if (skey[mid] < key) lo = mid + 1; else hi = mid;
+        }
+        if (lo < mp && skey[lo] == key) {
+            state[k] = pstate[sidx[lo]];
+            ++cnt;
+        }
+    }
+    if (cnt) atomicAdd(matched, cnt);   // a count (integer): order-independent
+}
+
+}  // namespace
+}  // namespace dda
+
+extern "C" dda_status_t dda_contact_transfer(dda_contacts_t prev, const int32_t* prev_state, dda_contacts_t cur,
+                                             int32_t* state, int64_t* matched, void* stream) {
+    using namespace dda;
+    if (!prev || !cur || (prev->count > 0 && !prev_state) || (cur->count > 0 && !state)) return DDA_ERR_ARG;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    const int64_t mp = prev->count, m = cur->count;
+    OTmp tmp(st);
+    uint64_t *key = nullptr, *skey = nullptr;
+    int32_t *idx = nullptr, *sidx = nullptr;
+    unsigned long long* cnt = nullptr;
+    DDA_CK(tmp.get(&key, mp));
+    DDA_CK(tmp.get(&skey, mp));
+    DDA_CK(tmp.get(&idx, mp));
+    DDA_CK(tmp.get(&sidx, mp));
+    DDA_CK(tmp.get(&cnt, 1));
+    DDA_CK(cudaMemsetAsync(cnt, 0, sizeof(unsigned long long), st));
+    if (mp > 0 && m > 0) {
+        k_tr_keys<<<ogrid(mp), OT, 0, st>>>(mp, prev->cv, prev->ce, key, idx);
+        DDA_LAUNCHED();
+        size_t tb = 0;
+        DDA_CK(cub::DeviceRadixSort::SortPairs(nullptr, tb, key, skey, idx, sidx, (int)mp, 0, 64, st));
+        char* ts = nullptr;
+        DDA_CK(tmp.get(&ts, tb));
+        DDA_CK(cub::DeviceRadixSort::SortPairs(ts, tb, key, skey, idx, sidx, (int)mp, 0, 64, st));
+        note_launch(4);
+        k_tr_search<<<ogrid(m), OT, 0, st>>>(m, cur->cv, cur->ce, mp, skey, sidx, prev_state, state, cnt);
+        DDA_LAUNCHED();
+    }
+    unsigned long long h = 0;
+    DDA_CK(cudaMemcpyAsync(&h, cnt, sizeof h, cudaMemcpyDeviceToHost, st));
+    DDA_CK(cudaStreamSynchronize(st));
+    if (matched) *matched = (int64_t)h;
+    return DDA_OK;
+}

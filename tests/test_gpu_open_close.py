@@ -166,3 +166,26 @@ def test_check_full_size_sampled(dda):
     Fg = Cg.loads(sp, torch.from_numpy(pen_all).cuda()).cpu().numpy()
     idx = (6 * blocks[:, None] + np.arange(6)).reshape(-1)
     assert np.array_equal(Fg[idx], Fo[idx])
+
+
+def test_contact_transfer_vs_oracle(dda):
+    """NEXT-3 contact transfer: states of a perturbed next step (contacts within 0.35 h) from the
+    previous step's converged states (contacts within 0.1 h), against O-13, bit-exact, matched count."""
+    P, vptr, vxy, F = _slope(1000)
+    Cg, sp = _gpu_set(dda, vptr, vxy, P.centroid, 0.1, STOL, P_N, SR)
+    state = Cg.init_states()
+    kd = torch.from_numpy(P.kdiag).cuda()
+    K = dda.build_matrix(kd, sp["bi"], sp["bj"], sp["pen"], sp["e"], sp["g"])
+    _, state, _, oc, _, conv, _ = Cg.open_close(K, kd, torch.from_numpy(F).cuda(), sp, state, p_n=P_N,
+                                                shear_ratio=SR, tan_phi=TPHI, open_tol=OTOL)
+    assert conv
+    rng = np.random.default_rng(3)
+    vxy2 = vxy + rng.uniform(-0.05, 0.05, vxy.shape)
+    C2, sp2 = _gpu_set(dda, vptr, vxy2, P.centroid, 0.35, STOL, P_N, SR)
+    st2 = C2.init_states()
+    init = st2.cpu().numpy().copy()
+    matched = C2.transfer_from(Cg, state, st2)
+    O1, O2 = Cg.export(), C2.export()
+    want, mo = oracle.contact_transfer(O1, state.cpu().numpy(), O2, init)
+    assert np.array_equal(st2.cpu().numpy(), want) and matched == mo
+    assert 0 < matched < C2.count

@@ -124,3 +124,36 @@ def test_open_close_loop_1k_converges():
     d, st, hist, conv = oracle.open_close_loop(P.n, P.kdiag, F, vptr, vxy, P.centroid, Cc, 40.0, 0.4, 0.577, 0.01)
     assert conv and len(hist) <= 15
     assert (st == 0).any() and (st == 1).any() and (st == 2).any()
+
+
+# ------------------------------------------------------------------ O-13: contact transfer
+
+def _perturbed(P, scale, seed):
+    """The slope's polygons moved by a small random displacement (the next step's geometry)."""
+    rng = np.random.default_rng(seed)
+    return P.verts.reshape(-1, 2) + rng.uniform(-scale, scale, (P.n * 4, 2))
+
+
+def test_contact_transfer_against_brute_force():
+    P, vptr, vxy, F, _ = _slope_case()
+    # step 1: the contacts within 0.1 h, their converged open-close states
+    Cc = oracle.classified_contacts(vptr, vxy, oracle.detect_contacts(vptr, vxy, 0.1), 0.35)
+    d, st, hist, conv = oracle.open_close_loop(P.n, P.kdiag, F, vptr, vxy, P.centroid, Cc, 40.0, 0.4, 0.577, 0.01)
+    assert conv
+    # step 2: moved polygons, contacts within 0.35 h: most persist, some are new
+    vxy2 = _perturbed(P, 0.05, 3)
+    C2 = oracle.classified_contacts(vptr, vxy2, oracle.detect_contacts(vptr, vxy2, 0.35), 0.35)
+    sp2 = oracle.classified_springs(vptr, vxy2, P.centroid, C2, 40.0, 0.4)
+    _, init = oracle.contact_loads(P.n, vptr, vxy2, C2, sp2["e"], sp2["g"], None)
+    got, matched = oracle.contact_transfer(Cc, st, C2, init)
+    prev = {(int(v), int(e)): int(s) for v, e, s in zip(Cc["v"], Cc["e"], st)}
+    want = np.array([prev.get((int(v), int(e)), int(s0)) for v, e, s0 in zip(C2["v"], C2["e"], init)])
+    assert np.array_equal(got, want)
+    assert matched == sum((int(v), int(e)) in prev for v, e in zip(C2["v"], C2["e"]))
+    assert 0 < matched < C2["v"].size                      # some contacts persist, some are new
+    # the identity step transfers everything; an empty previous step transfers nothing
+    same, mt = oracle.contact_transfer(Cc, st, Cc, np.zeros_like(st))
+    assert np.array_equal(same, st) and mt == st.size
+    empty = {k: v[:0] for k, v in Cc.items()}
+    none, m0 = oracle.contact_transfer(empty, st[:0], C2, init)
+    assert np.array_equal(none, init) and m0 == 0
