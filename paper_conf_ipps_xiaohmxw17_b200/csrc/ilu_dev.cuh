@@ -82,14 +82,25 @@ __device__ __forceinline__ double row_sum(const BsrView& A, const double* __rest
     return (a & 1) ? hi : lo;
 }
 
-// w_a = sum_c Finv_i[a][c] v_c, v on lanes 0..5 (full tiled pivot inverse)
-__device__ __forceinline__ double pivot_apply(const double* __restrict__ Finv, int i, double v, int lane) {
+// row a = lane (lanes 0..5) of the tiled pivot inverse U_ii^{-1}: independent of the dependencies,
+// so it is loaded before the warp waits for them (off the critical path of the sweep)
+struct PivRow {
+    double v[6];
+};
+__device__ __forceinline__ PivRow pivot_row(const double* __restrict__ Finv, int i, int lane) {
     const int a = lane < 6 ? lane : 0;
+    PivRow p;
+#pragma unroll
+    for (int c = 0; c < 6; ++c) p.v[c] = __ldg(Finv + (size_t)kBlk * i + tile_off(a, c));
+    return p;
+}
+// w_a = sum_c Finv_i[a][c] v_c, v on lanes 0..5
+__device__ __forceinline__ double pivot_apply(const PivRow& F, double v) {
     double s = 0.0;
 #pragma unroll
     for (int c = 0; c < 6; ++c) {
         const double vc = __shfl_sync(0xffffffffu, v, c);
-        s = fma(Finv[(size_t)kBlk * i + tile_off(a, c)], vc, s);
+        s = fma(F.v[c], vc, s);
     }
     return s;
 }
@@ -99,16 +110,18 @@ __device__ __forceinline__ void ilu_forward_rows(const BsrView& A, const double*
                                  double* yh, int* flags, int* counter, const int* order) {
     const int lane = threadIdx.x & 31;
     for (int i = next_row(counter, order, A.n, lane); i < A.n; i = next_row(counter, order, A.n, lane)) {
+        const PivRow F = pivot_row(Finv, i, lane);
+        const double ri = (lane < 6) ? r[6 * (size_t)i + lane] : 0.0;
         const double s = row_sum<true>(A, Fup, i, yh, flags, lane);
-        const double yi = (lane < 6) ? r[6 * (size_t)i + lane] - s : 0.0;
-        const double hi = pivot_apply(Finv, i, yi, lane);
+        const double yi = (lane < 6) ? ri - s : 0.0;
+        const double hi = pivot_apply(F, yi);
         if (lane < 6) {
             y[6 * (size_t)i + lane] = yi;
             yh[6 * (size_t)i + lane] = hi;
         }
-        __syncwarp();
-        if (lane == 0) {
-            __threadfence();
+        __syncwarp();                       // the six stores of the row precede the release (st.release.gpu
+        if (lane == 0) {                    // orders this thread's earlier writes; the warp's via __syncwarp
+            __threadfence();                // plus this fence, which makes them visible at gpu scope)
             st_release(flags + i, 1);
         }
     }
@@ -121,9 +134,11 @@ __device__ __forceinline__ double ilu_backward_rows(const BsrView& A, const doub
     const int lane = threadIdx.x & 31;
     double rz = 0.0;
     for (int i = next_row(counter, order, A.n, lane); i < A.n; i = next_row(counter, order, A.n, lane)) {
+        const PivRow F = pivot_row(Finv, i, lane);
+        const double yi = (lane < 6) ? y[6 * (size_t)i + lane] : 0.0;
         const double s = row_sum<false>(A, Fup, i, z, flags, lane);
-        const double t = (lane < 6) ? y[6 * (size_t)i + lane] - s : 0.0;
-        const double zi = pivot_apply(Finv, i, t, lane);
+        const double t = (lane < 6) ? yi - s : 0.0;
+        const double zi = pivot_apply(F, t);
         if (lane < 6) {
             z[6 * (size_t)i + lane] = zi;
             if (p_init) p_init[6 * (size_t)i + lane] = zi;

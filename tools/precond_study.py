@@ -5,6 +5,8 @@ import json, os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
 import paper_conf_ipps_xiaohmxw17_b200 as dda
+if os.environ.get("DDA_LIB_PATH"):          # A/B against another build of the library
+    dda.LIB_PATH = os.environ["DDA_LIB_PATH"]
 from synth import make_slope, preset
 
 
