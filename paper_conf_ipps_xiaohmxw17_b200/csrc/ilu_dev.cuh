@@ -45,8 +45,9 @@ __device__ __forceinline__ double row_sum(const BsrView& A, const double* __rest
     double4 a_pre = make_double4(0.0, 0.0, 0.0, 0.0);
     if (lane < 27 && g < nb)
         a_pre = ld_chunk(vals + (size_t)kBlk * (LOWER ? A.low_to_up[b0 + g] : b0 + g) + 4 * (LOWER ? 3 * C + R : q));
-    if (lane == 0)
-        for (int b = 0; b < nb; ++b) wait_ready(flags, deps[b0 + b]);
+    // the dependencies are polled in parallel, one lane each (a sequential poll costs one L2 round
+    // trip per dependency even when all are ready)
+    for (int b = lane; b < nb; b += 32) wait_ready(flags, deps[b0 + b]);
     __syncwarp();
     double f0 = 0.0, f1 = 0.0;
     for (int b = g; b < nb + 2; b += 3) {       // every lane iterates equally (nb + 2 >= g)
