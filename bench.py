@@ -64,6 +64,24 @@ def traffic_for(n_blocks: int, which: str):
         return None
 
 
+def l2_roofline(n_blocks: int, iters: int, pcg_ms: float):
+    """The secondary (L2) roofline of the PCG loop: its L2 sector traffic per iteration from the committed
+    ncu capture of k_sp_loop (profiles/traffic.json "sp_loop_l2"), times the iterations of this solve,
+    over the solve's CUDA-event time, against the practical L2 (LTS) throughput cap of the
+    microarchitecture guide (~6.3 kB per SM-clock cycle at the SM clock of the capture)."""
+    try:
+        t = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
+        e = t["sp_loop_l2"]
+        if int(t.get("n_blocks", -1)) != n_blocks:
+            return None
+    except Exception:
+        return None
+    tbps = e["l2_bytes_per_iter"] * iters / (pcg_ms * 1e-3) / 1e12
+    cap = e["lts_cap_bytes_per_cycle"] * e["sm_clock_hz"] / 1e12
+    return {"l2_bytes_per_iter": e["l2_bytes_per_iter"], "achieved_tbps": tbps, "cap_tbps": cap,
+            "frac": tbps / cap, "source": e["source"]}
+
+
 def bytes_per_row_spmv(u: float) -> float:
     """Algorithmic bytes of one symmetric SpMV per block row:
     D 288 + u*(V 288 + col 4 + low_row 4 + low_to_up 4) + row_ptr/low_ptr 8 + x 48 + y 48."""
@@ -475,7 +493,7 @@ def main():
         "roofline": {"kernel": pcg_kernel, "engine": engine,
                      "bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
                      "traffic": traffic_for(n, "pcg_" + str(engine)), "peak_source": peak_src,
-                     "algorithmic_bytes_per_launch": pcg_bytes},
+                     "algorithmic_bytes_per_launch": pcg_bytes, "l2": l2_roofline(n, iters, pcg_ms)},
         "spmv": {"kernel": "k_spmv<FULL,6>", "ms": spmv_ms, "traffic": traffic_for(n, "spmv"), "gbs": spmv_gbs, "frac_hbm": spmv_gbs / hbm_peak,
                  "gflops": n * (72 + 144 * u) / (spmv_ms * 1e-3) / 1e9, "bytes": spmv_bytes,
                  "timing": "back to back (hot), inputs > L2"},
