@@ -561,15 +561,19 @@ struct XPeer {
 };
 
 // A_k: q = Ks p_k over own rows (p_k own + halo through XL), partials sigma, r~.q, q.q -> scal[0..2]
+// rows: logical range [t0, t1) mapped as in for_rows_cr (t1 < 0: every own row).  mode 0: the only
+// launch (sums -> scal[0..2], moves 8..10 -> 3..5); mode 1: the interior launch of the halo overlap
+// (sums -> scal[12..14]); mode 2: the boundary launch (scal[0..2] = scal[12..14] + its sums, in that
+// order, and the move)
 template <class XL>
 __global__ void __launch_bounds__(DDA_THREADS, 3) k_v4_a(BsrView A, const double* __restrict__ rt, const XL xf,
                                                          double* __restrict__ q, const S4* st, double* part,
-                                                         unsigned* ticket, double* scal) {
+                                                         unsigned* ticket, double* scal, int t0, int t1, int ilo,
+                                                         int gap, int mode) {
     if (st->done) return;
     const int lane = threadIdx.x & 31;
     double s0 = 0.0, s1 = 0.0, s2 = 0.0;
-    for_rows_c<SPMV_OFFDIAG, 5>(A, blockIdx.x * WPB + (threadIdx.x >> 5), gridDim.x * WPB, xf, lane,
-                                [&](int i, bool ok, double y0, double y1) {
+    auto rowA = [&](int i, bool ok, double y0, double y1) {
                                     if (ok) {
                                         const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
                                         const double2 pv = xf(i, ccol_of(lane));
@@ -581,10 +585,28 @@ __global__ void __launch_bounds__(DDA_THREADS, 3) k_v4_a(BsrView A, const double
                                         s1 += rv.x * y0 + rv.y * y1;
                                         s2 += y0 * y0 + y1 * y1;
                                     }
-                                });
+                                };
+    const int w0 = blockIdx.x * WPB + (threadIdx.x >> 5), W = gridDim.x * WPB;
+    if (t1 < 0) for_rows_c<SPMV_OFFDIAG, 5>(A, w0, W, xf, lane, rowA);
+    else for_rows_cr<SPMV_OFFDIAG>(A, t0, t1, ilo, gap, w0, W, xf, lane, rowA);
     double v[3] = {s0, s1, s2};
-    if (last_cta_sum<3>(v, part, gridDim.x, ticket, scal) && threadIdx.x < 3)
+    double* out = mode == 1 ? scal + 12 : (mode == 2 ? scal + 16 : scal);
+    if (last_cta_sum<3>(v, part, gridDim.x, ticket, out) && mode != 1 && threadIdx.x < 3) {
+        if (mode == 2) scal[threadIdx.x] = scal[12 + threadIdx.x] + scal[16 + threadIdx.x];
         scal[3 + threadIdx.x] = scal[8 + threadIdx.x];    // B_{k-1}'s partials (written to 8..10)
+    }
+}
+
+// flag[i] = own row i references a halo row (a forward column or a transposed source >= n_own)
+__global__ void k_boundary_rows(int n_own, const int32_t* __restrict__ row_ptr, const int32_t* __restrict__ col,
+                                const int32_t* __restrict__ low_ptr, const int32_t* __restrict__ low_row,
+                                uint8_t* __restrict__ flag) {
+    for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n_own; i += gridDim.x * blockDim.x) {
+        bool b = false;
+        for (int u = row_ptr[i]; u < row_ptr[i + 1]; ++u) b = b || col[u] >= n_own;
+        for (int t = low_ptr[i]; t < low_ptr[i + 1]; ++t) b = b || low_row[t] >= n_own;
+        flag[i] = b ? 1 : 0;
+    }
 }
 
 // B_k (see above); red = the allreduced scal[0..5].  Every CTA reads the state at entry and takes the
@@ -762,6 +784,8 @@ struct DistPart {
     const double** scal_ptrs = nullptr;   // device [P] (loopback: every partition's scal)
     double *rt = nullptr, *pA = nullptr, *pB = nullptr;   // v3: r~, p ping-pong over local rows (own + halo)
     unsigned* ticket = nullptr;  // v4: last-CTA ticket of the partial sums
+    unsigned* ticket2 = nullptr; // v4 halo overlap: the interior launch's ticket
+    int ilo = 0, ihi = 0;        // v4 halo overlap: the longest run of own rows that read no halo row
     std::vector<int> h_send_idx; // host copy of send_idx (v5 peer tables)
     const double** hsrc = nullptr;   // v5: [n_halo] device pointers to the owners' rows of p
     int G_spmv = 0, G_vec = 0, G_spmv2 = 0, G_a3 = 0;
@@ -830,7 +854,7 @@ extern "C" void dda_comm_free(dda_comm_t c) {
     cudaDeviceSynchronize();
     for (DistPart& p : c->parts) {
         void* ptrs[] = {p.send_idx, p.sendbuf, p.x, p.q, p.r, p.z, p.part, p.scal, p.red, p.dst,
-                        (void*)p.scal_ptrs, p.rt, p.pA, p.pB, p.ticket, (void*)p.hsrc};
+                        (void*)p.scal_ptrs, p.rt, p.pA, p.pB, p.ticket, (void*)p.hsrc, p.ticket2};
         for (void* v : ptrs)
             if (v) dev_free(v);
     }
@@ -871,7 +895,7 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     if (D.K) {                                   // re-attach (e.g. a rebuilt matrix): release the old buffers
         cudaStreamSynchronize(st);
         void* ptrs[] = {D.send_idx, D.sendbuf, D.x, D.q, D.r, D.z, D.part, D.scal, D.red, D.dst,
-                        (void*)D.scal_ptrs, D.rt, D.pA, D.pB, D.ticket, (void*)D.hsrc};
+                        (void*)D.scal_ptrs, D.rt, D.pA, D.pB, D.ticket, (void*)D.hsrc, D.ticket2};
         for (void* v : ptrs)
             if (v) dev_free(v);
         D = DistPart();
@@ -926,6 +950,29 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.part), 4 * (size_t)Gm * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.ticket), sizeof(unsigned), st));
     DDA_CK(cudaMemsetAsync(D.ticket, 0, sizeof(unsigned), st));
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.ticket2), sizeof(unsigned), st));
+    DDA_CK(cudaMemsetAsync(D.ticket2, 0, sizeof(unsigned), st));
+    {   // the interior rows for the halo overlap: the longest run of rows that read no halo row
+        uint8_t* flag = nullptr;
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&flag), (size_t)n_own + 1, st));
+        k_boundary_rows<<<(n_own + 255) / 256, 256, 0, st>>>(n_own, K->row_ptr, K->col_idx, K->low_ptr, K->low_row,
+                                                            flag);
+        DDA_LAUNCHED();
+        std::vector<uint8_t> hf(n_own);
+        DDA_CK(cudaMemcpyAsync(hf.data(), flag, n_own, cudaMemcpyDeviceToHost, st));
+        DDA_CK(cudaStreamSynchronize(st));
+        dev_free_on(flag, st);
+        int best_lo = 0, best_len = 0;
+        for (int i = 0; i < n_own;) {
+            if (hf[i]) { ++i; continue; }
+            int j = i;
+            while (j < n_own && !hf[j]) ++j;
+            if (j - i > best_len) { best_len = j - i; best_lo = i; }
+            i = j;
+        }
+        D.ilo = best_lo;
+        D.ihi = best_lo + best_len;
+    }
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.scal), 16 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.red), 8 * sizeof(double), st));
     {
@@ -1315,6 +1362,26 @@ dda_status_t dist_v4_solve(dda_comm* c, const double* const* F, const double* co
         }
         DDA_CK(cudaStreamSynchronize(st));                  // the host table must outlive the copies
     }
+    // halo overlap (v4 with halo copies or NCCL; DDA_DIST_OVERLAP=0 disables): phase A of the interior
+    // rows runs while the halo is in flight on a second stream
+    const char* ove = getenv("DDA_DIST_OVERLAP");
+    bool overlap = !peer && !(ove && ove[0] == '0');
+    if (overlap) {
+        bool any_halo = false;
+        for (DistPart& D : c->parts) any_halo = any_halo || D.n_local > D.n_own;
+        overlap = any_halo;
+    }
+    cudaStream_t cs = nullptr;
+    cudaEvent_t ev_a = nullptr, ev_b = nullptr;
+    struct StreamGuard {
+        cudaStream_t& s; cudaEvent_t& a; cudaEvent_t& b;
+        ~StreamGuard() { if (a) cudaEventDestroy(a); if (b) cudaEventDestroy(b); if (s) cudaStreamDestroy(s); }
+    } sguard{cs, ev_a, ev_b};
+    if (overlap) {
+        DDA_CK(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+        DDA_CK(cudaEventCreateWithFlags(&ev_a, cudaEventDisableTiming));
+        DDA_CK(cudaEventCreateWithFlags(&ev_b, cudaEventDisableTiming));
+    }
     int chunk = 8;
     if (const char* e = getenv("DDA_DIST_CHUNK")) chunk = atoi(e) > 0 ? atoi(e) : 8;
     S4 out = h;
@@ -1337,21 +1404,47 @@ dda_status_t dist_v4_solve(dda_comm* c, const double* const* F, const double* co
     for (int k = 0; !out.done && k < maxit + 64; k += chunk) {
         for (int ci = 0; ci < chunk; ++ci) {
             mark(-1);
-            if (!peer) DDA_TRY(halo_exchange_w(c, st, 2, 6));                        // p_k
-            mark(0);
-            for (DistPart& D : c->parts) {
-                if (peer) {
-                    const XPeer xf{D.pA, D.hsrc, D.n_own};
-                    k_v4_a<XPeer><<<D.G_a3, DDA_THREADS, 0, st>>>(own_view_sc(D), D.rt, xf, D.q,
-                                                                  reinterpret_cast<S4*>(D.dst), D.part, D.ticket,
-                                                                  D.scal);
-                } else {
+            if (overlap) {
+                // the halo of p_k on the comm stream while the interior rows (which read no halo row)
+                // run phase A; then the boundary rows
+                DDA_CK(cudaEventRecord(ev_a, st));
+                DDA_CK(cudaStreamWaitEvent(cs, ev_a, 0));
+                DDA_TRY(halo_exchange_w(c, cs, 2, 6));
+                DDA_CK(cudaEventRecord(ev_b, cs));
+                for (DistPart& D : c->parts) {
                     const XLdC xf{D.pA};
                     k_v4_a<XLdC><<<D.G_a3, DDA_THREADS, 0, st>>>(own_view_sc(D), D.rt, xf, D.q,
-                                                                 reinterpret_cast<S4*>(D.dst), D.part, D.ticket,
-                                                                 D.scal);
+                                                                 reinterpret_cast<S4*>(D.dst), D.part, D.ticket2,
+                                                                 D.scal, D.ilo, D.ihi, D.ihi, 0, 1);
+                    DDA_LAUNCHED();
                 }
-                DDA_LAUNCHED();
+                mark(0);
+                DDA_CK(cudaStreamWaitEvent(st, ev_b, 0));
+                for (DistPart& D : c->parts) {
+                    const XLdC xf{D.pA};
+                    const int gap = D.ihi - D.ilo;
+                    k_v4_a<XLdC><<<D.G_a3, DDA_THREADS, 0, st>>>(own_view_sc(D), D.rt, xf, D.q,
+                                                                 reinterpret_cast<S4*>(D.dst), D.part, D.ticket,
+                                                                 D.scal, 0, D.n_own - gap, D.ilo, gap, 2);
+                    DDA_LAUNCHED();
+                }
+            } else {
+                if (!peer) DDA_TRY(halo_exchange_w(c, st, 2, 6));                    // p_k
+                mark(0);
+                for (DistPart& D : c->parts) {
+                    if (peer) {
+                        const XPeer xf{D.pA, D.hsrc, D.n_own};
+                        k_v4_a<XPeer><<<D.G_a3, DDA_THREADS, 0, st>>>(own_view_sc(D), D.rt, xf, D.q,
+                                                                      reinterpret_cast<S4*>(D.dst), D.part,
+                                                                      D.ticket, D.scal, 0, -1, 0, 0, 0);
+                    } else {
+                        const XLdC xf{D.pA};
+                        k_v4_a<XLdC><<<D.G_a3, DDA_THREADS, 0, st>>>(own_view_sc(D), D.rt, xf, D.q,
+                                                                     reinterpret_cast<S4*>(D.dst), D.part,
+                                                                     D.ticket, D.scal, 0, -1, 0, 0, 0);
+                    }
+                    DDA_LAUNCHED();
+                }
             }
             mark(1);
             if (!peer) DDA_TRY(allreduce_dev(c, 6, st));

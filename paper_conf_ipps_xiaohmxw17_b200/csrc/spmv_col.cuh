@@ -244,4 +244,28 @@ __device__ __forceinline__ void for_rows_c(const BsrView& A, int w, int W, const
     }
 }
 
+// for_rows_c over a row subset: logical rows t in [t0, t1) (ten per warp step, warp-strided), mapped to
+// matrix rows i = t < ilo ? t : t + gap — the interior range [ilo, ihi) of a partition with gap = 0
+// (t0 = ilo, t1 = ihi), or the rows around it with gap = ihi - ilo (t0 = 0, t1 = n - gap)
+template <int MODE, class XLoad, class Body>
+__device__ __forceinline__ void for_rows_cr(const BsrView& A, int t0, int t1, int ilo, int gap, int w, int W,
+                                            const XLoad& xload, int lane, const Body& body) {
+    const int h = cgrp_of(lane);
+    const bool lane_ok = lane < 30;
+    auto row_of = [&](int t) { return t < ilo ? t : t + gap; };
+    int t = t0 + 10 * w + h;
+    RowBounds nxt = row_bounds<MODE>(A, row_of(t), lane_ok && t < t1);
+    for (int base = t0 + 10 * w; base < t1; base += 10 * W) {
+        t = base + h;
+        const bool ok = lane_ok && t < t1;
+        const int i = ok ? row_of(t) : A.n;
+        const RowBounds cur = nxt;
+        const int tn = t + 10 * W;
+        nxt = row_bounds<MODE>(A, row_of(tn), lane_ok && tn < t1);
+        double y0, y1;
+        spmv_row_c5<MODE>(A, i, ok, cur, xload, lane, y0, y1);
+        body(i, ok, y0, y1);
+    }
+}
+
 }  // namespace dda

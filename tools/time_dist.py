@@ -23,8 +23,9 @@ for nparts in (1, 2, 4):
                                    t["g"])
         keep.append(K)
         Fs.append(t["F"][6 * r0: 6 * r1].contiguous())
-    for ver in ("5", "4", "3"):
-        os.environ["DDA_DIST_VERSION"] = ver
+    for ver in ("5", "4", "4s", "3"):
+        os.environ["DDA_DIST_VERSION"] = ver[0]
+        os.environ["DDA_DIST_OVERLAP"] = "0" if ver == "4s" else "1"
         ms = []
         for rep in range(4):
             a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)

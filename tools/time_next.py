@@ -85,6 +85,15 @@ if "openclose" in what:
     # check: per contact e, g of two springs (4 x 48 B), two 48 B rows of d, gap, state r/w, pen and
     # category writes (2 x 8 + 4), sort keys / values (8); the category sort is extra
     b_chk = m * (4 * 48 + 2 * 48 + 8 + 8 + 16 + 4 + 8)
+    # contact transfer to the next step (the same polygons moved by U(-0.01, 0.01) h)
+    vxy2 = vxy + (torch.rand_like(vxy) - 0.5) * 0.02
+    C2 = dda.detect_contacts(vptr, vxy2, 0.2)
+    C2.classify(0.35)
+    st2 = C2.init_states()
+    t_tr = timed(lambda: C2.transfer_from(C, st, st2.clone()))
+    matched = C2.transfer_from(C, st, st2)
+    print(json.dumps({"row": "NEXT-3 transfer", "prev": C.count, "cur": C2.count, "matched": matched,
+                      "transfer_ms": t_tr}), flush=True)
     print(json.dumps({"row": "NEXT-4", "blocks": P.n, "contacts": m, "converged": conv, "oc_iters": oc,
                       "pcg_iters_total": pit, "loop_ms": loop_ms, "final_states": {"open": int(counts[0]),
                       "slide": int(counts[1]), "lock": int(counts[2])}, "rel_res_last": rr,
