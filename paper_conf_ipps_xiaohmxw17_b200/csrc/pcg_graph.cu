@@ -57,7 +57,7 @@ struct GArgs {           // constant for a (matrix, preconditioner): baked into 
     BsrView A;
     const double* dinv;
     double *r, *z, *p0, *p1, *q, *t, *w;
-    double* part;        // [4][Gmax] CTA partials
+    double* part;        // [8][Gmax] CTA partials
     int Gmax;
     int pc;
     State* st;
@@ -1032,6 +1032,152 @@ __device__ __forceinline__ double exact_rr_pass(const GArgs& a, const double* rn
     return rl;
 }
 
+// ---- scaled BJ, single-reduction variant (Chronopoulos-Gear CG on Ks; A/B tuning aid, DDA_SCALED_CG1=1)
+//
+// The same Krylov iterates in exact arithmetic with ONE grid barrier per iteration instead of two:
+// s = Ks r is carried instead of q = Ks p (q_k = s_k + beta_k q_{k-1}), so the SpMV operand of pass k
+// is r_{k+1} = r_k - alpha_k (s_k + beta_k q_{k-1}), formed on the fly from vectors of pass k - 1,
+// and both inner products of the next step (rho = r.r, mu = r.s) come out of the same pass:
+//   beta_{k+1} = rho_{k+1} / rho_k,  alpha_{k+1} = rho_{k+1} / (mu_{k+1} - beta_{k+1} rho_{k+1} / alpha_k).
+// Pass k per row: q_k, p_k (own), x += alpha_k p_k, r_{k+1}, s_{k+1} = Ks r_{k+1}; partials rho, mu, w-bound.
+// r, s, q are ping-ponged (neighbours read pass k - 1's values while owners write pass k's); p and
+// x are own-row only and updated in place.  Partial slots alternate between passes (1-3 / 4-6) so a
+// fast CTA never overwrites partials a slow CTA is still summing; phase C keeps slot 0.
+struct XCg1 {   // r_{k+1} = r_k - alpha (s_k + beta q_{k-1}) (first pass: q_0 = s_0)
+    const double *r, *s, *q;
+    double alpha, beta;
+    bool first;
+    using Raw = double2;
+    __device__ __forceinline__ Raw raw(int vec, int pair) const {
+        const size_t o = 6 * (size_t)vec + 2 * pair;
+        const double2 rr = ld_cg2(r + o), ss = ld_cg2(s + o);
+        double2 qk = ss;
+        if (!first) {
+            const double2 qq = ld_cg2(q + o);
+            qk = make_double2(fma(beta, qq.x, ss.x), fma(beta, qq.y, ss.y));
+        }
+        return make_double2(fma(-alpha, qk.x, rr.x), fma(-alpha, qk.y, rr.y));
+    }
+    __device__ __forceinline__ double2 cook(const Raw& v) const { return v; }
+    __device__ __forceinline__ double2 operator()(int vec, int pair) const { return raw(vec, pair); }
+};
+
+template <int MINB>
+__global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_cg1(const GArgs a) {
+    cg::grid_group grid = cg::this_grid();
+    State* st = a.st;
+    if (st->done) return;
+    double rho = st->rho, alpha = 0.0, beta = 0.0, rr_last = st->rr;
+    const double thr = a.ca->tol * st->bnorm;
+    const int maxit = a.ca->maxit;
+    BsrView A = a.A;
+    A.upper = a.su;
+    const int lane = threadIdx.x & 31;
+    const int w0 = blockIdx.x * WPB + (threadIdx.x >> 5), W = gridDim.x * WPB;
+    const int n = A.n, ngrp = (n + 4) / 5;
+    double* x = a.ca->d;
+    double* Rb[2] = {a.r, a.z};
+    double* Sb[2] = {a.t, a.w};
+    double* Qb[2] = {a.q, a.p1};
+    double* P = a.p0;
+    int k = 0, status = DDA_ERR_NO_CONVERGENCE, iters = 0, checks = 0;
+    {   // pass 0: s_0 = Ks r_0, mu_0 = r_0 . s_0
+        const XPlainW xf{a.r};
+        double mu = 0.0;
+        for_rows_c<SPMV_OFFDIAG, 5>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+            if (ok) {
+                const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
+                const double2 rv = xf(i, ccol_of(lane));
+                const double2 sv = make_double2(y0 + rv.x, y1 + rv.y);
+                *reinterpret_cast<double2*>(Sb[0] + o) = sv;
+                mu += rv.x * sv.x + rv.y * sv.y;
+            }
+        });
+        double v[1] = {mu}, tot[1];
+        grid_allsum<1>(a, grid, 4, v, tot);
+        if (!(tot[0] > 0.0) || !isfinite(tot[0])) status = DDA_ERR_BREAKDOWN;
+        alpha = rho / tot[0];
+    }
+    while (status != DDA_ERR_BREAKDOWN) {
+        const int cur = k & 1, nxt = cur ^ 1;
+        const bool first = k == 0;
+        const XCg1 xf{Rb[cur], Sb[cur], Qb[nxt], alpha, beta, first};
+        const double* rk_ = Rb[cur];
+        const double* sk_ = Sb[cur];
+        const double* qp_ = Qb[nxt];
+        double* qk_ = Qb[cur];
+        double* r1_ = Rb[nxt];
+        double* s1_ = Sb[nxt];
+        double rz = 0.0, mu = 0.0, lb = 0.0;
+        for_rows_c<SPMV_OFFDIAG, 5>(A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+            if (ok) {
+                const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
+                const double2 rk = ld_cg2(rk_ + o), sk = ld_cg2(sk_ + o);
+                double2 qk = sk, pk = rk;
+                if (!first) {
+                    const double2 qp = ld_cg2(qp_ + o), pp = ld_cg2(P + o);
+                    qk = make_double2(fma(beta, qp.x, sk.x), fma(beta, qp.y, sk.y));
+                    pk = make_double2(fma(beta, pp.x, rk.x), fma(beta, pp.y, rk.y));
+                }
+                const double2 r1 = make_double2(fma(-alpha, qk.x, rk.x), fma(-alpha, qk.y, rk.y));
+                const double2 s1 = make_double2(y0 + r1.x, y1 + r1.y);
+                const double2 xo = ld_cg2(x + o);
+                *reinterpret_cast<double2*>(x + o) = make_double2(xo.x + alpha * pk.x, xo.y + alpha * pk.y);
+                *reinterpret_cast<double2*>(P + o) = pk;
+                *reinterpret_cast<double2*>(qk_ + o) = qk;
+                *reinterpret_cast<double2*>(r1_ + o) = r1;
+                *reinterpret_cast<double2*>(s1_ + o) = s1;
+                const double rr2 = r1.x * r1.x + r1.y * r1.y;
+                rz += rr2;
+                mu += r1.x * s1.x + r1.y * s1.y;
+                lb += __ldg(a.bj_w + i) * rr2;
+            }
+        });
+        double bv[3] = {rz, mu, lb}, btot[3];
+        grid_allsum<3>(a, grid, cur ? 4 : 1, bv, btot);
+        const double rho1 = btot[0];
+        iters = k + 1;
+        if (rho1 == 0.0) { status = DDA_OK; rr_last = 0.0; k = k + 1; break; }
+        if (isfinite(rho1) && !(0.999 * btot[2] > thr * thr)) {
+            double rl = 0.0;   // phase C: the exact test |L r~| <= tol ||F|| (reading Z1)
+            for (int grp = w0; grp < ngrp; grp += W) {
+                const Row5 R = row5(grp, lane, n);
+                const double rv = R.valid ? ld_cg(r1_ + R.idx) : 0.0;
+                const DinvRow Lrow = tri_row(a.lfac, R);
+                const double o0 = dinv_row_apply(Lrow, rv, R);
+                const double o = R.valid ? o0 : 0.0;
+                rl += o * o;
+            }
+            double cv[1] = {rl}, ctot[1];
+            grid_allsum<1>(a, grid, 0, cv, ctot);
+            checks += 1;
+            rr_last = ctot[0];
+            if (sqrt(ctot[0]) <= thr) { status = DDA_OK; k = k + 1; break; }
+        }
+        k = k + 1;
+        if (!(rho1 > 0.0) || !isfinite(rho1)) { status = DDA_ERR_BREAKDOWN; break; }
+        const double b1 = rho1 / rho;
+        const double den = btot[1] - b1 * rho1 / alpha;
+        if (!(den > 0.0) || !isfinite(den)) { status = DDA_ERR_BREAKDOWN; break; }   // p.Ks p <= 0
+        beta = b1;
+        alpha = rho1 / den;
+        rho = rho1;
+        if (k >= maxit) { status = DDA_ERR_NO_CONVERGENCE; break; }
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        st->k = k;
+        st->iters = iters;
+        st->status = status;
+        st->done = 1;
+        st->alpha = alpha;
+        st->beta = beta;
+        st->rho = rho;
+        st->rr = rr_last;
+        st->pend = 0;   // x already holds x_{k}
+        st->checks = checks;
+    }
+}
+
 __global__ void __launch_bounds__(DDA_THREADS, 3) k_sp_ssor(const GArgs a) {
     cg::grid_group grid = cg::this_grid();
     State* st = a.st;
@@ -1173,6 +1319,8 @@ int g_scaled_loop = -1;
 unsigned long long* g_trace = nullptr;   // k_sp_loop timeline (internal hook dda__set_loop_trace)
 int g_trace_iters = 0;
 
+constexpr int kCg1Rows = 60000;   // k_sp_cg1 below this many block rows (see pcg_graph_solve)
+
 // Per-handle cached graph engine
 struct PcgGraph {
     int pc = -1;
@@ -1227,7 +1375,14 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     }
     // scaled SSOR-AI exists as a persistent kernel only (k_sp_ssor)
     bool persist = scaled && (g_scaled_loop == 1 || pc == DDA_PC_SSOR_AI);
+    // scaled BJ engine: the single-reduction loop (one grid barrier per iteration, one more gathered
+    // vector per block) below kCg1Rows block rows, where the iteration is barrier-latency bound; the
+    // two-phase k_sp_loop above, where the gathers' L2 traffic decides (measured
+    // crossover).  DDA_SCALED_CG1 = 0 / 1 forces either (tests, A/B).
+    const int cg1_env = env_int("DDA_SCALED_CG1", -1);
+    const bool cg1 = scaled && pc == DDA_PC_BJ && (cg1_env >= 0 ? cg1_env != 0 : K->n < kCg1Rows);
     const void* persist_kernel = pc == DDA_PC_SSOR_AI ? reinterpret_cast<const void*>(k_sp_ssor)
+                                                      : cg1 ? reinterpret_cast<const void*>(k_sp_cg1<3>)
                                                       : reinterpret_cast<const void*>(k_sp_loop<3>);
     if (persist) {
         // The persistent kernels need every CTA co-resident (cooperative launch).  If not even one CTA
@@ -1243,7 +1398,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
             persist = false;
         }
     }
-    const int key = scaled ? (persist ? 200 : 100) + (int)pc : (int)pc;
+    const int key = (scaled ? (persist ? 200 : 100) + (int)pc : (int)pc) + (cg1 ? 1000 : 0);
     PcgGraph*& G = reinterpret_cast<PcgGraph*&>(K->graph_engine);
     if (G && G->pc != key) {
         pcg_graph_free(G);
@@ -1272,7 +1427,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
             if (cap > 0 && g_persist > cap) g_persist = cap;
             if (g_persist > Gmax) Gmax = g_persist;
         }
-        const size_t bytes = (7 * N + 4 * (size_t)Gmax) * sizeof(double) + sizeof(CallArgs) + sizeof(State) + 64;
+        const size_t bytes = (7 * N + 8 * (size_t)Gmax) * sizeof(double) + sizeof(CallArgs) + sizeof(State) + 64;
         // may reallocate the workspace (and drop any engine holding the old pointers): do it first
         dda_status_t s = ensure_workspace(K, bytes, st);
         if (s != DDA_OK) return s;
@@ -1289,7 +1444,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         a.w = ws + 6 * N;
         a.part = ws + 7 * N;
         a.Gmax = Gmax;
-        char* tail = reinterpret_cast<char*>(a.part + 4 * (size_t)Gmax);
+        char* tail = reinterpret_cast<char*>(a.part + 8 * (size_t)Gmax);
         a.ca = reinterpret_cast<CallArgs*>(tail);
         a.st = reinterpret_cast<State*>(tail + ((sizeof(CallArgs) + 15) / 16) * 16);
         a.pc = (int)pc;

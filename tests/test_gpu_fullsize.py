@@ -157,7 +157,11 @@ def test_ssor_ai_100k_z17(dda, precond100k):
     _z17(dda, O, P, d.cpu().numpy(), it, "ssor_ai")
 
 
-def test_bj_100k_z17(dda, precond100k):
+@pytest.mark.parametrize("cg1", ["0", "1"], ids=["2phase", "cg1"])
+def test_bj_100k_z17(dda, precond100k, cg1, monkeypatch):
+    """Scaled BJ at configs[2]'s size over its whole solve (Z17), with the two-phase k_sp_loop (the
+    default there) and with the single-reduction k_sp_cg1 forced."""
+    monkeypatch.setenv("DDA_SCALED_CG1", cg1)
     P, O = precond100k
     K = dda.build_from_problem(P)
     d, it, rr, st = K.pcg_solve(torch.from_numpy(P.F).cuda(), tol=1e-10, precond="bj")

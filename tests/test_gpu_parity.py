@@ -255,15 +255,18 @@ def _set_engine(dda, engine, loop=-1):
     g(loop)
 
 
-@pytest.fixture(params=["auto", "graph", "persistent", "scaled", "scaled_graph"])
-def engine(request, dda):
+@pytest.fixture(params=["auto", "graph", "persistent", "scaled", "scaled_2phase", "scaled_cg1", "scaled_graph"])
+def engine(request, dda, monkeypatch):
     """PCG engine: the CUDA-graph while loop, the persistent cooperative kernel, or the
     block-scaled matrix S K S^T (block-Jacobi only; other preconditioners fall back to
-    the graph loop) run by one persistent cooperative kernel ('scaled') or by the
+    the graph loop) run by one persistent cooperative kernel ('scaled': the two-phase k_sp_loop
+    or the single-reduction k_sp_cg1 by size; '_2phase' / '_cg1' force one) or by the
     CUDA-graph while loop ('scaled_graph') — internal hooks; 'auto' picks by size and
     preconditioner."""
+    if request.param in ("scaled_2phase", "scaled_cg1"):
+        monkeypatch.setenv("DDA_SCALED_CG1", "1" if request.param == "scaled_cg1" else "0")
     _set_engine(dda, *{"auto": (-1, -1), "graph": (0, -1), "persistent": (1, -1), "scaled": (2, 1),
-                       "scaled_graph": (2, 0)}[request.param])
+                       "scaled_2phase": (2, 1), "scaled_cg1": (2, 1), "scaled_graph": (2, 0)}[request.param])
     yield request.param
     _set_engine(dda, -1, -1)
 
@@ -360,8 +363,10 @@ def test_scaled_engine_stopping_test(dda, loop):
     assert np.linalg.norm(d2.cpu().numpy() - d0.cpu().numpy()) <= 1e-8 * np.linalg.norm(d0.cpu().numpy())
 
 
+@pytest.mark.parametrize("cg1", ["0", "1"], ids=["2phase", "cg1"])
 @pytest.mark.parametrize("eng", [(-1, -1), (2, 1), (2, 0)], ids=["auto", "scaled", "scaled_graph"])
-def test_pcg_deterministic(dda, eng):
+def test_pcg_deterministic(dda, eng, cg1, monkeypatch):
+    monkeypatch.setenv("DDA_SCALED_CG1", cg1)
     P, O = case("paper")
     K = dda.build_from_problem(P)
     F = torch.from_numpy(P.F).cuda()
@@ -391,6 +396,25 @@ def test_scaled_loops_agree(dda):
     (dp, itp, rrp, stp, cp), (dg, itg, rrg, stg, cg) = out[1], out[0]
     assert stp == stg == dda.OK and abs(itp - itg) <= 1 and rrp <= 1e-10 and rrg <= 1e-10
     assert np.linalg.norm(dp - dg) <= 1e-9 * np.linalg.norm(dg)
+
+
+@pytest.mark.parametrize("name", ["paper", "ragged_1k"])
+def test_single_reduction_loop_matches_two_phase(dda, name, monkeypatch):
+    """k_sp_cg1 (Chronopoulos-Gear: s = Ks r carried, one grid barrier per iteration) runs the same
+    Krylov iterates as k_sp_loop in exact arithmetic: same stopping iteration (+-1), solutions
+    within the PCG tolerance, and each matches the oracle at the matched iteration (reading Z17)."""
+    P, O = case(name)
+    out = {}
+    try:
+        _set_engine(dda, 2, 1)
+        for v in ("0", "1"):
+            monkeypatch.setenv("DDA_SCALED_CG1", v)
+            out[v] = _pcg_parity(dda, P, O, "bj")
+    finally:
+        _set_engine(dda, -1, -1)
+    (d0, it0), (d1, it1) = out["0"], out["1"]
+    assert abs(it0 - it1) <= 1, (it0, it1)
+    assert np.linalg.norm(d1 - d0) <= 1e-9 * np.linalg.norm(d0)
 
 
 def test_solve_host_e2e(dda):
