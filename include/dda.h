@@ -194,6 +194,37 @@ dda_status_t dda_solve_host(int32_t n_blocks, const double *kdiag, int64_t n_spr
                             dda_precond_t pc, double omega, int32_t *iters, double *rel_res, void *stream);
 
 /*
+ * Streamed end-to-end entry: nsys independent host systems solved in order (a
+ * time-stepping driver's loop 1 of PAPER.md Fig. 1, one system per step) with
+ * the host->device copy of system k+1 and the device->host copy of system k's d
+ * overlapping the assembly and solve of system k (a second, copy stream; two
+ * device input slots sized for the largest system).  Per system the work is
+ * exactly dda_solve_host's.  Host buffers should be pinned (pageable buffers
+ * work but their copies do not overlap) and must not change until the call
+ * returns.  Fields marked out are written per system; the call returns DDA_OK
+ * unless an argument or CUDA error stops the batch (then the systems before the
+ * failing one are complete and its status field holds the error).  d0 may be
+ * NULL.  Synchronising.
+ */
+typedef struct {
+    int32_t n_blocks;
+    int64_t n_springs;
+    const double *kdiag;          /* [n_blocks][36] */
+    const int32_t *bi, *bj;       /* [n_springs] */
+    const double *pen;            /* [n_springs] */
+    const double *e, *g;          /* [n_springs][6] */
+    const double *F;              /* [6 n_blocks] */
+    const double *d0;             /* [6 n_blocks] or NULL */
+    double *d;                    /* out: [6 n_blocks] */
+    int32_t iters;                /* out */
+    double rel_res;               /* out: TRUE relative residual */
+    dda_status_t status;          /* out: as dda_pcg_solve */
+} dda_host_system;
+
+dda_status_t dda_solve_host_batch(int32_t nsys, dda_host_system *sys, double tol, int32_t maxit, dda_precond_t pc,
+                                  double omega, void *stream);
+
+/*
  * (e) — Multi-GPU block-row partitioned PCG (beyond the paper: multi-GPU is its
  * future work).  A partition is an ordinary dda_matrix_t built on the
  * partition's LOCAL numbering: own rows 0..n_own-1 (a contiguous range of

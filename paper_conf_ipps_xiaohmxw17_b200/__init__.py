@@ -33,7 +33,7 @@ ABI_SYMBOLS = ("dda_build_matrix", "dda_update_values", "dda_matrix_info", "dda_
                "dda_dist_info", "dda_classify_contacts", "dda_contacts_classes",
                "dda_contact_init", "dda_contact_loads", "dda_contact_check", "dda_open_close",
                "dda_build_matrix_reordered", "dda_hsbcsr_build", "dda_hsbcsr_spmv", "dda_hsbcsr_export",
-               "dda_hsbcsr_free", "dda_contact_transfer")
+               "dda_hsbcsr_free", "dda_contact_transfer", "dda_solve_host_batch")
 
 _lib = None
 
@@ -86,6 +86,8 @@ def lib() -> C.CDLL:
         L.dda_solve_host.argtypes = [I32, P, I64, P, P, P, P, P, P, P, P, D, I32, st, D,
                                      C.POINTER(I32), C.POINTER(D), P]
         L.dda_solve_host.restype = st
+        L.dda_solve_host_batch.argtypes = [I32, C.POINTER(HostSystem), D, I32, st, D, P]
+        L.dda_solve_host_batch.restype = st
         L.dda_launch_count.argtypes = []
         L.dda_launch_count.restype = I64
         L.dda_matrix_free.argtypes = [P]
@@ -370,6 +372,45 @@ def problem_to_device(P, device="cuda") -> dict:
             "bj": torch.from_numpy(P.bj).to(device), "pen": torch.from_numpy(P.pen).to(device),
             "e": torch.from_numpy(P.e).to(device), "g": torch.from_numpy(P.g).to(device),
             "F": torch.from_numpy(P.F).to(device)}
+
+
+class HostSystem(C.Structure):
+    """dda_host_system (dda.h): one host system of dda_solve_host_batch."""
+    _fields_ = [("n_blocks", C.c_int32), ("n_springs", C.c_int64), ("kdiag", C.c_void_p), ("bi", C.c_void_p),
+                ("bj", C.c_void_p), ("pen", C.c_void_p), ("e", C.c_void_p), ("g", C.c_void_p), ("F", C.c_void_p),
+                ("d0", C.c_void_p), ("d", C.c_void_p), ("iters", C.c_int32), ("rel_res", C.c_double),
+                ("status", C.c_int)]
+
+
+def _host_ptr(a, dtype):
+    if a is None:
+        return None
+    if hasattr(a, "data_ptr"):
+        import torch
+        assert not a.is_cuda and a.is_contiguous() and a.dtype == {np.float64: torch.float64, np.int32: torch.int32}[dtype]
+        return a.data_ptr()
+    assert a.dtype == dtype and a.flags["C_CONTIGUOUS"]
+    return a.ctypes.data
+
+
+def solve_host_batch(systems, tol=1e-10, maxit=10000, precond="bj", omega=1.0, stream=None):
+    """Streamed end-to-end solves (dda_solve_host_batch): `systems` is a list of dicts with host arrays
+    kdiag, bi, bj, pen, e, g, F, optional d0, and the output d (numpy or pinned CPU tensors, pinned for
+    the copy overlap).  Returns [(iters, rel_res, status)] per system."""
+    arr = (HostSystem * len(systems))()
+    for k, S in enumerate(systems):
+        h = arr[k]
+        h.n_blocks = int(S["kdiag"].shape[0])
+        h.n_springs = int(S["bi"].shape[0])
+        for f, dt in (("kdiag", np.float64), ("bi", np.int32), ("bj", np.int32), ("pen", np.float64),
+                      ("e", np.float64), ("g", np.float64), ("F", np.float64), ("d", np.float64)):
+            setattr(h, f, _host_ptr(S[f], dt))
+        h.d0 = _host_ptr(S.get("d0"), np.float64)
+    st = lib().dda_solve_host_batch(len(systems), arr, float(tol), int(maxit), PRECOND[precond], float(omega),
+                                    C.c_void_p(_stream(stream)))
+    if st != OK:
+        raise DDAError(st, "dda_solve_host_batch")
+    return [(int(h.iters), float(h.rel_res), int(h.status)) for h in arr]
 
 
 def solve_host(kdiag, bi, bj, pen, e, g, F, d0=None, tol=1e-10, maxit=10000, precond="bj", omega=1.0,

@@ -268,13 +268,19 @@ dda_status_t cuda_fail(cudaError_t e);
 
 using namespace dda;
 
-extern "C" void dda_matrix_free(dda_matrix_t K) {
+extern "C" void dda_matrix_free(dda_matrix_t K) { dda::matrix_free_impl(K, nullptr); }
+
+// sync == nullptr: device-wide synchronisation first (the ABI's rule: no stream may still use the
+// arrays); else only that stream, the one every use of K was ordered on (dda_solve_host_batch, whose
+// copy stream keeps running)
+void dda::matrix_free_impl(dda_matrix_t K, cudaStream_t* sync) {
     if (!K) return;
     int prev = 0;
     cudaGetDevice(&prev);
     cudaSetDevice(K->device);
     trace("free: enter");
-    cudaDeviceSynchronize();   // no stream may still use the arrays
+    if (sync) cudaStreamSynchronize(*sync);
+    else cudaDeviceSynchronize();
     trace("free: synchronized");
     if (K->graph_engine) pcg_graph_free(K->graph_engine);
     trace("free: engine freed");

@@ -181,6 +181,7 @@ dda_status_t bj_setup(dda_matrix* K, cudaStream_t s, int32_t* bad_block);
 dda_status_t spmv(dda_matrix* K, const double* x, double* y, cudaStream_t s);
 void pcg_graph_free(void* g);
 dda_status_t scaled_setup(dda_matrix* K, cudaStream_t st);
+void matrix_free_impl(dda_matrix_t K, cudaStream_t* sync);
 dda_status_t build_matrix_impl(int32_t n, const double* kdiag, int64_t m, const int32_t* bi, const int32_t* bj,
                                const double* pen, const double* e, const double* g, cudaStream_t stream,
                                cudaEvent_t values_ready, dda_matrix_t* out);   // S_i V_ij S_j^T (needs lfac / sfac of every row)

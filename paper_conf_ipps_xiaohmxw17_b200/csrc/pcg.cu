@@ -619,3 +619,104 @@ extern "C" dda_status_t dda_solve_host(int32_t n, const double* kdiag, int64_t m
     dda_matrix_free(K);
     return s;
 }
+
+// Streamed end-to-end batch (dda.h): system k+1's inputs go host->device on a copy stream into the
+// free one of two input slots while system k is assembled and solved on the caller's stream; system
+// k's d goes device->host on the copy stream behind its solve.  Events order the reuse: a slot is
+// refilled only after the solve that read it (in_free), a result buffer is rewritten only after
+// its device->host copy (out_free).
+extern "C" dda_status_t dda_solve_host_batch(int32_t nsys, dda_host_system* sys, double tol, int32_t maxit,
+                                             dda_precond_t pc, double omega, void* stream) {
+    if (nsys < 0 || (nsys > 0 && !sys)) return DDA_ERR_ARG;
+    int32_t nmax = 0;
+    int64_t mmax = 0;
+    for (int k = 0; k < nsys; ++k) {
+        dda_host_system& S = sys[k];
+        S.iters = 0;
+        S.rel_res = 0.0;
+        S.status = DDA_ERR_ARG;
+        if (S.n_blocks <= 0 || S.n_springs < 0 || !S.kdiag || !S.F || !S.d) return DDA_ERR_ARG;
+        if (S.n_springs > 0 && (!S.bi || !S.bj || !S.pen || !S.e || !S.g)) return DDA_ERR_ARG;
+        nmax = S.n_blocks > nmax ? S.n_blocks : nmax;
+        mmax = S.n_springs > mmax ? S.n_springs : mmax;
+    }
+    if (nsys == 0) return DDA_OK;
+    cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+    const size_t Nmax = 6 * (size_t)nmax;
+    auto up = [](size_t b) { return (b + 255) & ~(size_t)255; };
+    // slot layout: kdiag, F, d0, pen, e, g, bi, bj (every sub-buffer 256-byte aligned)
+    const size_t sz[8] = {sizeof(double) * 36 * (size_t)nmax, sizeof(double) * Nmax, sizeof(double) * Nmax,
+                          sizeof(double) * (size_t)mmax, sizeof(double) * 6 * (size_t)mmax,
+                          sizeof(double) * 6 * (size_t)mmax, sizeof(int32_t) * (size_t)mmax,
+                          sizeof(int32_t) * (size_t)mmax};
+    size_t off[9] = {0};
+    for (int q = 0; q < 8; ++q) off[q + 1] = off[q] + up(sz[q] ? sz[q] : 1);
+    const size_t slot_bytes = off[8], res_bytes = up(sizeof(double) * Nmax);
+    char* buf = nullptr;
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&buf), 2 * slot_bytes + 2 * res_bytes, st));
+    struct Res {
+        char* b; cudaStream_t s; cudaStream_t cs = nullptr;
+        cudaEvent_t ev[7] = {};
+        ~Res() {
+            if (cs) { cudaStreamSynchronize(cs); cudaStreamDestroy(cs); }
+            cudaStreamSynchronize(s);
+            for (cudaEvent_t e : ev) if (e) cudaEventDestroy(e);
+            dev_free_on(b, s);
+        }
+    } res{buf, st};
+    DDA_CK(cudaStreamCreateWithFlags(&res.cs, cudaStreamNonBlocking));
+    for (cudaEvent_t& e : res.ev) DDA_CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    cudaEvent_t start = res.ev[0], *in_ready = res.ev + 1, *in_free = res.ev + 3, *out_free = res.ev + 5;
+    cudaStream_t cs = res.cs;
+    DDA_CK(cudaEventRecord(start, st));                     // the buffer is allocated stream-ordered on st
+    DDA_CK(cudaStreamWaitEvent(cs, start, 0));
+    auto slot = [&](int k, int q) { return buf + (size_t)(k & 1) * slot_bytes + off[q]; };
+    auto result = [&](int k) { return reinterpret_cast<double*>(buf + 2 * slot_bytes + (size_t)(k & 1) * res_bytes); };
+    auto copy_in = [&](int k) -> cudaError_t {
+        const dda_host_system& S = sys[k];
+        const size_t N = 6 * (size_t)S.n_blocks, m = (size_t)S.n_springs;
+        cudaError_t e = k >= 2 ? cudaStreamWaitEvent(cs, in_free[k & 1], 0) : cudaSuccess;
+        if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 0), S.kdiag, sizeof(double) * 6 * N, cudaMemcpyHostToDevice, cs);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 1), S.F, sizeof(double) * N, cudaMemcpyHostToDevice, cs);
+        if (e == cudaSuccess && S.d0) e = cudaMemcpyAsync(slot(k, 2), S.d0, sizeof(double) * N, cudaMemcpyHostToDevice, cs);
+        if (m > 0) {
+            if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 3), S.pen, sizeof(double) * m, cudaMemcpyHostToDevice, cs);
+            if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 4), S.e, sizeof(double) * 6 * m, cudaMemcpyHostToDevice, cs);
+            if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 5), S.g, sizeof(double) * 6 * m, cudaMemcpyHostToDevice, cs);
+            if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 6), S.bi, sizeof(int32_t) * m, cudaMemcpyHostToDevice, cs);
+            if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 7), S.bj, sizeof(int32_t) * m, cudaMemcpyHostToDevice, cs);
+        }
+        if (e == cudaSuccess) e = cudaEventRecord(in_ready[k & 1], cs);
+        return e;
+    };
+    DDA_CK(copy_in(0));
+    for (int k = 0; k < nsys; ++k) {
+        dda_host_system& S = sys[k];
+        if (k + 1 < nsys) DDA_CK(copy_in(k + 1));          // overlaps this system's assembly and solve
+        DDA_CK(cudaStreamWaitEvent(st, in_ready[k & 1], 0));
+        if (k >= 2) DDA_CK(cudaStreamWaitEvent(st, out_free[k & 1], 0));
+        const double* dk = reinterpret_cast<const double*>(slot(k, 0));
+        dda_matrix_t K = nullptr;
+        dda_status_t s = build_matrix_impl(S.n_blocks, dk, S.n_springs, reinterpret_cast<const int32_t*>(slot(k, 6)),
+                                           reinterpret_cast<const int32_t*>(slot(k, 7)),
+                                           reinterpret_cast<const double*>(slot(k, 3)),
+                                           reinterpret_cast<const double*>(slot(k, 4)),
+                                           reinterpret_cast<const double*>(slot(k, 5)), st, nullptr, &K);
+        if (s != DDA_OK) { S.status = s; return s; }
+        s = dda_pcg_solve(K, reinterpret_cast<const double*>(slot(k, 1)),
+                          S.d0 ? reinterpret_cast<const double*>(slot(k, 2)) : nullptr, result(k), tol, maxit, pc,
+                          omega, &S.iters, &S.rel_res, stream);
+        S.status = s;
+        const bool solved = s == DDA_OK || s == DDA_ERR_NO_CONVERGENCE || s == DDA_ERR_BREAKDOWN;
+        DDA_CK(cudaEventRecord(in_free[k & 1], st));        // the slot's inputs are no longer read
+        if (solved) {
+            DDA_CK(cudaStreamWaitEvent(cs, in_free[k & 1], 0));
+            DDA_CK(cudaMemcpyAsync(S.d, result(k), sizeof(double) * 6 * (size_t)S.n_blocks, cudaMemcpyDeviceToHost, cs));
+        }
+        DDA_CK(cudaEventRecord(out_free[k & 1], cs));
+        matrix_free_impl(K, &st);
+        if (!solved) return s;
+    }
+    DDA_CK(cudaStreamSynchronize(cs));
+    return DDA_OK;
+}

@@ -426,6 +426,30 @@ def test_solve_host_e2e(dda):
     assert np.array_equal(d, d2.cpu().numpy())
 
 
+def test_solve_host_batch(dda):
+    """Streamed batch (dda_solve_host_batch): systems of different sizes, one with a warm start and
+    one repeated (so both input slots are refilled), each bit-identical to dda_solve_host; pinned and
+    pageable host buffers."""
+    names = ["paper", "tiny", "paper", "ragged_1k", "tiny"]
+    systems, refs = [], []
+    for k, name in enumerate(names):
+        P, O = case(name)
+        pin = (lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()) if k % 2 == 0 else (lambda a: a)
+        S = {f: pin(getattr(P, f)) for f in ("kdiag", "bi", "bj", "pen", "e", "g", "F")}
+        d0 = warm_start(np.zeros(6 * P.n), 3) if k == 2 else None
+        if d0 is not None:
+            S["d0"] = pin(d0)
+        S["d"] = pin(np.full(6 * P.n, np.nan))
+        systems.append(S)
+        refs.append(dda.solve_host(P.kdiag, P.bi, P.bj, P.pen, P.e, P.g, P.F, d0=d0))
+    out = dda.solve_host_batch(systems)
+    for S, (dr, itr, rrr, str_), (it, rr, st) in zip(systems, refs, out):
+        d = S["d"].numpy() if hasattr(S["d"], "numpy") else S["d"]
+        assert st == str_ == dda.OK and it == itr and rr == rrr
+        assert np.array_equal(d, dr)
+    assert dda.solve_host_batch([]) == []
+
+
 @pytest.mark.parametrize("name", ["tiny", "paper"])
 def test_scaled_ssor_omega0_is_bj(dda, name):
     """SSOR-AI with omega = 0 is M^{-1} = D^{-1} (reading Z14): the scaled SSOR-AI kernel must take the

@@ -3,7 +3,7 @@
 Runs every kernel family of the hot path once on a small system, through the C ABI:
 assembly + value-only re-assembly, the symmetric SpMV (and full storage), the
 block-Jacobi setup, PCG with each engine — the scaled persistent kernel k_sp_loop
-(including its exact stopping test, phase C), the scaled graph loop, the unscaled
+(including its exact stopping test, phase C) and the single-reduction k_sp_cg1, the scaled graph loop, the unscaled
 graph loop, the scaled SSOR-AI persistent kernel k_sp_ssor, the ILU(0) sync-free
 sweeps — the partitioned solver over the loopback transport (P = 2), and contact
 detection.  Every result is checked against the oracle's iteration count so a
@@ -35,7 +35,7 @@ def engine(eng, loop):
     g(loop)
 
 
-CASES = ("build", "spmv", "bj_graph_phases", "bj_scaled_persistent", "bj_scaled_graph", "bj_graph", "bj_persistent", "ssor_ai",
+CASES = ("build", "spmv", "bj_graph_phases", "bj_scaled_persistent", "bj_scaled_2phase", "bj_scaled_cg1", "bj_scaled_graph", "bj_graph", "bj_persistent", "ssor_ai",
          "ilu0", "none", "dist", "contacts")
 
 
@@ -48,8 +48,9 @@ def main(name, cases):
     K = dda.build_matrix(t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
     out = {}
     _, ito, _, _ = O.pcg(P.F, tol=1e-10, precond="bj")
-    engines = {"bj_scaled_persistent": (2, 1), "bj_scaled_graph": (0 + 2, 0), "bj_graph": (0, -1),
-               "bj_persistent": (1, -1)}
+    engines = {"bj_scaled_persistent": (2, 1), "bj_scaled_2phase": (2, 1), "bj_scaled_cg1": (2, 1),
+               "bj_scaled_graph": (0 + 2, 0), "bj_graph": (0, -1), "bj_persistent": (1, -1)}
+    forced = {"bj_scaled_2phase": "0", "bj_scaled_cg1": "1"}   # k_sp_loop / k_sp_cg1 (DDA_SCALED_CG1)
     for c in cases:
         print(f"case {c} ...", flush=True)
         if c == "build":
@@ -74,7 +75,10 @@ def main(name, cases):
             out[c] = (ms[0], ms[1])
         elif c in engines:
             engine(*engines[c])
+            if c in forced:
+                os.environ["DDA_SCALED_CG1"] = forced[c]
             d, it, rr, st = K.pcg_solve(F, tol=1e-10, precond="bj")
+            os.environ.pop("DDA_SCALED_CG1", None)
             engine(-1, -1)
             out[c] = (it, st, K.last_checks())
             assert st == dda.OK and abs(it - ito) <= max(2, ito // 100), (c, it, ito)
