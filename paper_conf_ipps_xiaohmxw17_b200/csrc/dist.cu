@@ -21,6 +21,7 @@
 // solve has finished.  The host issues iterations in chunks and reads the
 // state once per chunk (DDA_DIST_CHUNK, default 8) instead of twice per
 // iteration.  The SpMV is the column-pair map (spmv_col.cuh, v5) over own rows.
+#include <cooperative_groups.h>
 #include <nccl.h>
 
 #include <cmath>
@@ -29,6 +30,8 @@
 
 #include "precond_dev.cuh"
 #include "spmv_col.cuh"
+
+namespace cg = cooperative_groups;
 
 namespace dda {
 namespace {
@@ -749,6 +752,223 @@ __global__ void __launch_bounds__(DDA_THREADS) k_v4_final(int n, double* d, cons
     for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
         const Row5 R = row5(grp, lane, n);
         const double xv = R.valid ? d[R.idx] : 0.0;
+        const double dv = tri_apply(sfac, R, xv, true);
+        if (R.valid) d[R.idx] = dv;
+    }
+}
+
+// ---- v6 (loopback): every partition in ONE persistent cooperative kernel.
+//
+// The single-GPU scaled engine (k_sp_loop, pcg_graph.cu) run over partitions: CTA range [c0, c1) of the
+// grid serves partition p's own rows; a halo row of p is read straight from its owner's r~ and p_old
+// (pointer tables: owner partition, owner's local row), so p_k = r~_k + beta p_{k-1} is formed on the
+// fly for halo rows exactly as for own rows and no halo is ever copied; every grid-wide sum is a
+// fixed-order read of all partitions' CTA partials (the allreduce).  Per iteration:
+//   A  p_k (own, written to the ping-pong buffer), q = Ks p_k over own rows, x += alpha_{k-1} p_{k-1}
+//      | grid barrier, sigma
+//   B  r~ -= alpha q; |r~|^2 and the w-bound                     | grid barrier
+//   C  (rare) the exact test |L r~| (reading Z1)                 | grid barrier
+// Two barriers per iteration, as on one GPU.  On separate GPUs the same kernel needs the peer
+// pointers mapped over NVLink and the grid barrier extended by a flag exchange between ranks.
+struct DPart {
+    BsrView A;            // Ks over own rows (local columns: own, then halo)
+    double *rt, *p0, *p1, *q, *x;
+    const double* w;      // the w-bound weights (bj_setup)
+    const double* lfac;
+    const int2* hmap;     // [n_halo]: (owner partition, owner's local row)
+    int n_own, c0, c1;
+};
+struct DPState {
+    double alpha, beta, rho, rr;
+    int k, iters, status, pend, checks;
+};
+constexpr int kDPMax = 8;   // partitions held in the kernel's parameter block (more: v5)
+struct DPArgs {
+    DPart parts[kDPMax];
+    const DPart* gparts;  // the same table in global memory (halo owners' arrays)
+    int P;
+    double* part;         // [4][gridDim] CTA partials
+    DPState* st;
+    double rho0, thr;
+    int maxit;
+};
+
+// p = r~ + beta p_old for own and halo rows (sel: 0 -> p_old = r~ (k = 0), 1 -> p0, 2 -> p1)
+struct XFusedPeer {
+    const DPart* parts;
+    const double* rt;
+    const double* pold;
+    const int2* hmap;
+    int n_own, sel;
+    double beta;
+    using Raw = double2;
+    __device__ __forceinline__ Raw raw(int vec, int pair) const {
+        const double* z;
+        const double* p;
+        size_t o;
+        if (vec < n_own) {
+            z = rt;
+            p = pold;
+            o = 6 * (size_t)vec + 2 * pair;
+        } else {
+            const int2 h = __ldg(hmap + (vec - n_own));
+            const DPart& Q = parts[h.x];
+            z = Q.rt;
+            p = sel == 0 ? Q.rt : (sel == 1 ? Q.p0 : Q.p1);
+            o = 6 * (size_t)h.y + 2 * pair;
+        }
+        const double2 zz = *reinterpret_cast<const double2*>(z + o), pp = *reinterpret_cast<const double2*>(p + o);
+        return make_double2(fma(beta, pp.x, zz.x), fma(beta, pp.y, zz.y));
+    }
+    __device__ __forceinline__ double2 cook(const Raw& r) const { return r; }
+    __device__ __forceinline__ double2 operator()(int vec, int pair) const { return raw(vec, pair); }
+};
+
+// fixed-order grid sum of NV values (every CTA gets the same totals): partials -> part[(slot+k)*G + cta]
+template <int NV>
+__device__ __forceinline__ void dp_allsum(const DPArgs& a, cg::grid_group& grid, int slot, double (&v)[NV],
+                                          double (&tot)[NV]) {
+    __shared__ double red[NV][DDA_THREADS];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5, G = gridDim.x;
+#pragma unroll
+    for (int k = 0; k < NV; ++k) v[k] = warp_sum(v[k]);
+    if (lane == 0) {
+#pragma unroll
+        for (int k = 0; k < NV; ++k) red[k][wib] = v[k];
+    }
+    cta_barrier();
+    if (threadIdx.x == 0) {
+#pragma unroll
+        for (int k = 0; k < NV; ++k) {
+            double s = 0.0;
+            for (int w = 0; w < WPB; ++w) s += red[k][w];
+            a.part[(size_t)(slot + k) * G + blockIdx.x] = s;
+        }
+    }
+    grid.sync();
+#pragma unroll
+    for (int k = 0; k < NV; ++k) {
+        const double* part = a.part + (size_t)(slot + k) * G;
+        double s = 0.0;
+        for (int j = threadIdx.x; j < G; j += DDA_THREADS) s += *(volatile const double*)(part + j);
+        red[k][threadIdx.x] = s;
+    }
+    cta_barrier();
+    for (int h = DDA_THREADS / 2; h > 0; h >>= 1) {
+        if (threadIdx.x < h) {
+#pragma unroll
+            for (int k = 0; k < NV; ++k) red[k][threadIdx.x] += red[k][threadIdx.x + h];
+        }
+        cta_barrier();
+    }
+#pragma unroll
+    for (int k = 0; k < NV; ++k) tot[k] = red[k][0];
+    cta_barrier();
+}
+
+__global__ void __launch_bounds__(DDA_THREADS, 3) k_dist_loop(const DPArgs a) {
+    cg::grid_group grid = cg::this_grid();
+    int pi = 0;
+#pragma unroll
+    for (int q = 0; q + 1 < kDPMax; ++q)
+        if (q + 1 < a.P && (int)blockIdx.x >= a.parts[q].c1) pi = q + 1;
+    const DPart& D = a.parts[pi];
+    const int lane = threadIdx.x & 31;
+    const int w0 = ((int)blockIdx.x - D.c0) * WPB + (threadIdx.x >> 5), W = (D.c1 - D.c0) * WPB;
+    const int n = D.n_own, ngrp = (n + 4) / 5;
+    const double thr = a.thr;
+    double rho = a.rho0, alpha = 0.0, beta = 0.0, rr_last = 0.0;
+    int k = 0, status = DDA_ERR_NO_CONVERGENCE, iters = 0, checks = 0, pend = 0;
+    for (;;) {
+        double* pnew = (k & 1) ? D.p1 : D.p0;
+        const double* pold = k == 0 ? D.rt : ((k & 1) ? D.p0 : D.p1);
+        const XFusedPeer xf{a.gparts, D.rt, pold, D.hmap, n, k == 0 ? 0 : ((k & 1) ? 1 : 2), beta};
+        const double ap = alpha;
+        double acc = 0.0;
+        for_rows_c<SPMV_OFFDIAG, 5>(D.A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+            if (ok) {
+                const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
+                const double2 pv = xf(i, ccol_of(lane));
+                y0 += pv.x;
+                y1 += pv.y;
+                const double2 po = *reinterpret_cast<const double2*>(pold + o);
+                const double2 xo = *reinterpret_cast<const double2*>(D.x + o);
+                *reinterpret_cast<double2*>(D.x + o) = make_double2(xo.x + ap * po.x, xo.y + ap * po.y);
+                *reinterpret_cast<double2*>(D.q + o) = make_double2(y0, y1);
+                *reinterpret_cast<double2*>(pnew + o) = pv;
+                acc += pv.x * y0 + pv.y * y1;
+            }
+        });
+        double sv[1] = {acc}, stot[1];
+        dp_allsum<1>(a, grid, 0, sv, stot);
+        const double sigma = stot[0];
+        pend = 0;
+        if (!(sigma > 0.0) || !isfinite(sigma)) { status = DDA_ERR_BREAKDOWN; break; }
+        alpha = rho / sigma;
+        double rz = 0.0, lb = 0.0;
+        for (int grp = w0; grp < ngrp; grp += 2 * W) {     // two row groups in flight per warp
+            const Row5 RA = row5(grp, lane, n);
+            const Row5 RB = row5(grp + W, lane, n);
+            double ra = 0, qa = 0, rb = 0, qb = 0, wa = 0, wb = 0;
+            if (RA.valid) { ra = D.rt[RA.idx]; qa = D.q[RA.idx]; wa = __ldg(D.w + RA.i); }
+            if (RB.valid) { rb = D.rt[RB.idx]; qb = D.q[RB.idx]; wb = __ldg(D.w + RB.i); }
+            const double rva = RA.valid ? ra - alpha * qa : 0.0;
+            const double rvb = RB.valid ? rb - alpha * qb : 0.0;
+            if (RA.valid) D.rt[RA.idx] = rva;
+            if (RB.valid) D.rt[RB.idx] = rvb;
+            rz += rva * rva + rvb * rvb;
+            lb += wa * (rva * rva) + wb * (rvb * rvb);
+        }
+        double bv[2] = {rz, lb}, btot[2];
+        dp_allsum<2>(a, grid, 1, bv, btot);
+        const double rho1 = btot[0];
+        pend = 1;
+        iters = k + 1;
+        if (rho1 == 0.0) { status = DDA_OK; rr_last = 0.0; k = k + 1; break; }
+        if (isfinite(rho1) && !(0.999 * btot[1] > thr * thr)) {   // the exact test (reading Z1)
+            double rl = 0.0;
+            for (int grp = w0; grp < ngrp; grp += W) {
+                const Row5 R = row5(grp, lane, n);
+                const double rv = R.valid ? D.rt[R.idx] : 0.0;
+                const double o0 = tri_apply(D.lfac, R, rv, false);
+                const double o = R.valid ? o0 : 0.0;
+                rl += o * o;
+            }
+            double cv[1] = {rl}, ctot[1];
+            dp_allsum<1>(a, grid, 3, cv, ctot);
+            checks += 1;
+            rr_last = ctot[0];
+            if (sqrt(ctot[0]) <= thr) { status = DDA_OK; k = k + 1; break; }
+        }
+        k = k + 1;
+        if (!(rho1 > 0.0) || !isfinite(rho1)) { status = DDA_ERR_BREAKDOWN; break; }
+        beta = rho1 / rho;
+        rho = rho1;
+        if (k >= a.maxit) { status = DDA_ERR_NO_CONVERGENCE; break; }
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        DPState* st = a.st;
+        st->k = k;
+        st->iters = iters;
+        st->status = status;
+        st->alpha = alpha;
+        st->beta = beta;
+        st->rho = rho;
+        st->rr = rr_last;
+        st->pend = pend;
+        st->checks = checks;
+    }
+}
+
+// the pending x += alpha p_{k-1} of the last iteration, then d = S^T x (own rows)
+__global__ void __launch_bounds__(DDA_THREADS) k_dp_final(int n, double* d, const double* __restrict__ pk,
+                                                          const DPState* st, const double* __restrict__ sfac) {
+    const bool pend = st->pend;
+    const double alpha = st->alpha;
+    const int lane = threadIdx.x & 31, ngrp = (n + 4) / 5, W = gridDim.x * WPB;
+    for (int grp = blockIdx.x * WPB + (threadIdx.x >> 5); grp < ngrp; grp += W) {
+        const Row5 R = row5(grp, lane, n);
+        const double xv = R.valid ? (pend ? d[R.idx] + alpha * pk[R.idx] : d[R.idx]) : 0.0;
         const double dv = tri_apply(sfac, R, xv, true);
         if (R.valid) d[R.idx] = dv;
     }
@@ -1485,6 +1705,138 @@ dda_status_t dist_v4_solve(dda_comm* c, const double* const* F, const double* co
     return DDA_OK;
 }
 
+// v6 solve (loopback, BJ): the whole iteration loop in one cooperative launch (k_dist_loop).  *ran is
+// false (nothing done) when the cooperative grid cannot give every partition a CTA: the caller runs v5.
+dda_status_t dist_v6_solve(dda_comm* c, const double* const* F, const double* const* d0, double* const* d,
+                           double tol, int32_t maxit, dda_status_t* status, int* it, bool* zero, double* bnorm_out,
+                           int* checks_out, bool* ran, cudaStream_t st) {
+    *zero = false;
+    *it = 0;
+    *ran = false;
+    const int P = (int)c->parts.size();
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_dist_loop, DDA_THREADS, 0);
+    if (per_sm > 3) per_sm = 3;
+    const int G = device_sms() * per_sm;
+    if (per_sm < 1 || G < P || P > kDPMax) return DDA_OK;   // not co-resident / too many: the caller runs v5
+    *ran = true;
+    DDA_TRY(halo_exchange_w(c, st, 4, kDinv));             // S_j of the halo rows
+    for (DistPart& D : c->parts) {
+        D.K->scaled_valid = false;
+        DDA_TRY(scaled_setup(D.K, st));
+    }
+    const bool have_d0 = d0 != nullptr;
+    if (have_d0) {                                          // q = K d0 over own rows (unscaled)
+        for (int p = 0; p < P; ++p) {
+            DistPart& D = c->parts[p];
+            if (d0[p]) DDA_CK(cudaMemcpyAsync(D.x, d0[p], 6 * sizeof(double) * D.n_own, cudaMemcpyDeviceToDevice, st));
+            else DDA_CK(cudaMemsetAsync(D.x, 0, 6 * sizeof(double) * D.n_own, st));
+        }
+        DDA_TRY(halo_exchange(c, st));
+        DDA_TRY(spmv_parts(c, false, st));
+    }
+    for (int p = 0; p < P; ++p) {
+        DistPart& D = c->parts[p];
+        k_v4_init<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, F[p], have_d0 ? D.q : nullptr,
+                                                   have_d0 ? d0[p] : nullptr, d[p], D.K->sfac, D.K->lfac,
+                                                   D.K->bj_w, D.rt, D.pA, D.part, D.ticket, D.scal);
+        DDA_LAUNCHED();
+    }
+    double s4[4];
+    DDA_TRY(allreduce_host_at(c, 8, 4, s4, st));
+    const double rho = s4[0], rr = s4[2], FF = s4[3], bnorm = std::sqrt(FF);
+    *bnorm_out = bnorm;
+    *checks_out = 0;
+    if (FF == 0.0) {                                        // reading Z2
+        for (int p = 0; p < P; ++p) DDA_CK(cudaMemsetAsync(d[p], 0, 6 * sizeof(double) * c->parts[p].n_own, st));
+        DDA_CK(cudaStreamSynchronize(st));
+        *zero = true;
+        *status = DDA_OK;
+        return DDA_OK;
+    }
+    // decided at setup (converged at the start, breakdown, maxit = 0): no loop, d = S^T x0 below
+    int pre = -1;
+    if (std::sqrt(rr) <= tol * bnorm) pre = DDA_OK;
+    else if (!(rho > 0.0) || !std::isfinite(rho)) pre = DDA_ERR_BREAKDOWN;
+    else if (maxit <= 0) pre = DDA_ERR_NO_CONVERGENCE;
+    // device tables: the partitions, their halo maps (owner partition, owner's local row), the CTA split
+    std::vector<DPart> h(P);
+    int64_t tot = 0;
+    for (DistPart& D : c->parts) tot += D.n_own;
+    int64_t cum = 0;
+    int prev = 0;
+    std::vector<int2> hm;
+    std::vector<size_t> hoff(P + 1, 0);
+    for (int p = 0; p < P; ++p) {
+        DistPart& D = c->parts[p];
+        const int nh = D.n_local - D.n_own;
+        hoff[p] = hm.size();
+        hm.resize(hm.size() + nh);
+        for (int q = 0; q < P; ++q) {
+            if (q == p) continue;
+            const DistPart& S = c->parts[q];
+            for (int t = 0; t < D.recv_counts[q]; ++t)
+                hm[hoff[p] + D.recv_off[q] + t] = make_int2(q, S.h_send_idx[S.send_off[p] + t]);
+        }
+        cum += D.n_own;
+        int c1 = (int)((G * cum) / (tot > 0 ? tot : 1));
+        if (c1 < prev + 1) c1 = prev + 1;                   // at least one CTA per partition ...
+        if (c1 > G - (P - 1 - p)) c1 = G - (P - 1 - p);     // ... and one left for each later one
+        if (p == P - 1) c1 = G;
+        h[p].A = own_view_sc(D);
+        h[p].rt = D.rt; h[p].p0 = D.pA; h[p].p1 = D.pB; h[p].q = D.q; h[p].x = d[p];
+        h[p].w = D.K->bj_w; h[p].lfac = D.K->lfac;
+        h[p].n_own = D.n_own; h[p].c0 = prev; h[p].c1 = c1;
+        prev = c1;
+    }
+    hoff[P] = hm.size();
+    const size_t tb = sizeof(DPart) * P, hb = sizeof(int2) * (hm.size() + 1), pb = sizeof(double) * 4 * (size_t)G;
+    char* ws = nullptr;
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&ws), tb + hb + pb + sizeof(DPState) + 256, st));
+    struct WsFree { char* b; cudaStream_t s; ~WsFree() { cudaStreamSynchronize(s); dev_free_on(b, s); } } wf{ws, st};
+    DPart* dparts = reinterpret_cast<DPart*>(ws);
+    int2* dh = reinterpret_cast<int2*>(ws + ((tb + 15) / 16) * 16);
+    double* dpart = reinterpret_cast<double*>(ws + ((tb + 15) / 16) * 16 + ((hb + 15) / 16) * 16);
+    DPState* dst = reinterpret_cast<DPState*>(dpart + 4 * (size_t)G);
+    for (int p = 0; p < P; ++p) h[p].hmap = dh + hoff[p];
+    DDA_CK(cudaMemcpyAsync(dparts, h.data(), tb, cudaMemcpyHostToDevice, st));
+    if (!hm.empty()) DDA_CK(cudaMemcpyAsync(dh, hm.data(), sizeof(int2) * hm.size(), cudaMemcpyHostToDevice, st));
+    DPArgs a{};
+    for (int p = 0; p < P; ++p) a.parts[p] = h[p];
+    a.gparts = dparts;
+    a.P = P;
+    a.part = dpart;
+    a.st = dst;
+    a.rho0 = rho;
+    a.thr = tol * bnorm;
+    a.maxit = maxit;
+    DPState z{};
+    DDA_CK(cudaMemsetAsync(dst, 0, sizeof(DPState), st));   // (struct padding: every byte defined)
+    if (pre < 0) {
+        void* args[] = {&a};
+        DDA_CK(cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_dist_loop), dim3(G), dim3(DDA_THREADS),
+                                           args, 0, st));
+        note_launch();
+    } else {
+        z.status = pre;
+        z.rr = rr;
+        DDA_CK(cudaMemcpyAsync(dst, &z, sizeof z, cudaMemcpyHostToDevice, st));
+    }
+    DPState out{};
+    DDA_CK(cudaMemcpyAsync(&out, dst, sizeof out, cudaMemcpyDeviceToHost, st));
+    DDA_CK(cudaStreamSynchronize(st));
+    for (int p = 0; p < P; ++p) {
+        DistPart& D = c->parts[p];
+        k_dp_final<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, d[p], ((out.k - 1) & 1) ? D.pB : D.pA, dst, D.K->sfac);
+        DDA_LAUNCHED();
+    }
+    DDA_CK(cudaStreamSynchronize(st));
+    *status = (dda_status_t)out.status;
+    *it = out.iters;
+    *checks_out = out.checks;
+    return DDA_OK;
+}
+
 }  // namespace
 
 extern "C" dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double* const* F, const double* const* d0,
@@ -1510,7 +1862,13 @@ extern "C" dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double* const* F,
         int it = 0, checks = 0;
         bool zero = false;
         double bnorm = 0.0;
-        if (v3) DDA_TRY(dist_scaled_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, st));
+        // v6 (loopback default): one persistent kernel for every partition; DDA_DIST_VERSION=5 / 4 / 3
+        // select the per-iteration launches (v5: peer-load halo, v4: halo copies, v3)
+        bool ran = false;
+        if (c->loopback && !(dve && (dve[0] == '3' || dve[0] == '4' || dve[0] == '5')))
+            DDA_TRY(dist_v6_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, &checks, &ran, st));
+        if (ran) {
+        } else if (v3) DDA_TRY(dist_scaled_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, st));
         else DDA_TRY(dist_v4_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, &checks, st));
         c->last_checks = checks;
         if (zero) return DDA_OK;

@@ -60,20 +60,22 @@ def test_spmv_dist_loopback(dda, prob, nparts):
     assert (np.abs(y - yo) <= 1e-12 * bound).all()
 
 
-@pytest.fixture(params=["v5", "v4", "v4_seq", "v3", "v2"])
+@pytest.fixture(params=["v6", "v5", "v4", "v4_seq", "v3", "v2"])
 def dist_version(request, monkeypatch):
-    """v5 = the v4 iteration with the halo read from the owners' rows (peer loads) and the allreduce
-    taken inside phase B (loopback default); v4 = one halo copy and one allreduce per iteration
+    """v6 = every partition in one persistent cooperative kernel, halo rows read from their owners'
+    r~ / p_old and every sum a fixed-order read of all partitions' partials (loopback default; NCCL runs
+    v4); v5 = the v4 iteration with the halo read from the owners' rows (peer loads) and the allreduce
+    taken inside phase B (DDA_DIST_VERSION=5); v4 = one halo copy and one allreduce per iteration
     (DDA_DIST_VERSION=4; the NCCL transport always runs it), phase A of the interior rows overlapped with
     the halo on a second stream; v4_seq = the same without the overlap (DDA_DIST_OVERLAP=0); v3 = two
-    halos and three allreduces
-    (DDA_DIST_VERSION=3); v2 = the unscaled loop (DDA_DIST_SCALED=0).  Read on every solve."""
+    halos and three allreduces (DDA_DIST_VERSION=3); v2 = the unscaled loop (DDA_DIST_SCALED=0).  Read on
+    every solve."""
     monkeypatch.delenv("DDA_DIST_SCALED", raising=False)
     monkeypatch.delenv("DDA_DIST_VERSION", raising=False)
     monkeypatch.delenv("DDA_DIST_OVERLAP", raising=False)
     if request.param == "v2":
         monkeypatch.setenv("DDA_DIST_SCALED", "0")
-    elif request.param in ("v3", "v4", "v4_seq"):
+    elif request.param in ("v3", "v4", "v4_seq", "v5"):
         monkeypatch.setenv("DDA_DIST_VERSION", request.param[1])
         if request.param == "v4_seq":
             monkeypatch.setenv("DDA_DIST_OVERLAP", "0")
