@@ -146,6 +146,7 @@ struct dda_matrix {
     size_t ws_bytes = 0;
     void* scratch = nullptr;        // small device scratch (result struct, flags)
     void* graph_engine = nullptr;   // cached CUDA-graph PCG engine (pcg_graph.cu)
+    void* tma_tiles = nullptr;      // spmv_tma.cu tile descriptors (int4 per 40-row tile), built on first use
     int32_t* full_ptr = nullptr;    // full-storage BSR6 copy for the configs[3] comparison (dda_spmv_full)
     int32_t* full_col = nullptr;
     double* full_val = nullptr;
@@ -179,6 +180,7 @@ namespace dda {
 dda_status_t ensure_workspace(dda_matrix* K, size_t bytes, cudaStream_t st);
 dda_status_t bj_setup(dda_matrix* K, cudaStream_t s, int32_t* bad_block);
 dda_status_t spmv(dda_matrix* K, const double* x, double* y, cudaStream_t s);
+dda_status_t spmv_tma(dda_matrix* K, const double* x, double* y, cudaStream_t s);
 void pcg_graph_free(void* g);
 dda_status_t scaled_setup(dda_matrix* K, cudaStream_t st);
 void matrix_free_impl(dda_matrix_t K, cudaStream_t* sync);

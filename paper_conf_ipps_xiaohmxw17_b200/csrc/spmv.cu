@@ -130,6 +130,8 @@ __global__ void k_full_fill(int32_t n, BsrView A, const int32_t* __restrict__ fp
 }  // namespace
 
 dda_status_t spmv(dda_matrix* K, const double* x, double* y, cudaStream_t s) {
+    const char* te = getenv("DDA_SPMV_TMA");
+    if (te && te[0] == '1') return spmv_tma(K, x, y, s);
     const Variant& V = kVariants[variant()];
     const SpmvKernel k = V.k;
     int g = spmv_grid(k);

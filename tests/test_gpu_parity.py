@@ -172,6 +172,21 @@ def test_spmv_unit_vectors_exact(dda):
         assert np.array_equal(K.spmv(x).cpu().numpy(), A[:, k]), k
 
 
+@pytest.mark.parametrize("name", ["tiny", "tiny_shuffled", "ragged_1k", "paper"])
+def test_spmv_tma_ablation_bit_identical(dda, name, monkeypatch):
+    """The TMA-staged SpMV ablation (spmv_tma.cu: bulk copies of each 40-row tile's diagonal and
+    forward blocks into shared memory, DDA_SPMV_TMA=1) does the default kernel's arithmetic in the same
+    order: y bit-identical, including rows whose blocks fall outside the staged ranges (shuffled)."""
+    P, O = case(name)
+    K = dda.build_from_problem(P)
+    x = torch.from_numpy(random_vector(P.n, 5)).cuda()
+    monkeypatch.delenv("DDA_SPMV_TMA", raising=False)
+    a = K.spmv(x).cpu().numpy()
+    monkeypatch.setenv("DDA_SPMV_TMA", "1")
+    b = K.spmv(x).cpu().numpy()
+    assert np.array_equal(a, b)
+
+
 def test_spmv_deterministic(dda):
     P, O = case("paper")
     K = dda.build_from_problem(P)
