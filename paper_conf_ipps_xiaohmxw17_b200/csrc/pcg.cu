@@ -656,7 +656,7 @@ extern "C" dda_status_t dda_solve_host_batch(int32_t nsys, dda_host_system* sys,
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&buf), 2 * slot_bytes + 2 * res_bytes, st));
     struct Res {
         char* b; cudaStream_t s; cudaStream_t cs = nullptr;
-        cudaEvent_t ev[7] = {};
+        cudaEvent_t ev[11] = {};
         ~Res() {
             if (cs) { cudaStreamSynchronize(cs); cudaStreamDestroy(cs); }
             cudaStreamSynchronize(s);
@@ -666,34 +666,44 @@ extern "C" dda_status_t dda_solve_host_batch(int32_t nsys, dda_host_system* sys,
     } res{buf, st};
     DDA_CK(cudaStreamCreateWithFlags(&res.cs, cudaStreamNonBlocking));
     for (cudaEvent_t& e : res.ev) DDA_CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-    cudaEvent_t start = res.ev[0], *in_ready = res.ev + 1, *in_free = res.ev + 3, *out_free = res.ev + 5;
+    // per slot: keys (bi, bj, pen) landed / values (e, g, kdiag) landed / right-hand side (F, d0) landed;
+    // the slot's inputs no longer read; the result buffer copied out
+    cudaEvent_t start = res.ev[0], *keys_ready = res.ev + 1, *vals_ready = res.ev + 3, *rhs_ready = res.ev + 5,
+                *in_free = res.ev + 7, *out_free = res.ev + 9;
     cudaStream_t cs = res.cs;
     DDA_CK(cudaEventRecord(start, st));                     // the buffer is allocated stream-ordered on st
     DDA_CK(cudaStreamWaitEvent(cs, start, 0));
     auto slot = [&](int k, int q) { return buf + (size_t)(k & 1) * slot_bytes + off[q]; };
     auto result = [&](int k) { return reinterpret_cast<double*>(buf + 2 * slot_bytes + (size_t)(k & 1) * res_bytes); };
+    // copy order = use order: the key arrays first, so the assembly's key sorts start while the
+    // 96 B / spring of e, g are still in flight (matters for the first system; later ones were copied
+    // during the previous solve)
     auto copy_in = [&](int k) -> cudaError_t {
         const dda_host_system& S = sys[k];
         const size_t N = 6 * (size_t)S.n_blocks, m = (size_t)S.n_springs;
         cudaError_t e = k >= 2 ? cudaStreamWaitEvent(cs, in_free[k & 1], 0) : cudaSuccess;
-        if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 0), S.kdiag, sizeof(double) * 6 * N, cudaMemcpyHostToDevice, cs);
-        if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 1), S.F, sizeof(double) * N, cudaMemcpyHostToDevice, cs);
-        if (e == cudaSuccess && S.d0) e = cudaMemcpyAsync(slot(k, 2), S.d0, sizeof(double) * N, cudaMemcpyHostToDevice, cs);
         if (m > 0) {
-            if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 3), S.pen, sizeof(double) * m, cudaMemcpyHostToDevice, cs);
-            if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 4), S.e, sizeof(double) * 6 * m, cudaMemcpyHostToDevice, cs);
-            if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 5), S.g, sizeof(double) * 6 * m, cudaMemcpyHostToDevice, cs);
             if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 6), S.bi, sizeof(int32_t) * m, cudaMemcpyHostToDevice, cs);
             if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 7), S.bj, sizeof(int32_t) * m, cudaMemcpyHostToDevice, cs);
+            if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 3), S.pen, sizeof(double) * m, cudaMemcpyHostToDevice, cs);
         }
-        if (e == cudaSuccess) e = cudaEventRecord(in_ready[k & 1], cs);
+        if (e == cudaSuccess) e = cudaEventRecord(keys_ready[k & 1], cs);
+        if (m > 0) {
+            if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 4), S.e, sizeof(double) * 6 * m, cudaMemcpyHostToDevice, cs);
+            if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 5), S.g, sizeof(double) * 6 * m, cudaMemcpyHostToDevice, cs);
+        }
+        if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 0), S.kdiag, sizeof(double) * 6 * N, cudaMemcpyHostToDevice, cs);
+        if (e == cudaSuccess) e = cudaEventRecord(vals_ready[k & 1], cs);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(slot(k, 1), S.F, sizeof(double) * N, cudaMemcpyHostToDevice, cs);
+        if (e == cudaSuccess && S.d0) e = cudaMemcpyAsync(slot(k, 2), S.d0, sizeof(double) * N, cudaMemcpyHostToDevice, cs);
+        if (e == cudaSuccess) e = cudaEventRecord(rhs_ready[k & 1], cs);
         return e;
     };
     DDA_CK(copy_in(0));
     for (int k = 0; k < nsys; ++k) {
         dda_host_system& S = sys[k];
         if (k + 1 < nsys) DDA_CK(copy_in(k + 1));          // overlaps this system's assembly and solve
-        DDA_CK(cudaStreamWaitEvent(st, in_ready[k & 1], 0));
+        DDA_CK(cudaStreamWaitEvent(st, keys_ready[k & 1], 0));
         if (k >= 2) DDA_CK(cudaStreamWaitEvent(st, out_free[k & 1], 0));
         const double* dk = reinterpret_cast<const double*>(slot(k, 0));
         dda_matrix_t K = nullptr;
@@ -701,8 +711,9 @@ extern "C" dda_status_t dda_solve_host_batch(int32_t nsys, dda_host_system* sys,
                                            reinterpret_cast<const int32_t*>(slot(k, 7)),
                                            reinterpret_cast<const double*>(slot(k, 3)),
                                            reinterpret_cast<const double*>(slot(k, 4)),
-                                           reinterpret_cast<const double*>(slot(k, 5)), st, nullptr, &K);
+                                           reinterpret_cast<const double*>(slot(k, 5)), st, vals_ready[k & 1], &K);
         if (s != DDA_OK) { S.status = s; return s; }
+        DDA_CK(cudaStreamWaitEvent(st, rhs_ready[k & 1], 0));
         s = dda_pcg_solve(K, reinterpret_cast<const double*>(slot(k, 1)),
                           S.d0 ? reinterpret_cast<const double*>(slot(k, 2)) : nullptr, result(k), tol, maxit, pc,
                           omega, &S.iters, &S.rel_res, stream);
