@@ -183,6 +183,21 @@ dda_status_t dda_pcg_solve(dda_matrix_t K, const double *F, const double *d0, do
                            void *stream);
 
 /*
+ * Optional residual history: registers a DEVICE buffer of 2*cap doubles that the
+ * following dda_pcg_solve calls on K fill, one pair per iteration k (0-based, k < min(iters, cap)):
+ *   hist[2k]     rho_{k+1} = r_{k+1}^T M^{-1} r_{k+1}, the PCG inner product of the new residual
+ *                (block-Jacobi: |L^{-1} r|^2, L the block Cholesky factors);
+ *   hist[2k + 1] |r_{k+1}|^2 when the exact stopping test (reading Z1) was evaluated at that
+ *                iteration, else NaN.
+ * Written by the block-Jacobi scaled engine (the default BJ path: persistent two-phase or
+ * single-reduction loop, or its CUDA-graph loop); other preconditioners leave the buffer untouched.
+ * buf = NULL with cap = 0 unregisters.  The buffer must stay valid while registered.  Registering
+ * or changing it rebuilds the cached solver engine on the next solve.  DDA_ERR_ARG: K NULL, cap < 0,
+ * or buf / cap inconsistent.
+ */
+dda_status_t dda_pcg_set_history(dda_matrix_t K, double *buf, int32_t cap);
+
+/*
  * End-to-end entry with HOST buffers (the benchmark's e2e leg): copies the
  * inputs host→device, assembles, sets up the preconditioner, solves, copies d
  * device→host and frees everything.  Arguments as dda_build_matrix and

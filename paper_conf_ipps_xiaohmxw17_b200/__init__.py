@@ -33,7 +33,7 @@ ABI_SYMBOLS = ("dda_build_matrix", "dda_update_values", "dda_matrix_info", "dda_
                "dda_dist_info", "dda_classify_contacts", "dda_contacts_classes",
                "dda_contact_init", "dda_contact_loads", "dda_contact_check", "dda_open_close",
                "dda_build_matrix_reordered", "dda_hsbcsr_build", "dda_hsbcsr_spmv", "dda_hsbcsr_export",
-               "dda_hsbcsr_free", "dda_contact_transfer", "dda_solve_host_batch")
+               "dda_hsbcsr_free", "dda_contact_transfer", "dda_solve_host_batch", "dda_pcg_set_history")
 
 _lib = None
 
@@ -88,6 +88,8 @@ def lib() -> C.CDLL:
         L.dda_solve_host.restype = st
         L.dda_solve_host_batch.argtypes = [I32, C.POINTER(HostSystem), D, I32, st, D, P]
         L.dda_solve_host_batch.restype = st
+        L.dda_pcg_set_history.argtypes = [P, P, I32]
+        L.dda_pcg_set_history.restype = st
         L.dda_launch_count.argtypes = []
         L.dda_launch_count.restype = I64
         L.dda_matrix_free.argtypes = [P]
@@ -287,6 +289,22 @@ class Matrix:
         if st not in (OK, ERR_NO_CONVERGENCE, ERR_BREAKDOWN) or (raise_on_fail and st != OK):
             raise DDAError(st, "dda_pcg_solve")
         return d, int(it.value), float(rr.value), int(st)
+
+    def set_history(self, hist=None):
+        """dda_pcg_set_history: register a device float64 tensor of shape (cap, 2) that the following
+        solves fill per iteration with (rho_k+1 = r^T M^-1 r, |r|^2 of the exact stopping test or NaN);
+        None unregisters.  The tensor must stay alive while registered."""
+        torch = _torch()
+        if hist is None:
+            _check(lib().dda_pcg_set_history(self.handle, None, 0), "dda_pcg_set_history")
+            self._hist = None
+            return
+        if not (isinstance(hist, torch.Tensor) and hist.is_cuda and hist.dtype == torch.float64
+                and hist.is_contiguous() and hist.dim() == 2 and hist.shape[1] == 2):
+            raise ValueError("hist must be a contiguous CUDA float64 tensor of shape (cap, 2)")
+        _check(lib().dda_pcg_set_history(self.handle, C.c_void_p(hist.data_ptr()), int(hist.shape[0])),
+               "dda_pcg_set_history")
+        self._hist = hist
 
     def pcg_engine(self, precond="bj") -> str:
         """The PCG engine dda_pcg_solve picks for this matrix (internal query, for byte accounting)."""

@@ -297,6 +297,7 @@ void dda::matrix_free_impl(dda_matrix_t K, cudaStream_t* sync) {
 extern "C" dda_status_t dda_build_matrix(int32_t n, const double* kdiag, int64_t m, const int32_t* bi,
                                          const int32_t* bj, const double* pen, const double* e, const double* g,
                                          void* stream, dda_matrix_t* out) {
+    DDA_NVTX("dda_build_matrix");
     return dda::build_matrix_impl(n, kdiag, m, bi, bj, pen, e, g, reinterpret_cast<cudaStream_t>(stream), nullptr,
                                   out);
 }
@@ -458,6 +459,7 @@ dda_status_t dda::build_matrix_impl(int32_t n, const double* kdiag, int64_t m, c
 
 extern "C" dda_status_t dda_update_values(dda_matrix_t K, const double* kdiag, int64_t m, const double* pen,
                                           const double* e, const double* g, void* stream) {
+    DDA_NVTX("dda_update_values");
     if (!K || !kdiag || m != K->m) return DDA_ERR_ARG;
     if (m > 0 && (!pen || !e || !g)) return DDA_ERR_ARG;
     if (m > 0 && ((reinterpret_cast<uintptr_t>(e) | reinterpret_cast<uintptr_t>(g)) & 15)) return DDA_ERR_ARG;

@@ -396,6 +396,7 @@ extern "C" void dda_contacts_free(dda_contacts_t C) {
 
 extern "C" dda_status_t dda_detect_contacts(int32_t n, const int32_t* vptr, const double* vxy, double d0,
                                             void* stream, dda_contacts_t* out) {
+    DDA_NVTX("dda_detect_contacts");
     if (!out) return DDA_ERR_ARG;
     *out = nullptr;
     if (n <= 0 || !vptr || !vxy || !(d0 > 0.0) || !isfinite(d0)) return DDA_ERR_ARG;
@@ -577,6 +578,7 @@ extern "C" dda_status_t dda_contacts_export(dda_contacts_t C, int32_t* i, int32_
 extern "C" dda_status_t dda_contact_springs(dda_contacts_t C, const double* cxy, double p_n, double shear_ratio,
                                             int32_t* bi, int32_t* bj, double* pen, double* e, double* g,
                                             void* stream) {
+    DDA_NVTX("dda_contact_springs");
     if (!C || !cxy || !(p_n >= 0.0) || !(shear_ratio >= 0.0) || !isfinite(p_n) || !isfinite(shear_ratio))
         return DDA_ERR_ARG;
     const int64_t m = C->count;
@@ -615,6 +617,7 @@ extern "C" dda_status_t dda_contact_springs(dda_contacts_t C, const double* cxy,
 // 2-bit radix sort of the class keys ("scan and radix sort methods are used to classify or abandon
 // data") and one gather per field.
 extern "C" dda_status_t dda_classify_contacts(dda_contacts_t C, double sin_tol, void* stream) {
+    DDA_NVTX("dda_classify_contacts");
     if (!C || !(sin_tol >= 0.0) || !(sin_tol < 1.0) || C->classified) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     const int64_t m = C->count;

@@ -16,6 +16,10 @@
 
 #include "dda.h"
 
+// NVTX ranges on the C ABI entry points (SURVEY §5 tracing): header-only NVTX v3, a no-op unless a
+// tool (nsys, ncu --nvtx) injects itself, so the ranges cost nothing in normal runs
+#include <nvtx3/nvToolsExt.h>
+
 #ifndef DDA_THREADS
 #define DDA_THREADS 256
 #endif
@@ -60,6 +64,14 @@ void dev_free(void* p);   // on the legacy default stream
         cudaError_t _e = cudaGetLastError();           \
         if (_e != cudaSuccess) return dda::cuda_fail(_e); \
     } while (0)
+
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange&) = delete;
+    NvtxRange& operator=(const NvtxRange&) = delete;
+};
+#define DDA_NVTX(name) ::dda::NvtxRange dda_nvtx_range_(name)
 
 // ------------------------------------------------------------------ device-side load helpers
 
@@ -152,6 +164,8 @@ struct dda_matrix {
     double* full_val = nullptr;
     int64_t graph_iters = 0;        // loop-body launches issued inside graphs (launch accounting)
     int last_checks = 0;            // scaled engine: exact stopping tests in the last solve
+    double* hist = nullptr;         // residual history (dda_pcg_set_history): [hist_cap][2] device doubles
+    int hist_cap = 0;
     // NEXT-2 internal block order (dda_build_matrix_reordered): the arrays above are in the internal
     // (RCM) numbering; rperm[new] = user id, rinv[user] = new; vectors are permuted at the ABI
     int32_t* rperm = nullptr;

@@ -1367,6 +1367,7 @@ dda_status_t spmv_parts(dda_comm* c, bool dot, cudaStream_t st) {
     } while (0)
 
 extern "C" dda_status_t dda_spmv_dist(dda_comm_t c, const double* const* x_own, double* const* y_own, void* stream) {
+    DDA_NVTX("dda_spmv_dist");
     if (!c || !x_own || !y_own) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     for (size_t p = 0; p < c->parts.size(); ++p) {
@@ -1842,6 +1843,7 @@ dda_status_t dist_v6_solve(dda_comm* c, const double* const* F, const double* co
 extern "C" dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double* const* F, const double* const* d0,
                                            double* const* d, double tol, int32_t maxit, dda_precond_t pc,
                                            int32_t* iters, double* rel_res, void* stream) {
+    DDA_NVTX("dda_pcg_solve_dist");
     if (iters) *iters = 0;
     if (rel_res) *rel_res = 0.0;
     if (!c || !F || !d || !(tol > 0.0) || maxit < 0) return DDA_ERR_ARG;

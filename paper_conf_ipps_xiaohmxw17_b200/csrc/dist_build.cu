@@ -139,6 +139,7 @@ extern "C" dda_status_t dda_build_matrix_dist(dda_comm_t c, int32_t part, int32_
                                               const double* kdiag_own, int64_t m, const int32_t* bi,
                                               const int32_t* bj, const double* pen, const double* e,
                                               const double* g, void* stream, dda_matrix_t* out) {
+    DDA_NVTX("dda_build_matrix_dist");
     using namespace dda;
     if (!out) return DDA_ERR_ARG;
     *out = nullptr;

@@ -120,6 +120,7 @@ extern "C" void dda_hsbcsr_free(dda_hsbcsr_t H) {
 }
 
 extern "C" dda_status_t dda_hsbcsr_build(dda_matrix_t K, void* stream, dda_hsbcsr_t* out) {
+    DDA_NVTX("dda_hsbcsr_build");
     using namespace dda;
     if (!out) return DDA_ERR_ARG;
     *out = nullptr;
@@ -156,6 +157,7 @@ extern "C" dda_status_t dda_hsbcsr_build(dda_matrix_t K, void* stream, dda_hsbcs
 }
 
 extern "C" dda_status_t dda_hsbcsr_spmv(dda_hsbcsr_t H, const double* x, double* y, void* stream) {
+    DDA_NVTX("dda_hsbcsr_spmv");
     using namespace dda;
     if (!H || !x || !y || x == y) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);

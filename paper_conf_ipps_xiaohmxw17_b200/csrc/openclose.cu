@@ -272,6 +272,7 @@ extern "C" dda_status_t dda_contact_init(dda_contacts_t C, int32_t* state, void*
 
 extern "C" dda_status_t dda_contact_loads(dda_contacts_t C, const double* e, const double* g, const double* pen,
                                           const double* F, double* out, void* stream) {
+    DDA_NVTX("dda_contact_loads");
     using namespace dda;
     if (!oc_ready(C) || !out || (C->count > 0 && (!e || !g || !pen))) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
@@ -284,6 +285,7 @@ extern "C" dda_status_t dda_contact_check(dda_contacts_t C, const double* d, con
                                           double p_n, double shear_ratio, double tan_phi, double open_tol,
                                           int32_t* state, double* pen, int32_t* cat, int32_t* cat_order,
                                           int64_t* counts, void* stream) {
+    DDA_NVTX("dda_contact_check");
     using namespace dda;
     if (!oc_ready(C) || !counts || !(p_n >= 0.0) || !(shear_ratio >= 0.0) || !(tan_phi >= 0.0) ||
         !(open_tol >= 0.0) || !isfinite(p_n) || !isfinite(shear_ratio) || !isfinite(tan_phi) || !isfinite(open_tol))
@@ -298,6 +300,7 @@ extern "C" dda_status_t dda_open_close(dda_matrix_t K, dda_contacts_t C, const d
                                        double tan_phi, double open_tol, double tol, int32_t maxit, int32_t max_oc,
                                        int32_t* state, double* pen, double* d, int32_t* oc_iters,
                                        int32_t* pcg_iters, int32_t* converged, double* rel_res, void* stream) {
+    DDA_NVTX("dda_open_close");
     using namespace dda;
     if (oc_iters) *oc_iters = 0;
     if (pcg_iters) *pcg_iters = 0;
@@ -378,6 +381,7 @@ __global__ void k_tr_search(int64_t m, const int32_t* __restrict__ v, const int3
 
 extern "C" dda_status_t dda_contact_transfer(dda_contacts_t prev, const int32_t* prev_state, dda_contacts_t cur,
                                              int32_t* state, int64_t* matched, void* stream) {
+    DDA_NVTX("dda_contact_transfer");
     using namespace dda;
     if (!prev || !cur || (prev->count > 0 && !prev_state) || (cur->count > 0 && !state)) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);

@@ -518,6 +518,7 @@ extern "C" int dda__pcg_engine(dda_matrix_t K, int pc) { return K ? pcg_engine(K
 extern "C" dda_status_t dda_pcg_solve(dda_matrix_t K, const double* F, const double* d0, double* d, double tol,
                                       int32_t maxit, dda_precond_t pc, double omega, int32_t* iters,
                                       double* rel_res, void* stream) {
+    DDA_NVTX("dda_pcg_solve");
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (!K) return DDA_ERR_ARG;
     if (K->rperm) return dda::ro_pcg(K, F, d0, d, tol, maxit, pc, omega, iters, rel_res, st);
@@ -549,6 +550,7 @@ extern "C" dda_status_t dda_solve_host(int32_t n, const double* kdiag, int64_t m
                                        const double* F, const double* d0, double* d, double tol, int32_t maxit,
                                        dda_precond_t pc, double omega, int32_t* iters, double* rel_res,
                                        void* stream) {
+    DDA_NVTX("dda_solve_host");
     if (n <= 0 || m < 0 || !kdiag || !F || !d) return DDA_ERR_ARG;
     if (m > 0 && (!bi || !bj || !pen || !e || !g)) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
@@ -627,6 +629,7 @@ extern "C" dda_status_t dda_solve_host(int32_t n, const double* kdiag, int64_t m
 // its device->host copy (out_free).
 extern "C" dda_status_t dda_solve_host_batch(int32_t nsys, dda_host_system* sys, double tol, int32_t maxit,
                                              dda_precond_t pc, double omega, void* stream) {
+    DDA_NVTX("dda_solve_host_batch");
     if (nsys < 0 || (nsys > 0 && !sys)) return DDA_ERR_ARG;
     int32_t nmax = 0;
     int64_t mmax = 0;

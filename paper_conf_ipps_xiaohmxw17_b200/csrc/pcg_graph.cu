@@ -77,6 +77,8 @@ struct GArgs {           // constant for a (matrix, preconditioner): baked into 
     int use_cond;        // 0 only for the internal phase-timing hook (kernels launched outside the graph)
     unsigned long long* trace;   // k_sp_loop timeline [iter][cta][4] (%globaltimer), null = off (internal hook)
     int trace_iters;
+    double* hist;        // residual history [hist_cap][2] (dda_pcg_set_history), null = off
+    int hist_cap;
 };
 
 __device__ __forceinline__ unsigned long long gtimer() {
@@ -658,6 +660,10 @@ __global__ void __launch_bounds__(DDA_THREADS, 4) k_s_update(const GArgs a, cuda
         State* st = a.st;
         st->pend = 1;                                       // x += alpha p_k: next SpMV or k_s_final
         const double rho1 = tot[0];
+        if (a.hist && k < a.hist_cap) {
+            a.hist[2 * (size_t)k] = rho1;
+            a.hist[2 * (size_t)k + 1] = __longlong_as_double(0x7FF8000000000000ll);
+        }
         st->iters = k + 1;
         const double thr = a.ca->tol * st->bnorm;
         if (rho1 == 0.0) {                                  // r~ = 0 exactly: r = L r~ = 0
@@ -697,6 +703,7 @@ __global__ void __launch_bounds__(DDA_THREADS, 4) k_s_check(const GArgs a, cudaG
         st->maybe = 0;
         st->checks += 1;
         st->rr = tot[0];
+        if (a.hist && st->k < a.hist_cap) a.hist[2 * (size_t)st->k + 1] = tot[0];
         if (sqrt(tot[0]) <= a.ca->tol * st->bnorm) {
             st->status = DDA_OK;
             st->k = st->k + 1;
@@ -875,6 +882,10 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_loop(const GArgs a) {
         const double rho1 = btot[0];
         pend = 1;                                           // x += alpha p_k: next phase A or k_s_final
         iters = k + 1;
+        if (a.hist && k < a.hist_cap && blockIdx.x == 0 && threadIdx.x == 0) {
+            a.hist[2 * (size_t)k] = rho1;
+            a.hist[2 * (size_t)k + 1] = __longlong_as_double(0x7FF8000000000000ll);
+        }
         if (rho1 == 0.0) { status = DDA_OK; rr_last = 0.0; k = k + 1; break; }
         if (isfinite(rho1) && !(0.999 * btot[1] > thr * thr)) {
             // phase C (rare): the exact stopping test |L r~| <= tol ||F|| (reading Z1; see k_s_update)
@@ -890,6 +901,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_loop(const GArgs a) {
             double cv[1] = {rl}, ctot[1];
             grid_allsum<1>(a, grid, 3, cv, ctot);   // slot 3: slot 0 is rewritten by the next phase A
             const double rr = ctot[0];
+            if (a.hist && k < a.hist_cap && blockIdx.x == 0 && threadIdx.x == 0) a.hist[2 * (size_t)k + 1] = rr;
             checks += 1;
             rr_last = rr;
             if (sqrt(rr) <= thr) { status = DDA_OK; k = k + 1; break; }
@@ -1137,6 +1149,10 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_cg1(const GArgs a) {
         grid_allsum<3>(a, grid, cur ? 4 : 1, bv, btot);
         const double rho1 = btot[0];
         iters = k + 1;
+        if (a.hist && k < a.hist_cap && blockIdx.x == 0 && threadIdx.x == 0) {
+            a.hist[2 * (size_t)k] = rho1;
+            a.hist[2 * (size_t)k + 1] = __longlong_as_double(0x7FF8000000000000ll);
+        }
         if (rho1 == 0.0) { status = DDA_OK; rr_last = 0.0; k = k + 1; break; }
         if (isfinite(rho1) && !(0.999 * btot[2] > thr * thr)) {
             double rl = 0.0;   // phase C: the exact test |L r~| <= tol ||F|| (reading Z1)
@@ -1150,6 +1166,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_cg1(const GArgs a) {
             }
             double cv[1] = {rl}, ctot[1];
             grid_allsum<1>(a, grid, 0, cv, ctot);
+            if (a.hist && k < a.hist_cap && blockIdx.x == 0 && threadIdx.x == 0) a.hist[2 * (size_t)k + 1] = ctot[0];
             checks += 1;
             rr_last = ctot[0];
             if (sqrt(ctot[0]) <= thr) { status = DDA_OK; k = k + 1; break; }
@@ -1456,6 +1473,8 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         a.ilu_flags_b = K->ilu_flags ? K->ilu_flags + 2 * (size_t)K->n : nullptr;
         a.ilu_counters = K->ilu_flags ? K->ilu_flags + 3 * (size_t)K->n + 2 : nullptr;
         a.ilu_order = K->ilu_order;
+        a.hist = K->hist;          // (the graph loop bakes it at capture: dda_pcg_set_history drops the engine)
+        a.hist_cap = K->hist_cap;
         a.su = K->sc_upper;
         a.lfac = K->lfac;
         a.sfac = K->sfac;
@@ -1553,6 +1572,8 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     if (G->G_persist) {
         a.trace = g_trace;
         a.trace_iters = g_trace_iters;
+        a.hist = K->hist;
+        a.hist_cap = K->hist_cap;
         void* kargs[] = {reinterpret_cast<void*>(&a)};
         DDA_CK(cudaLaunchCooperativeKernel(persist_kernel, dim3(G->G_persist),
                                            dim3(DDA_THREADS), kargs, 0, st));
@@ -1719,4 +1740,20 @@ extern "C" int dda__time_ks_variants(dda_matrix_t K, const double* F, double* d,
     }
     cudaEventDestroy(e0); cudaEventDestroy(e1);
     return cudaGetLastError() == cudaSuccess ? 0 : -3;
+}
+
+// Residual history (dda.h): registered per matrix; a change drops the cached engine, whose CUDA graph
+// bakes the pointer
+extern "C" dda_status_t dda_pcg_set_history(dda_matrix_t K, double* buf, int32_t cap) {
+    if (!K || cap < 0 || (buf == nullptr) != (cap == 0)) return DDA_ERR_ARG;
+    if (K->hist != buf || K->hist_cap != cap) {
+        if (K->graph_engine) {
+            cudaDeviceSynchronize();
+            dda::pcg_graph_free(K->graph_engine);
+            K->graph_engine = nullptr;
+        }
+        K->hist = buf;
+        K->hist_cap = cap;
+    }
+    return DDA_OK;
 }

@@ -218,6 +218,7 @@ dda_status_t bj_setup_rows(dda_matrix* K, int32_t nrows, cudaStream_t st, int32_
 using namespace dda;
 
 extern "C" dda_status_t dda_bj_setup(dda_matrix_t K, double* dinv_full, int32_t* bad_block, void* stream) {
+    DDA_NVTX("dda_bj_setup");
     if (!K) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     if (K->rperm) return ro_bj_setup(K, dinv_full, bad_block, st);
@@ -226,6 +227,7 @@ extern "C" dda_status_t dda_bj_setup(dda_matrix_t K, double* dinv_full, int32_t*
 
 extern "C" dda_status_t dda_precond_apply(dda_matrix_t K, dda_precond_t pc, double omega, const double* r, double* z,
                                           void* stream) {
+    DDA_NVTX("dda_precond_apply");
     if (!K || !r || !z || r == z) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     return K->rperm ? ro_precond(K, pc, omega, r, z, st) : dda::precond_apply(K, pc, omega, r, z, st);

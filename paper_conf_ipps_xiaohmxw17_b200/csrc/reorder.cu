@@ -87,6 +87,7 @@ int32_t bfs(const Graph& G, int32_t root, std::vector<int32_t>& level, std::vect
 }  // namespace
 
 extern "C" dda_status_t dda_rcm_order(int32_t n, int64_t m, const int32_t* bi, const int32_t* bj, int32_t* perm) {
+    DDA_NVTX("dda_rcm_order");
     if (n <= 0 || m < 0 || !perm || (m > 0 && (!bi || !bj))) return DDA_ERR_ARG;
     for (int64_t s = 0; s < m; ++s)
         if (bi[s] < 0 || bi[s] >= n || bj[s] < 0 || bj[s] >= n || bi[s] == bj[s]) return DDA_ERR_ARG;
@@ -299,6 +300,7 @@ dda_status_t ro_export(dda_matrix* K, int32_t* row_ptr, int32_t* col_idx, int32_
 extern "C" dda_status_t dda_build_matrix_reordered(int32_t n, const double* kdiag, int64_t m, const int32_t* bi,
                                                    const int32_t* bj, const double* pen, const double* e,
                                                    const double* g, void* stream, dda_matrix_t* out) {
+    DDA_NVTX("dda_build_matrix_reordered");
     using namespace dda;
     if (!out) return DDA_ERR_ARG;
     *out = nullptr;

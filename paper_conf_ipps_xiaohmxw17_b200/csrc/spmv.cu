@@ -183,12 +183,14 @@ dda_status_t dda::spmv_full(dda_matrix* K, const double* x, double* y, cudaStrea
 }
 
 extern "C" dda_status_t dda_spmv_full(dda_matrix_t K, const double* x, double* y, void* stream) {
+    DDA_NVTX("dda_spmv_full");
     if (!K || !x || !y || x == y) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     return K->rperm ? dda::ro_spmv(K, x, y, st, true) : dda::spmv_full(K, x, y, st);
 }
 
 extern "C" dda_status_t dda_spmv(dda_matrix_t K, const double* x, double* y, void* stream) {
+    DDA_NVTX("dda_spmv");
     if (!K || !x || !y || x == y) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     return K->rperm ? dda::ro_spmv(K, x, y, st, false) : dda::spmv(K, x, y, st);

@@ -441,6 +441,42 @@ def test_solve_host_e2e(dda):
     assert np.array_equal(d, d2.cpu().numpy())
 
 
+@pytest.mark.parametrize("loop", ["2phase", "cg1", "graph"])
+def test_residual_history(dda, loop, monkeypatch):
+    """dda_pcg_set_history: per iteration rho_{k+1} = r^T M^-1 r and, where the exact stopping test
+    ran, |r|^2.  rho_k is checked against r_k = F - K d_k recomputed from a maxit = k solve (d_k from
+    the same engine; r^T D^-1 r through dda_precond_apply); the exact entries against the reported
+    true residual at the stop; entries past the last iteration stay untouched."""
+    monkeypatch.setenv("DDA_SCALED_CG1", "1" if loop == "cg1" else "0")
+    P, O = case("paper")
+    K = dda.build_from_problem(P)
+    F = torch.from_numpy(P.F).cuda()
+    try:
+        _set_engine(dda, 2, 0 if loop == "graph" else 1)
+        hist = torch.full((400, 2), -1.0, dtype=torch.float64, device="cuda")
+        K.set_history(hist)
+        d, it, rr, st = K.pcg_solve(F)
+        h = hist.cpu().numpy()
+        assert st == dda.OK and 0 < it < 400
+        assert np.all(np.isfinite(h[:it, 0])) and np.all(h[:it, 0] > 0) and np.all(h[it:] == -1.0)
+        exact = ~np.isnan(h[:it, 1])
+        assert exact.sum() == K.last_checks() and exact[it - 1]
+        fn = float(np.linalg.norm(P.F))
+        assert abs(np.sqrt(h[it - 1, 1]) / fn - rr) <= 1e-3 * rr          # recursive vs true residual at the stop
+        assert np.sqrt(h[it - 1, 1]) <= 1e-10 * fn
+        for k in (1, 5, 20):
+            dk, itk, _, _ = K.pcg_solve(F, tol=1e-300, maxit=k)
+            r = F - K.spmv(dk)
+            rho = float(torch.dot(r, K.precond_apply(r, precond="bj")))
+            assert abs(hist[k - 1, 0].item() - rho) <= 1e-8 * rho, (k, hist[k - 1, 0].item(), rho)
+        K.set_history(None)
+        hist.fill_(-1.0)
+        K.pcg_solve(F)
+        assert bool((hist == -1.0).all())
+    finally:
+        _set_engine(dda, -1, -1)
+
+
 def test_solve_host_batch(dda):
     """Streamed batch (dda_solve_host_batch): systems of different sizes, one with a warm start and
     one repeated (so both input slots are refilled), each bit-identical to dda_solve_host; pinned and
