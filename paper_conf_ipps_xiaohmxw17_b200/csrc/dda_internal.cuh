@@ -109,6 +109,14 @@ __device__ __forceinline__ void cta_barrier() {
     __syncwarp();
     __syncthreads();
 }
+// the same with the NON-aligned barrier.sync, defined for threads of a warp that arrive separately:
+// used in the last-CTA reductions of the CUDA-graph loop kernels, where synccheck reported the
+// aligned form as divergent under programmatic dependent launch (and the persistent loops keep the
+// aligned one: the non-aligned form measured slower there)
+__device__ __forceinline__ void cta_barrier_na() {
+    __syncwarp();
+    asm volatile("barrier.sync 0;" ::: "memory");
+}
 
 __device__ __forceinline__ double warp_sum(double v) {
 #pragma unroll

@@ -115,7 +115,7 @@ __device__ __forceinline__ bool grid_reduce_last(const GArgs& a, double (&v)[NV]
 #pragma unroll
         for (int k = 0; k < NV; ++k) red[k][wib] = v[k];
     }
-    cta_barrier();
+    cta_barrier_na();
     if (threadIdx.x == 0) {
 #pragma unroll
         for (int k = 0; k < NV; ++k) {
@@ -127,7 +127,7 @@ __device__ __forceinline__ bool grid_reduce_last(const GArgs& a, double (&v)[NV]
         const unsigned t = atomicAdd(&a.st->ticket, 1u);
         last = (t == gridDim.x - 1);
     }
-    cta_barrier();
+    cta_barrier_na();
     if (!last) return false;
     __threadfence();
     const int G = gridDim.x;
@@ -137,13 +137,13 @@ __device__ __forceinline__ bool grid_reduce_last(const GArgs& a, double (&v)[NV]
         for (int j = threadIdx.x; j < G; j += DDA_THREADS) s += __ldcg(a.part + k * a.Gmax + j);
         red[k][threadIdx.x] = s;
     }
-    cta_barrier();
+    cta_barrier_na();
     for (int h = DDA_THREADS / 2; h > 0; h >>= 1) {      // fixed-shape tree
         if (threadIdx.x < h) {
 #pragma unroll
             for (int k = 0; k < NV; ++k) red[k][threadIdx.x] += red[k][threadIdx.x + h];
         }
-        cta_barrier();
+        cta_barrier_na();
     }
 #pragma unroll
     for (int k = 0; k < NV; ++k) tot[k] = red[k][0];
