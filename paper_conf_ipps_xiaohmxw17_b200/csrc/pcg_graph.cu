@@ -1408,6 +1408,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         // kernels), SSOR-AI to the unscaled graph engine.
         int per_sm = 0;
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, persist_kernel, DDA_THREADS, 0);
+        if (env_int("DDA_SIMULATE_NO_COOP", 0)) per_sm = 0;   // test hook: exercise the fallback
         if (per_sm < 1) {
             trace("solve: cooperative grid does not fit, graph loop fallback");
             if (pc == DDA_PC_SSOR_AI)

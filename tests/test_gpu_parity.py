@@ -477,6 +477,20 @@ def test_residual_history(dda, loop, monkeypatch):
         _set_engine(dda, -1, -1)
 
 
+@pytest.mark.parametrize("pc", ["bj", "ssor_ai"])
+def test_cooperative_fallback(dda, pc, monkeypatch):
+    """When not even one CTA of the persistent kernel fits per SM (DDA_SIMULATE_NO_COOP stands in for a
+    caller context with a smaller shared-memory carve-out), the solve falls back before writing any
+    state: scaled BJ to the CUDA-graph while loop, SSOR-AI to the unscaled graph engine.  Same stop
+    rule; parity against the oracle (Z17)."""
+    P, O = case("paper")
+    monkeypatch.setenv("DDA_SIMULATE_NO_COOP", "1")
+    d, it = _pcg_parity(dda, P, O, pc)
+    monkeypatch.delenv("DDA_SIMULATE_NO_COOP")
+    d2, it2 = _pcg_parity(dda, P, O, pc)
+    assert abs(it - it2) <= 1 and np.linalg.norm(d - d2) <= 1e-9 * np.linalg.norm(d2)
+
+
 def test_solve_host_batch(dda):
     """Streamed batch (dda_solve_host_batch): systems of different sizes, one with a warm start and
     one repeated (so both input slots are refilled), each bit-identical to dda_solve_host; pinned and
