@@ -974,6 +974,192 @@ __global__ void __launch_bounds__(DDA_THREADS) k_dp_final(int n, double* d, cons
     }
 }
 
+// ---- v7 (loopback): one persistent cooperative kernel PER PARTITION ("rank"), the launches running
+// concurrently on their own streams, exactly the structure one process per GPU would run.
+//
+// Each rank's kernel runs k_sp_loop's iteration over its own rows with its own grid.  What crosses
+// ranks: the halo rows (read from the owners' r~ / p_old through the partition table, as in v6) and
+// every reduction, taken as a two-level fixed-order sum: the rank's CTA partials (grid barrier),
+// then the ranks' totals, which each rank's leader publishes to a slot set and announces on a shared
+// arrival counter; every CTA of every rank waits for all P arrivals of that epoch and sums the P
+// totals in rank order (a one-shot deterministic allreduce, identical everywhere).  The arrival
+// wait is also the inter-rank barrier that orders one phase's halo writes before the next phase's
+// reads.  Across GPUs the same code needs the partition table and the slot / counter words mapped over
+// NVLink (IPC handles) and system-scope fences; here they are one device's memory.  Every wait is
+// bounded (an error flag instead of a hang).
+__device__ __forceinline__ int ld_acquire(const int* p) {
+    int v;
+    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+constexpr int kRankSets = 4;                 // slot sets in rotation (a rank is at most one epoch ahead)
+struct RArgs {
+    const DPart* parts;                       // every rank's table entry (the owners' arrays)
+    int P, rank;
+    double* part;                             // this rank's CTA partials [4][gridDim]
+    double* slots;                            // [kRankSets][P][4] rank totals
+    unsigned* arrive;                         // shared arrival counter (monotone over epochs)
+    DPState* st;                              // this rank's result
+    int* err;                                 // set when a wait hit its bound
+    double rho0, thr;
+    int maxit;
+};
+
+template <int NV>
+__device__ __forceinline__ void rank_allsum(const RArgs& a, cg::grid_group& grid, int slot, unsigned& epoch,
+                                            double (&v)[NV], double (&tot)[NV]) {
+    __shared__ double red[NV][DDA_THREADS];
+    const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5, G = gridDim.x;
+#pragma unroll
+    for (int k = 0; k < NV; ++k) v[k] = warp_sum(v[k]);
+    if (lane == 0) {
+#pragma unroll
+        for (int k = 0; k < NV; ++k) red[k][wib] = v[k];
+    }
+    cta_barrier();
+    if (threadIdx.x == 0) {
+#pragma unroll
+        for (int k = 0; k < NV; ++k) {
+            double s = 0.0;
+            for (int w = 0; w < WPB; ++w) s += red[k][w];
+            a.part[(size_t)(slot + k) * G + blockIdx.x] = s;
+        }
+    }
+    grid.sync();
+    epoch += 1;
+    double* set = a.slots + (size_t)(epoch % kRankSets) * a.P * 4;
+    if (blockIdx.x == 0) {                   // the rank's total, in CTA order (a fixed-shape tree)
+#pragma unroll
+        for (int k = 0; k < NV; ++k) {
+            const double* part = a.part + (size_t)(slot + k) * G;
+            double s = 0.0;
+            for (int j = threadIdx.x; j < G; j += DDA_THREADS) s += *(volatile const double*)(part + j);
+            red[k][threadIdx.x] = s;
+        }
+        cta_barrier();
+        for (int h = DDA_THREADS / 2; h > 0; h >>= 1) {
+            if (threadIdx.x < h) {
+#pragma unroll
+                for (int k = 0; k < NV; ++k) red[k][threadIdx.x] += red[k][threadIdx.x + h];
+            }
+            cta_barrier();
+        }
+        if (threadIdx.x == 0) {
+#pragma unroll
+            for (int k = 0; k < NV; ++k) set[(size_t)a.rank * 4 + k] = red[k][0];
+            __threadfence();                 // (across GPUs: __threadfence_system)
+            atomicAdd(a.arrive, 1u);
+        }
+        cta_barrier();
+    }
+    if (threadIdx.x == 0) {                  // every rank's total of this epoch has arrived
+        const unsigned target = epoch * (unsigned)a.P;
+        unsigned long long spins = 0;
+        while ((int)(ld_acquire(reinterpret_cast<const int*>(a.arrive)) - (int)target) < 0) {
+            if (++spins > (1ull << 28)) { atomicExch(a.err, 1); break; }
+            __nanosleep(32);
+        }
+    }
+    cta_barrier();
+#pragma unroll
+    for (int k = 0; k < NV; ++k) {
+        double s = 0.0;
+        for (int q = 0; q < a.P; ++q) s += *(volatile const double*)(set + (size_t)q * 4 + k);
+        tot[k] = s;
+    }
+}
+
+__global__ void __launch_bounds__(DDA_THREADS, 3) k_rank_loop(const RArgs a) {
+    cg::grid_group grid = cg::this_grid();
+    const DPart& D = a.parts[a.rank];
+    const int lane = threadIdx.x & 31;
+    const int w0 = blockIdx.x * WPB + (threadIdx.x >> 5), W = gridDim.x * WPB;
+    const int n = D.n_own, ngrp = (n + 4) / 5;
+    const double thr = a.thr;
+    double rho = a.rho0, alpha = 0.0, beta = 0.0, rr_last = 0.0;
+    int k = 0, status = DDA_ERR_NO_CONVERGENCE, iters = 0, checks = 0, pend = 0;
+    unsigned epoch = 0;
+    for (;;) {
+        double* pnew = (k & 1) ? D.p1 : D.p0;
+        const double* pold = k == 0 ? D.rt : ((k & 1) ? D.p0 : D.p1);
+        const XFusedPeer xf{a.parts, D.rt, pold, D.hmap, n, k == 0 ? 0 : ((k & 1) ? 1 : 2), beta};
+        const double ap = alpha;
+        double acc = 0.0;
+        for_rows_c<SPMV_OFFDIAG, 5>(D.A, w0, W, xf, lane, [&](int i, bool ok, double y0, double y1) {
+            if (ok) {
+                const size_t o = 6 * (size_t)i + 2 * ccol_of(lane);
+                const double2 pv = xf(i, ccol_of(lane));
+                y0 += pv.x;
+                y1 += pv.y;
+                const double2 po = *reinterpret_cast<const double2*>(pold + o);
+                const double2 xo = *reinterpret_cast<const double2*>(D.x + o);
+                *reinterpret_cast<double2*>(D.x + o) = make_double2(xo.x + ap * po.x, xo.y + ap * po.y);
+                *reinterpret_cast<double2*>(D.q + o) = make_double2(y0, y1);
+                *reinterpret_cast<double2*>(pnew + o) = pv;
+                acc += pv.x * y0 + pv.y * y1;
+            }
+        });
+        double sv[1] = {acc}, stot[1];
+        rank_allsum<1>(a, grid, 0, epoch, sv, stot);
+        const double sigma = stot[0];
+        pend = 0;
+        if (!(sigma > 0.0) || !isfinite(sigma)) { status = DDA_ERR_BREAKDOWN; break; }
+        alpha = rho / sigma;
+        double rz = 0.0, lb = 0.0;
+        for (int grp = w0; grp < ngrp; grp += 2 * W) {
+            const Row5 RA = row5(grp, lane, n);
+            const Row5 RB = row5(grp + W, lane, n);
+            double ra = 0, qa = 0, rb = 0, qb = 0, wa = 0, wb = 0;
+            if (RA.valid) { ra = D.rt[RA.idx]; qa = D.q[RA.idx]; wa = __ldg(D.w + RA.i); }
+            if (RB.valid) { rb = D.rt[RB.idx]; qb = D.q[RB.idx]; wb = __ldg(D.w + RB.i); }
+            const double rva = RA.valid ? ra - alpha * qa : 0.0;
+            const double rvb = RB.valid ? rb - alpha * qb : 0.0;
+            if (RA.valid) D.rt[RA.idx] = rva;
+            if (RB.valid) D.rt[RB.idx] = rvb;
+            rz += rva * rva + rvb * rvb;
+            lb += wa * (rva * rva) + wb * (rvb * rvb);
+        }
+        double bv[2] = {rz, lb}, btot[2];
+        rank_allsum<2>(a, grid, 1, epoch, bv, btot);
+        const double rho1 = btot[0];
+        pend = 1;
+        iters = k + 1;
+        if (rho1 == 0.0) { status = DDA_OK; rr_last = 0.0; k = k + 1; break; }
+        if (isfinite(rho1) && !(0.999 * btot[1] > thr * thr)) {   // the exact test (reading Z1)
+            double rl = 0.0;
+            for (int grp = w0; grp < ngrp; grp += W) {
+                const Row5 R = row5(grp, lane, n);
+                const double rv = R.valid ? D.rt[R.idx] : 0.0;
+                const double o0 = tri_apply(D.lfac, R, rv, false);
+                const double o = R.valid ? o0 : 0.0;
+                rl += o * o;
+            }
+            double cv[1] = {rl}, ctot[1];
+            rank_allsum<1>(a, grid, 3, epoch, cv, ctot);
+            checks += 1;
+            rr_last = ctot[0];
+            if (sqrt(ctot[0]) <= thr) { status = DDA_OK; k = k + 1; break; }
+        }
+        k = k + 1;
+        if (!(rho1 > 0.0) || !isfinite(rho1)) { status = DDA_ERR_BREAKDOWN; break; }
+        beta = rho1 / rho;
+        rho = rho1;
+        if (k >= a.maxit) { status = DDA_ERR_NO_CONVERGENCE; break; }
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        DPState* st = a.st;
+        st->k = k;
+        st->iters = iters;
+        st->status = status;
+        st->alpha = alpha;
+        st->beta = beta;
+        st->rho = rho;
+        st->rr = rr_last;
+        st->pend = pend;
+        st->checks = checks;
+    }
+}
+
 int grid_of(const void* k, int cap_per_sm) {
     int per = 0;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k, DDA_THREADS, 0);
@@ -1710,13 +1896,14 @@ dda_status_t dist_v4_solve(dda_comm* c, const double* const* F, const double* co
 // false (nothing done) when the cooperative grid cannot give every partition a CTA: the caller runs v5.
 dda_status_t dist_v6_solve(dda_comm* c, const double* const* F, const double* const* d0, double* const* d,
                            double tol, int32_t maxit, dda_status_t* status, int* it, bool* zero, double* bnorm_out,
-                           int* checks_out, bool* ran, cudaStream_t st) {
+                           int* checks_out, bool* ran, cudaStream_t st, bool per_rank = false) {
     *zero = false;
     *it = 0;
     *ran = false;
     const int P = (int)c->parts.size();
     int per_sm = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_dist_loop, DDA_THREADS, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, per_rank ? (const void*)k_rank_loop : (const void*)k_dist_loop,
+                                                  DDA_THREADS, 0);
     if (per_sm > 3) per_sm = 3;
     const int G = device_sms() * per_sm;
     if (per_sm < 1 || G < P || P > kDPMax) return DDA_OK;   // not co-resident / too many: the caller runs v5
@@ -1813,7 +2000,55 @@ dda_status_t dist_v6_solve(dda_comm* c, const double* const* F, const double* co
     a.maxit = maxit;
     DPState z{};
     DDA_CK(cudaMemsetAsync(dst, 0, sizeof(DPState), st));   // (struct padding: every byte defined)
-    if (pre < 0) {
+    if (pre < 0 && per_rank) {
+        // v7: one cooperative kernel per rank, each on its own stream, all resident together (the grid is
+        // split evenly); the ranks meet only through the slot sets and the arrival counter
+        const int Gr = G / P;
+        const size_t pb_r = sizeof(double) * 4 * (size_t)Gr, sb = sizeof(double) * kRankSets * 4 * (size_t)P;
+        char* rw = nullptr;
+        DDA_CK(dev_alloc(reinterpret_cast<void**>(&rw), P * (pb_r + sizeof(DPState) + 64) + sb + 64, st));
+        struct RwFree { char* b; cudaStream_t s; ~RwFree() { cudaStreamSynchronize(s); dev_free_on(b, s); } } rf{rw, st};
+        double* slots = reinterpret_cast<double*>(rw);
+        unsigned* arrive = reinterpret_cast<unsigned*>(rw + sb);
+        int* err = reinterpret_cast<int*>(rw + sb + 16);
+        char* base = rw + sb + 64;
+        DDA_CK(cudaMemsetAsync(rw + sb, 0, 64, st));
+        std::vector<cudaStream_t> rs(P, nullptr);
+        cudaEvent_t ev0 = nullptr;
+        struct RsFree {
+            std::vector<cudaStream_t>& v; cudaEvent_t& e;
+            ~RsFree() { for (cudaStream_t x : v) if (x) cudaStreamDestroy(x); if (e) cudaEventDestroy(e); }
+        } rsf{rs, ev0};
+        DDA_CK(cudaEventCreateWithFlags(&ev0, cudaEventDisableTiming));
+        DDA_CK(cudaEventRecord(ev0, st));
+        std::vector<RArgs> ra(P);
+        for (int p = 0; p < P; ++p) {
+            DDA_CK(cudaStreamCreateWithFlags(&rs[p], cudaStreamNonBlocking));
+            DDA_CK(cudaStreamWaitEvent(rs[p], ev0, 0));
+            char* mine = base + (size_t)p * (pb_r + sizeof(DPState) + 64);
+            DPState* rst = reinterpret_cast<DPState*>(mine + pb_r);
+            DDA_CK(cudaMemsetAsync(rst, 0, sizeof(DPState), rs[p]));
+            ra[p] = RArgs{dparts, P, p, reinterpret_cast<double*>(mine), slots, arrive, rst, err, rho, tol * bnorm, maxit};
+        }
+        for (int p = 0; p < P; ++p) {       // all ranks are launched before any is waited on
+            void* args[] = {&ra[p]};
+            DDA_CK(cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_rank_loop), dim3(Gr),
+                                               dim3(DDA_THREADS), args, 0, rs[p]));
+            note_launch();
+        }
+        for (int p = 0; p < P; ++p) {
+            cudaEvent_t e;
+            DDA_CK(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+            DDA_CK(cudaEventRecord(e, rs[p]));
+            DDA_CK(cudaStreamWaitEvent(st, e, 0));
+            cudaEventDestroy(e);
+        }
+        DDA_CK(cudaMemcpyAsync(dst, ra[0].st, sizeof(DPState), cudaMemcpyDeviceToDevice, st));   // rank 0's copy
+        int herr = 0;
+        DDA_CK(cudaMemcpyAsync(&herr, err, sizeof(int), cudaMemcpyDeviceToHost, st));
+        DDA_CK(cudaStreamSynchronize(st));
+        if (herr) return DDA_ERR_CUDA;      // a rank waited past the bound on the others
+    } else if (pre < 0) {
         void* args[] = {&a};
         DDA_CK(cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_dist_loop), dim3(G), dim3(DDA_THREADS),
                                            args, 0, st));
@@ -1868,7 +2103,8 @@ extern "C" dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double* const* F,
         // select the per-iteration launches (v5: peer-load halo, v4: halo copies, v3)
         bool ran = false;
         if (c->loopback && !(dve && (dve[0] == '3' || dve[0] == '4' || dve[0] == '5')))
-            DDA_TRY(dist_v6_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, &checks, &ran, st));
+            DDA_TRY(dist_v6_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, &checks, &ran, st,
+                                  dve && dve[0] == '7'));
         if (ran) {
         } else if (v3) DDA_TRY(dist_scaled_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, st));
         else DDA_TRY(dist_v4_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, &checks, st));

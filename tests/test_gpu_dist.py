@@ -60,9 +60,11 @@ def test_spmv_dist_loopback(dda, prob, nparts):
     assert (np.abs(y - yo) <= 1e-12 * bound).all()
 
 
-@pytest.fixture(params=["v6", "v5", "v4", "v4_seq", "v3", "v2"])
+@pytest.fixture(params=["v7", "v6", "v5", "v4", "v4_seq", "v3", "v2"])
 def dist_version(request, monkeypatch):
-    """v6 = every partition in one persistent cooperative kernel, halo rows read from their owners'
+    """v7 = one persistent cooperative kernel PER partition, the launches running concurrently and
+    meeting only through published rank totals and an arrival counter (DDA_DIST_VERSION=7, the
+    one-process-per-GPU structure under loopback); v6 = every partition in one persistent cooperative kernel, halo rows read from their owners'
     r~ / p_old and every sum a fixed-order read of all partitions' partials (loopback default; NCCL runs
     v4); v5 = the v4 iteration with the halo read from the owners' rows (peer loads) and the allreduce
     taken inside phase B (DDA_DIST_VERSION=5); v4 = one halo copy and one allreduce per iteration
@@ -75,7 +77,7 @@ def dist_version(request, monkeypatch):
     monkeypatch.delenv("DDA_DIST_OVERLAP", raising=False)
     if request.param == "v2":
         monkeypatch.setenv("DDA_DIST_SCALED", "0")
-    elif request.param in ("v3", "v4", "v4_seq", "v5"):
+    elif request.param in ("v3", "v4", "v4_seq", "v5", "v7"):
         monkeypatch.setenv("DDA_DIST_VERSION", request.param[1])
         if request.param == "v4_seq":
             monkeypatch.setenv("DDA_DIST_OVERLAP", "0")

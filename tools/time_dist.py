@@ -1,6 +1,6 @@
 """Per-iteration cost of the partitioned solver (dda_pcg_solve_dist) with the loopback transport on
 one GPU.  v5 / v4 / v3 run the partitions' kernels one after another, so their time is the driver's
-overhead + the partitions' summed work; v6 runs every partition in one persistent kernel.  Not a
+overhead + the partitions' summed work; v6 runs every partition in one persistent kernel; v7 one persistent kernel per partition, concurrently.  Not a
 scaling measurement.  DDA_DIST_CHUNK selects the host-check chunk."""
 import json, os, sys, statistics
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
@@ -24,7 +24,7 @@ for nparts in (1, 2, 4):
                                    t["g"])
         keep.append(K)
         Fs.append(t["F"][6 * r0: 6 * r1].contiguous())
-    for ver in ("6", "5", "4", "4s", "3"):
+    for ver in ("7", "6", "5", "4", "4s", "3"):
         os.environ["DDA_DIST_VERSION"] = ver[0]
         os.environ["DDA_DIST_OVERLAP"] = "0" if ver == "4s" else "1"
         ms = []
