@@ -276,6 +276,24 @@ typedef struct dda_comm *dda_comm_t;
 dda_status_t dda_comm_unique_id(void *id128);
 dda_status_t dda_comm_init(int32_t nranks, int32_t rank, const void *id128, dda_comm_t *out);
 dda_status_t dda_comm_init_loopback(int32_t nparts, dda_comm_t *out);
+
+/*
+ * IPC transport (one partition per process; the processes may share a GPU or sit on NVLink-connected
+ * GPUs): no NCCL.  Each rank's partition buffers that peers read in place (halo send rows, r~ and the
+ * PCG direction vectors, the send lists) are exported as CUDA IPC handles; rank 0 also exports the
+ * arrival counter and slot sets the collectives use.  Sequence: dda_comm_init_ipc, build or attach the
+ * rank's partition (dda_build_matrix_dist / dda_dist_attach), dda_comm_ipc_export (blob NULL: *bytes =
+ * the blob size), exchange the blobs between the processes by any means (the caller's), then
+ * dda_comm_ipc_import with all blobs in rank order, each `bytes` long.  dda_pcg_solve_dist (BJ) then
+ * runs v7: one persistent cooperative kernel per rank, halo rows read from the owners' mapped arrays,
+ * every reduction a fixed-order one-shot sum through rank 0's slot sets, every wait bounded
+ * (DDA_ERR_CUDA if a peer never arrives).  nranks <= 8.  DDA_ERR_ARG: a blob from another rank count,
+ * a send list that does not match this rank's receive list, re-import, or no partition attached.
+ * Beyond the paper (multi-GPU is its future work).
+ */
+dda_status_t dda_comm_init_ipc(int32_t nranks, int32_t rank, dda_comm_t *out);
+dda_status_t dda_comm_ipc_export(dda_comm_t c, void *blob, int64_t *bytes);
+dda_status_t dda_comm_ipc_import(dda_comm_t c, const void *blobs, int64_t bytes);
 dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t K, int32_t n_own, const int32_t *send_counts,
                              const int32_t *send_idx, const int32_t *recv_counts, void *stream);
 dda_status_t dda_spmv_dist(dda_comm_t c, const double *const *x_own, double *const *y_own, void *stream);

@@ -33,7 +33,8 @@ ABI_SYMBOLS = ("dda_build_matrix", "dda_update_values", "dda_matrix_info", "dda_
                "dda_dist_info", "dda_classify_contacts", "dda_contacts_classes",
                "dda_contact_init", "dda_contact_loads", "dda_contact_check", "dda_open_close",
                "dda_build_matrix_reordered", "dda_hsbcsr_build", "dda_hsbcsr_spmv", "dda_hsbcsr_export",
-               "dda_hsbcsr_free", "dda_contact_transfer", "dda_solve_host_batch", "dda_pcg_set_history")
+               "dda_hsbcsr_free", "dda_contact_transfer", "dda_solve_host_batch", "dda_pcg_set_history",
+               "dda_comm_init_ipc", "dda_comm_ipc_export", "dda_comm_ipc_import")
 
 _lib = None
 
@@ -104,6 +105,12 @@ def lib() -> C.CDLL:
         L.dda_comm_init.restype = st
         L.dda_comm_init_loopback.argtypes = [I32, C.POINTER(P)]
         L.dda_comm_init_loopback.restype = st
+        L.dda_comm_init_ipc.argtypes = [I32, I32, C.POINTER(P)]
+        L.dda_comm_init_ipc.restype = st
+        L.dda_comm_ipc_export.argtypes = [P, P, C.POINTER(I64)]
+        L.dda_comm_ipc_export.restype = st
+        L.dda_comm_ipc_import.argtypes = [P, P, I64]
+        L.dda_comm_ipc_import.restype = st
         L.dda_dist_attach.argtypes = [P, I32, P, I32, P, P, P, P]
         L.dda_dist_attach.restype = st
         L.dda_spmv_dist.argtypes = [P, P, P, P]
@@ -482,6 +489,27 @@ class Comm:
         h = C.c_void_p()
         _check(lib().dda_comm_init_loopback(int(nparts), C.byref(h)), "dda_comm_init_loopback")
         return cls(h, nparts)
+
+    @classmethod
+    def ipc(cls, nranks: int, rank: int) -> "Comm":
+        """dda_comm_init_ipc: one partition per process, peers' buffers mapped with CUDA IPC handles
+        (exchange the ipc_export() blobs by any means, then ipc_import them in rank order)."""
+        h = C.c_void_p()
+        _check(lib().dda_comm_init_ipc(int(nranks), int(rank), C.byref(h)), "dda_comm_init_ipc")
+        return cls(h, 1)
+
+    def ipc_export(self) -> bytes:
+        n = C.c_int64()
+        _check(lib().dda_comm_ipc_export(self._h, None, C.byref(n)), "dda_comm_ipc_export")
+        buf = C.create_string_buffer(n.value)
+        _check(lib().dda_comm_ipc_export(self._h, buf, C.byref(n)), "dda_comm_ipc_export")
+        return buf.raw[:n.value]
+
+    def ipc_import(self, blobs):
+        size = len(blobs[0])
+        assert all(len(b) == size for b in blobs)
+        buf = C.create_string_buffer(b"".join(blobs), size * len(blobs))
+        _check(lib().dda_comm_ipc_import(self._h, buf, size), "dda_comm_ipc_import")
 
     def attach(self, part: int, K: "Matrix", lp, stream=None):
         sc = np.ascontiguousarray(lp.send_counts, np.int32)

@@ -781,6 +781,7 @@ struct DPart {
 struct DPState {
     double alpha, beta, rho, rr;
     int k, iters, status, pend, checks;
+    unsigned epoch_end;   // v7: the arrival epoch the loop ended at (the IPC transport continues from it)
 };
 constexpr int kDPMax = 8;   // partitions held in the kernel's parameter block (more: v5)
 struct DPArgs {
@@ -987,18 +988,21 @@ __global__ void __launch_bounds__(DDA_THREADS) k_dp_final(int n, double* d, cons
 // reads.  Across GPUs the same code needs the partition table and the slot / counter words mapped over
 // NVLink (IPC handles) and system-scope fences; here they are one device's memory.  Every wait is
 // bounded (an error flag instead of a hang).
-__device__ __forceinline__ int ld_acquire(const int* p) {
+__device__ __forceinline__ int ld_acquire(const int* p) {   // system scope: the counter may be a peer's
     int v;
-    asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    asm volatile("ld.acquire.sys.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
     return v;
 }
+constexpr int kSlotStride = 16;              // doubles per rank in a slot set
+constexpr size_t kSyncHdr = 64;              // IPC sync buffer: counter, error flag; the slot sets follow
 constexpr int kRankSets = 4;                 // slot sets in rotation (a rank is at most one epoch ahead)
 struct RArgs {
     const DPart* parts;                       // every rank's table entry (the owners' arrays)
     int P, rank;
     double* part;                             // this rank's CTA partials [4][gridDim]
-    double* slots;                            // [kRankSets][P][4] rank totals
+    double* slots;                            // [kRankSets][P][kSlotStride] rank totals
     unsigned* arrive;                         // shared arrival counter (monotone over epochs)
+    unsigned epoch0;                          // epochs already consumed on this counter
     DPState* st;                              // this rank's result
     int* err;                                 // set when a wait hit its bound
     double rho0, thr;
@@ -1027,7 +1031,7 @@ __device__ __forceinline__ void rank_allsum(const RArgs& a, cg::grid_group& grid
     }
     grid.sync();
     epoch += 1;
-    double* set = a.slots + (size_t)(epoch % kRankSets) * a.P * 4;
+    double* set = a.slots + (size_t)(epoch % kRankSets) * a.P * kSlotStride;
     if (blockIdx.x == 0) {                   // the rank's total, in CTA order (a fixed-shape tree)
 #pragma unroll
         for (int k = 0; k < NV; ++k) {
@@ -1046,9 +1050,9 @@ __device__ __forceinline__ void rank_allsum(const RArgs& a, cg::grid_group& grid
         }
         if (threadIdx.x == 0) {
 #pragma unroll
-            for (int k = 0; k < NV; ++k) set[(size_t)a.rank * 4 + k] = red[k][0];
-            __threadfence();                 // (across GPUs: __threadfence_system)
-            atomicAdd(a.arrive, 1u);
+            for (int k = 0; k < NV; ++k) set[(size_t)a.rank * kSlotStride + k] = red[k][0];
+            __threadfence_system();          // the slot is read by other ranks (other processes / GPUs)
+            atomicAdd_system(a.arrive, 1u);
         }
         cta_barrier();
     }
@@ -1064,7 +1068,7 @@ __device__ __forceinline__ void rank_allsum(const RArgs& a, cg::grid_group& grid
 #pragma unroll
     for (int k = 0; k < NV; ++k) {
         double s = 0.0;
-        for (int q = 0; q < a.P; ++q) s += *(volatile const double*)(set + (size_t)q * 4 + k);
+        for (int q = 0; q < a.P; ++q) s += *(volatile const double*)(set + (size_t)q * kSlotStride + k);
         tot[k] = s;
     }
 }
@@ -1078,7 +1082,7 @@ __global__ void __launch_bounds__(DDA_THREADS, 3) k_rank_loop(const RArgs a) {
     const double thr = a.thr;
     double rho = a.rho0, alpha = 0.0, beta = 0.0, rr_last = 0.0;
     int k = 0, status = DDA_ERR_NO_CONVERGENCE, iters = 0, checks = 0, pend = 0;
-    unsigned epoch = 0;
+    unsigned epoch = a.epoch0;
     for (;;) {
         double* pnew = (k & 1) ? D.p1 : D.p0;
         const double* pold = k == 0 ? D.rt : ((k & 1) ? D.p0 : D.p1);
@@ -1157,7 +1161,33 @@ __global__ void __launch_bounds__(DDA_THREADS, 3) k_rank_loop(const RArgs a) {
         st->rr = rr_last;
         st->pend = pend;
         st->checks = checks;
+        st->epoch_end = epoch;
     }
+}
+
+__global__ void k_ipc_coll(const double* in, int nv, double* out, char* sync, int P, int rank, unsigned epoch) {
+    unsigned* arrive = reinterpret_cast<unsigned*>(sync);
+    int* err = reinterpret_cast<int*>(sync + 16);
+    double* set = reinterpret_cast<double*>(sync + kSyncHdr) + (size_t)(epoch % kRankSets) * P * kSlotStride;
+    for (int k = 0; k < nv; ++k) set[(size_t)rank * kSlotStride + k] = in[k];
+    __threadfence_system();
+    atomicAdd_system(arrive, 1u);
+    const unsigned target = epoch * (unsigned)P;
+    unsigned long long spins = 0;
+    while ((int)(ld_acquire(reinterpret_cast<const int*>(arrive)) - (int)target) < 0) {
+        if (++spins > (1ull << 28)) { atomicExch_system(err, 1); break; }
+        __nanosleep(64);
+    }
+    for (int k = 0; k < nv; ++k) {
+        double acc = 0.0;
+        for (int q = 0; q < P; ++q) acc += *(volatile const double*)(set + (size_t)q * kSlotStride + k);
+        out[k] = acc;
+    }
+}
+
+__global__ void k_ipc_hmap(int n, int q, const int* __restrict__ peer_idx, int2* __restrict__ out) {
+    for (int t = blockIdx.x * blockDim.x + threadIdx.x; t < n; t += gridDim.x * blockDim.x)
+        out[t] = make_int2(q, peer_idx[t]);
 }
 
 int grid_of(const void* k, int cap_per_sm) {
@@ -1195,10 +1225,38 @@ struct DistPart {
     std::vector<int> h_send_idx; // host copy of send_idx (v5 peer tables)
     const double** hsrc = nullptr;   // v5: [n_halo] device pointers to the owners' rows of p
     int G_spmv = 0, G_vec = 0, G_spmv2 = 0, G_a3 = 0;
+    bool ipc_alloc = false;      // sendbuf, rt, pA, pB, send_idx from cudaMalloc (exported through IPC handles)
+};
+
+// release a partition's device buffers (the IPC-exported ones were cudaMalloc'd)
+static void free_part(DistPart& p) {
+    void* exported[] = {p.send_idx, p.sendbuf, p.rt, p.pA, p.pB};
+    void* pooled[] = {p.x, p.q, p.r, p.z, p.part, p.scal, p.red, p.dst, (void*)p.scal_ptrs, p.ticket,
+                      (void*)p.hsrc, p.ticket2};
+    for (void* v : exported)
+        if (v) { if (p.ipc_alloc) cudaFree(v); else dda::dev_free(v); }
+    for (void* v : pooled)
+        if (v) dda::dev_free(v);
+}
+
+// IPC transport (one partition per process; peers' buffers mapped with CUDA IPC handles): what this
+// rank reads of peer q
+struct IpcPeer {
+    double* sendbuf = nullptr;   // q's packed halo rows, in q's send order
+    double *rt = nullptr, *pA = nullptr, *pB = nullptr;   // q's r~ and p ping-pong (own rows first)
+    int* send_idx = nullptr;     // q's send lists (local rows), concatenated by destination
+    std::vector<int> send_off;   // [P + 1] q's send offsets
+    std::vector<void*> opened;   // mapped handles to close
 };
 
 struct dda_comm {
     bool loopback = false;
+    bool ipc = false;            // IPC transport (dda_comm_init_ipc)
+    bool ipc_ready = false;      // peers mapped (dda_comm_ipc_import)
+    std::vector<IpcPeer> peers;  // [P] (own entry: own pointers)
+    char* sync = nullptr;        // rank 0's arrival counter + slot sets (mapped on the other ranks)
+    bool sync_owned = false;
+    unsigned epoch = 0;          // arrival epochs consumed (identical on every rank)
     int last_checks = 0;         // v4: exact stopping tests of the last solve
     double prof_ms[4] = {0, 0, 0, 0};   // v4 with DDA_DIST_PROFILE=1: halo, A, allreduce, B (summed, ms)
     int nranks = 1, rank = 0;    // NCCL: world; loopback: nranks = partitions, rank unused
@@ -1255,15 +1313,103 @@ extern "C" dda_status_t dda_comm_init_loopback(int32_t nparts, dda_comm_t* out) 
     return DDA_OK;
 }
 
+extern "C" dda_status_t dda_comm_init_ipc(int32_t nranks, int32_t rank, dda_comm_t* out) {
+    if (!out || nranks < 1 || nranks > kDPMax || rank < 0 || rank >= nranks) return DDA_ERR_ARG;
+    dda_comm* c = new dda_comm();
+    c->ipc = true;
+    c->nranks = nranks;
+    c->rank = rank;
+    c->parts.resize(1);
+    c->peers.resize(nranks);
+    *out = c;
+    return DDA_OK;
+}
+
+static constexpr uint32_t kIpcMagic = 0x44444149u;   // "DDAI"
+struct IpcBlob {   // what dda_comm_ipc_export writes: this rank's exchange plan and buffer handles
+    uint32_t magic;
+    int32_t rank, nranks, n_send, has_sync;
+    int32_t send_off[kDPMax + 1];
+    cudaIpcMemHandle_t sendbuf, rt, pA, pB, send_idx, sync;
+};
+
+extern "C" dda_status_t dda_comm_ipc_export(dda_comm_t c, void* blob, int64_t* bytes) {
+    if (!c || !c->ipc || !bytes) return DDA_ERR_ARG;
+    const int64_t need = (int64_t)sizeof(IpcBlob);
+    if (!blob) { *bytes = need; return DDA_OK; }
+    if (*bytes < need) return DDA_ERR_ARG;
+    DistPart& D = c->parts[0];
+    if (!D.K || !D.ipc_alloc) return DDA_ERR_ARG;          // attach (or build) this rank's partition first
+    IpcBlob b{};
+    b.magic = kIpcMagic;
+    b.rank = c->rank;
+    b.nranks = c->nranks;
+    b.n_send = D.n_send;
+    for (int q = 0; q <= c->nranks; ++q) b.send_off[q] = D.send_off[q];
+    if (c->rank == 0 && !c->sync) {   // rank 0 owns the arrival counter and the slot sets
+        const size_t sb = kSyncHdr + sizeof(double) * kRankSets * kSlotStride * (size_t)c->nranks;
+        DDA_CK(cudaMalloc(reinterpret_cast<void**>(&c->sync), sb));
+        DDA_CK(cudaMemset(c->sync, 0, sb));
+        c->sync_owned = true;
+    }
+    DDA_CK(cudaDeviceSynchronize());
+    DDA_CK(cudaIpcGetMemHandle(&b.sendbuf, D.sendbuf));
+    DDA_CK(cudaIpcGetMemHandle(&b.rt, D.rt));
+    DDA_CK(cudaIpcGetMemHandle(&b.pA, D.pA));
+    DDA_CK(cudaIpcGetMemHandle(&b.pB, D.pB));
+    DDA_CK(cudaIpcGetMemHandle(&b.send_idx, D.send_idx));
+    b.has_sync = c->rank == 0;
+    if (b.has_sync) DDA_CK(cudaIpcGetMemHandle(&b.sync, c->sync));
+    std::memcpy(blob, &b, sizeof b);
+    *bytes = need;
+    return DDA_OK;
+}
+
+extern "C" dda_status_t dda_comm_ipc_import(dda_comm_t c, const void* blobs, int64_t bytes) {
+    if (!c || !c->ipc || !blobs || bytes != (int64_t)sizeof(IpcBlob) || c->ipc_ready) return DDA_ERR_ARG;
+    DistPart& D = c->parts[0];
+    if (!D.K) return DDA_ERR_ARG;
+    const int P = c->nranks, me = c->rank;
+    std::vector<IpcBlob> b(P);
+    for (int q = 0; q < P; ++q) {
+        std::memcpy(&b[q], static_cast<const char*>(blobs) + (size_t)q * sizeof(IpcBlob), sizeof(IpcBlob));
+        if (b[q].magic != kIpcMagic || b[q].rank != q || b[q].nranks != P) return DDA_ERR_ARG;
+        // q's send list to this rank must match this rank's receive list from q
+        if (q != me && b[q].send_off[me + 1] - b[q].send_off[me] != D.recv_counts[q]) return DDA_ERR_ARG;
+    }
+    if (!b[0].has_sync) return DDA_ERR_ARG;
+    auto open = [&](IpcPeer& Q, const cudaIpcMemHandle_t& h, void** out) -> cudaError_t {
+        cudaError_t e = cudaIpcOpenMemHandle(out, h, cudaIpcMemLazyEnablePeerAccess);
+        if (e == cudaSuccess) Q.opened.push_back(*out);
+        return e;
+    };
+    for (int q = 0; q < P; ++q) {
+        IpcPeer& Q = c->peers[q];
+        Q.send_off.assign(b[q].send_off, b[q].send_off + P + 1);
+        if (q == me) {
+            Q.sendbuf = D.sendbuf; Q.rt = D.rt; Q.pA = D.pA; Q.pB = D.pB; Q.send_idx = D.send_idx;
+            continue;
+        }
+        DDA_CK(open(Q, b[q].sendbuf, reinterpret_cast<void**>(&Q.sendbuf)));
+        DDA_CK(open(Q, b[q].rt, reinterpret_cast<void**>(&Q.rt)));
+        DDA_CK(open(Q, b[q].pA, reinterpret_cast<void**>(&Q.pA)));
+        DDA_CK(open(Q, b[q].pB, reinterpret_cast<void**>(&Q.pB)));
+        DDA_CK(open(Q, b[q].send_idx, reinterpret_cast<void**>(&Q.send_idx)));
+    }
+    if (me != 0) DDA_CK(cudaIpcOpenMemHandle(reinterpret_cast<void**>(&c->sync), b[0].sync, cudaIpcMemLazyEnablePeerAccess));
+    c->epoch = 0;
+    c->ipc_ready = true;
+    return DDA_OK;
+}
+
 extern "C" void dda_comm_free(dda_comm_t c) {
     if (!c) return;
     cudaDeviceSynchronize();
-    for (DistPart& p : c->parts) {
-        void* ptrs[] = {p.send_idx, p.sendbuf, p.x, p.q, p.r, p.z, p.part, p.scal, p.red, p.dst,
-                        (void*)p.scal_ptrs, p.rt, p.pA, p.pB, p.ticket, (void*)p.hsrc, p.ticket2};
-        for (void* v : ptrs)
-            if (v) dev_free(v);
-    }
+    for (IpcPeer& q : c->peers)
+        for (void* v : q.opened) cudaIpcCloseMemHandle(v);
+    if (c->sync && !c->sync_owned) cudaIpcCloseMemHandle(c->sync);
+    for (DistPart& p : c->parts) free_part(p);
+    if (c->sync && c->sync_owned) cudaFree(c->sync);
     if (c->nccl) ncclCommDestroy(c->nccl);
     delete c;
 }
@@ -1299,11 +1445,9 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     DistPart& D = c->parts[slot];
     if (D.K) {                                   // re-attach (e.g. a rebuilt matrix): release the old buffers
+        if (c->ipc_ready) return DDA_ERR_ARG;    // peers have mapped the exported ones
         cudaStreamSynchronize(st);
-        void* ptrs[] = {D.send_idx, D.sendbuf, D.x, D.q, D.r, D.z, D.part, D.scal, D.red, D.dst,
-                        (void*)D.scal_ptrs, D.rt, D.pA, D.pB, D.ticket, (void*)D.hsrc, D.ticket2};
-        for (void* v : ptrs)
-            if (v) dev_free(v);
+        free_part(D);
         D = DistPart();
     }
     for (int q = 0; q < P; ++q)
@@ -1347,8 +1491,14 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     int Gm = D.G_spmv > D.G_vec ? D.G_spmv : D.G_vec;
     if (D.G_spmv2 > Gm) Gm = D.G_spmv2;
     if (D.G_a3 > Gm) Gm = D.G_a3;
-    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.send_idx), (D.n_send + 1) * sizeof(int), st));
-    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.sendbuf), (24 * (size_t)D.n_send + 1) * sizeof(double), st));
+    // the buffers peers read in place under the IPC transport come from cudaMalloc (an IPC handle maps a
+    // whole allocation); everything else from the stream-ordered pool
+    D.ipc_alloc = c->ipc;
+    auto xalloc = [&](void** ptr, size_t bytes) -> cudaError_t {
+        return c->ipc ? cudaMalloc(ptr, bytes) : dev_alloc(ptr, bytes, st);
+    };
+    DDA_CK(xalloc(reinterpret_cast<void**>(&D.send_idx), (D.n_send + 1) * sizeof(int)));
+    DDA_CK(xalloc(reinterpret_cast<void**>(&D.sendbuf), (24 * (size_t)D.n_send + 1) * sizeof(double)));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.x), nl6 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.q), no6 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.r), no6 * sizeof(double), st));
@@ -1386,9 +1536,9 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
         if (sizeof(S4) > ds) ds = sizeof(S4);
         DDA_CK(dev_alloc(&D.dst, ds, st));
     }
-    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.rt), nl6 * sizeof(double), st));
-    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.pA), nl6 * sizeof(double), st));
-    DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.pB), nl6 * sizeof(double), st));
+    DDA_CK(xalloc(reinterpret_cast<void**>(&D.rt), nl6 * sizeof(double)));
+    DDA_CK(xalloc(reinterpret_cast<void**>(&D.pA), nl6 * sizeof(double)));
+    DDA_CK(xalloc(reinterpret_cast<void**>(&D.pB), nl6 * sizeof(double)));
     DDA_CK(cudaMemsetAsync(D.rt, 0, nl6 * sizeof(double), st));
     DDA_CK(cudaMemsetAsync(D.pA, 0, nl6 * sizeof(double), st));
     DDA_CK(cudaMemsetAsync(D.pB, 0, nl6 * sizeof(double), st));
@@ -1396,7 +1546,7 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     if (D.n_send)
         DDA_CK(cudaMemcpyAsync(D.send_idx, send_idx, D.n_send * sizeof(int), cudaMemcpyHostToDevice, st));
     DDA_CK(cudaMemsetAsync(D.x, 0, nl6 * sizeof(double), st));
-    if (!c->loopback && P > 1) {   // the peers' send counts must equal this rank's receive counts
+    if (!c->loopback && !c->ipc && P > 1) {   // the peers' send counts must equal this rank's receive counts
         int* cnt = nullptr;
         DDA_CK(dev_alloc(reinterpret_cast<void**>(&cnt), (size_t)P * (P + 1) * sizeof(int), st));
         DDA_CK(cudaMemcpyAsync(cnt, send_counts, P * sizeof(int), cudaMemcpyHostToDevice, st));
@@ -1427,6 +1577,22 @@ double* part_buf(DistPart& D, int which) {
 }
 
 // fill rows n_own.. of buffer `which` (w doubles per row) of every local partition from the peers' own rows
+// IPC transport collective (one thread): publish nv values to this rank's slot of the epoch's set,
+// announce the arrival on rank 0's counter, wait for all P ranks (bounded), sum the P slots in rank
+// order into out (nv = 0: a barrier).  epoch is the 1-based arrival epoch this call completes.
+#define DDA_TRY_S(expr)                    \
+    do {                                   \
+        dda_status_t _s = (expr);          \
+        if (_s != DDA_OK) return _s;       \
+    } while (0)
+dda_status_t ipc_coll(dda_comm* c, const double* in, int nv, double* out, cudaStream_t st) {
+    if (nv > kSlotStride) return DDA_ERR_ARG;
+    c->epoch += 1;
+    k_ipc_coll<<<1, 1, 0, st>>>(in, nv, out, c->sync, c->nranks, c->rank, c->epoch);
+    DDA_LAUNCHED();
+    return DDA_OK;
+}
+
 dda_status_t halo_exchange_w(dda_comm* c, cudaStream_t st, int which, int w) {
     const int P = c->nranks;
     for (DistPart& D : c->parts) {
@@ -1436,6 +1602,20 @@ dda_status_t halo_exchange_w(dda_comm* c, cudaStream_t st, int which, int w) {
                 D.n_send, w, D.send_idx, part_buf(D, which), D.sendbuf);
             DDA_LAUNCHED();
         }
+    }
+    if (c->ipc) {   // packed by every rank -> each copies its halo from the peers' send buffers -> released
+        if (!c->ipc_ready) return DDA_ERR_ARG;
+        DistPart& D = c->parts[0];
+        DDA_TRY_S(ipc_coll(c, nullptr, 0, nullptr, st));
+        for (int q = 0; q < P; ++q) {
+            if (q == c->rank || !D.recv_counts[q]) continue;
+            const IpcPeer& Q = c->peers[q];
+            DDA_CK(cudaMemcpyAsync(part_buf(D, which) + (size_t)w * ((size_t)D.n_own + D.recv_off[q]),
+                                   Q.sendbuf + (size_t)w * Q.send_off[c->rank],
+                                   (size_t)w * sizeof(double) * D.recv_counts[q], cudaMemcpyDeviceToDevice, st));
+        }
+        DDA_TRY_S(ipc_coll(c, nullptr, 0, nullptr, st));
+        return DDA_OK;
     }
     if (c->loopback) {
         for (int p = 0; p < P; ++p)
@@ -1483,7 +1663,8 @@ dda_status_t allreduce_host(dda_comm* c, int nv, double* out, cudaStream_t st) {
         return DDA_OK;
     }
     DistPart& D = c->parts[0];
-    if (c->nranks > 1) DDA_NCCL(ncclAllReduce(D.scal, D.scal, nv, ncclDouble, ncclSum, c->nccl, st));
+    if (c->ipc) DDA_TRY_S(ipc_coll(c, D.scal, nv, D.scal, st));
+    else if (c->nranks > 1) DDA_NCCL(ncclAllReduce(D.scal, D.scal, nv, ncclDouble, ncclSum, c->nccl, st));
     DDA_CK(cudaMemcpyAsync(out, D.scal, nv * sizeof(double), cudaMemcpyDeviceToHost, st));
     DDA_CK(cudaStreamSynchronize(st));
     return DDA_OK;
@@ -1504,7 +1685,8 @@ dda_status_t allreduce_host_at(dda_comm* c, int off, int nv, double* out, cudaSt
         return DDA_OK;
     }
     DistPart& D = c->parts[0];
-    if (c->nranks > 1) DDA_NCCL(ncclAllReduce(D.scal + off, D.red, nv, ncclDouble, ncclSum, c->nccl, st));
+    if (c->ipc) DDA_TRY_S(ipc_coll(c, D.scal + off, nv, D.red, st));
+    else if (c->nranks > 1) DDA_NCCL(ncclAllReduce(D.scal + off, D.red, nv, ncclDouble, ncclSum, c->nccl, st));
     else DDA_CK(cudaMemcpyAsync(D.red, D.scal + off, nv * sizeof(double), cudaMemcpyDeviceToDevice, st));
     DDA_CK(cudaMemcpyAsync(out, D.red, nv * sizeof(double), cudaMemcpyDeviceToHost, st));
     DDA_CK(cudaStreamSynchronize(st));
@@ -1521,6 +1703,7 @@ dda_status_t allreduce_dev(dda_comm* c, int nv, cudaStream_t st) {
         return DDA_OK;
     }
     DistPart& D = c->parts[0];
+    if (c->ipc) return ipc_coll(c, D.scal, nv, D.red, st);
     if (c->nranks > 1) DDA_NCCL(ncclAllReduce(D.scal, D.red, nv, ncclDouble, ncclSum, c->nccl, st));
     else DDA_CK(cudaMemcpyAsync(D.red, D.scal, nv * sizeof(double), cudaMemcpyDeviceToDevice, st));
     return DDA_OK;
@@ -2004,7 +2187,7 @@ dda_status_t dist_v6_solve(dda_comm* c, const double* const* F, const double* co
         // v7: one cooperative kernel per rank, each on its own stream, all resident together (the grid is
         // split evenly); the ranks meet only through the slot sets and the arrival counter
         const int Gr = G / P;
-        const size_t pb_r = sizeof(double) * 4 * (size_t)Gr, sb = sizeof(double) * kRankSets * 4 * (size_t)P;
+        const size_t pb_r = sizeof(double) * 4 * (size_t)Gr, sb = sizeof(double) * kRankSets * kSlotStride * (size_t)P;
         char* rw = nullptr;
         DDA_CK(dev_alloc(reinterpret_cast<void**>(&rw), P * (pb_r + sizeof(DPState) + 64) + sb + 64, st));
         struct RwFree { char* b; cudaStream_t s; ~RwFree() { cudaStreamSynchronize(s); dev_free_on(b, s); } } rf{rw, st};
@@ -2028,7 +2211,7 @@ dda_status_t dist_v6_solve(dda_comm* c, const double* const* F, const double* co
             char* mine = base + (size_t)p * (pb_r + sizeof(DPState) + 64);
             DPState* rst = reinterpret_cast<DPState*>(mine + pb_r);
             DDA_CK(cudaMemsetAsync(rst, 0, sizeof(DPState), rs[p]));
-            ra[p] = RArgs{dparts, P, p, reinterpret_cast<double*>(mine), slots, arrive, rst, err, rho, tol * bnorm, maxit};
+            ra[p] = RArgs{dparts, P, p, reinterpret_cast<double*>(mine), slots, arrive, 0u, rst, err, rho, tol * bnorm, maxit};
         }
         for (int p = 0; p < P; ++p) {       // all ranks are launched before any is waited on
             void* args[] = {&ra[p]};
@@ -2073,6 +2256,112 @@ dda_status_t dist_v6_solve(dda_comm* c, const double* const* F, const double* co
     return DDA_OK;
 }
 
+// ---- IPC transport solve: this process's rank of the v7 loop (one persistent kernel per rank); the
+// peers' r~ / p rows are read through their IPC-mapped arrays, every reduction through rank 0's
+// mapped counter and slot sets
+dda_status_t dist_ipc_solve(dda_comm* c, const double* const* F, const double* const* d0, double* const* d,
+                            double tol, int32_t maxit, dda_status_t* status, int* it, bool* zero, double* bnorm_out,
+                            int* checks_out, cudaStream_t st) {
+    *zero = false;
+    *it = 0;
+    const int P = c->nranks, me = c->rank;
+    DistPart& D = c->parts[0];
+    if (!c->ipc_ready || !D.K || P > kDPMax) return DDA_ERR_ARG;
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_rank_loop, DDA_THREADS, 0);
+    if (per_sm > 3) per_sm = 3;
+    if (per_sm < 1) return DDA_ERR_CUDA;
+    const int G = device_sms() * per_sm;
+    DDA_TRY_S(halo_exchange_w(c, st, 4, kDinv));           // S_j of the halo rows
+    D.K->scaled_valid = false;
+    DDA_TRY_S(scaled_setup(D.K, st));
+    const bool have_d0 = d0 != nullptr && d0[0] != nullptr;
+    if (have_d0) {
+        DDA_CK(cudaMemcpyAsync(D.x, d0[0], 6 * sizeof(double) * D.n_own, cudaMemcpyDeviceToDevice, st));
+        DDA_TRY_S(halo_exchange(c, st));
+        DDA_TRY_S(spmv_parts(c, false, st));
+    }
+    k_v4_init<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, F[0], have_d0 ? D.q : nullptr, have_d0 ? d0[0] : nullptr,
+                                               d[0], D.K->sfac, D.K->lfac, D.K->bj_w, D.rt, D.pA, D.part, D.ticket,
+                                               D.scal);
+    DDA_LAUNCHED();
+    double s4[4];
+    DDA_TRY_S(allreduce_host_at(c, 8, 4, s4, st));
+    const double rho = s4[0], rr = s4[2], FF = s4[3], bnorm = std::sqrt(FF);
+    *bnorm_out = bnorm;
+    *checks_out = 0;
+    if (FF == 0.0) {                                        // reading Z2
+        DDA_CK(cudaMemsetAsync(d[0], 0, 6 * sizeof(double) * D.n_own, st));
+        DDA_CK(cudaStreamSynchronize(st));
+        *zero = true;
+        *status = DDA_OK;
+        return DDA_OK;
+    }
+    int pre = -1;
+    if (std::sqrt(rr) <= tol * bnorm) pre = DDA_OK;
+    else if (!(rho > 0.0) || !std::isfinite(rho)) pre = DDA_ERR_BREAKDOWN;
+    else if (maxit <= 0) pre = DDA_ERR_NO_CONVERGENCE;
+    // the rank table: own entry complete; a peer's entry carries its mapped r~ / p arrays
+    std::vector<DPart> h(P);
+    for (int q = 0; q < P; ++q) {
+        h[q] = DPart{};
+        h[q].rt = c->peers[q].rt;
+        h[q].p0 = c->peers[q].pA;
+        h[q].p1 = c->peers[q].pB;
+    }
+    const int nh = D.n_local - D.n_own;
+    const size_t tb = sizeof(DPart) * P, hb = sizeof(int2) * (nh + 1), pb = sizeof(double) * 4 * (size_t)G;
+    char* ws = nullptr;
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&ws), tb + hb + pb + 2 * sizeof(DPState) + 256, st));
+    struct WsFree { char* b; cudaStream_t s; ~WsFree() { cudaStreamSynchronize(s); dev_free_on(b, s); } } wf{ws, st};
+    DPart* dparts = reinterpret_cast<DPart*>(ws);
+    int2* dh = reinterpret_cast<int2*>(ws + ((tb + 15) / 16) * 16);
+    double* dpart = reinterpret_cast<double*>(ws + ((tb + 15) / 16) * 16 + ((hb + 15) / 16) * 16);
+    DPState* dst = reinterpret_cast<DPState*>(dpart + 4 * (size_t)G);
+    for (int q = 0; q < P; ++q) {       // halo rows from q -> (q, q's local row) read from q's send list
+        if (q == me || !D.recv_counts[q]) continue;
+        const IpcPeer& Q = c->peers[q];
+        k_ipc_hmap<<<(D.recv_counts[q] + 255) / 256, 256, 0, st>>>(D.recv_counts[q], q, Q.send_idx + Q.send_off[me],
+                                                                     dh + D.recv_off[q]);
+        DDA_LAUNCHED();
+    }
+    h[me].A = own_view_sc(D);
+    h[me].rt = D.rt; h[me].p0 = D.pA; h[me].p1 = D.pB; h[me].q = D.q; h[me].x = d[0];
+    h[me].w = D.K->bj_w; h[me].lfac = D.K->lfac; h[me].hmap = dh;
+    h[me].n_own = D.n_own; h[me].c0 = 0; h[me].c1 = G;
+    DDA_CK(cudaMemcpyAsync(dparts, h.data(), tb, cudaMemcpyHostToDevice, st));
+    DDA_CK(cudaMemsetAsync(dst, 0, sizeof(DPState), st));
+    int* err = reinterpret_cast<int*>(c->sync + 16);
+    if (pre < 0) {
+        RArgs ra{dparts, P, me, dpart, reinterpret_cast<double*>(c->sync + kSyncHdr),
+                 reinterpret_cast<unsigned*>(c->sync), c->epoch, dst, err, rho, tol * bnorm, maxit};
+        void* args[] = {&ra};
+        DDA_CK(cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_rank_loop), dim3(G), dim3(DDA_THREADS),
+                                           args, 0, st));
+        note_launch();
+    } else {
+        DPState z{};
+        z.status = pre;
+        z.rr = rr;
+        z.epoch_end = c->epoch;
+        DDA_CK(cudaMemcpyAsync(dst, &z, sizeof z, cudaMemcpyHostToDevice, st));
+    }
+    DPState out{};
+    int herr = 0;
+    DDA_CK(cudaMemcpyAsync(&out, dst, sizeof out, cudaMemcpyDeviceToHost, st));
+    DDA_CK(cudaMemcpyAsync(&herr, err, sizeof(int), cudaMemcpyDeviceToHost, st));
+    DDA_CK(cudaStreamSynchronize(st));
+    if (herr) return DDA_ERR_CUDA;                        // a wait on the other ranks hit its bound
+    c->epoch = out.epoch_end;
+    k_dp_final<<<D.G_vec, DDA_THREADS, 0, st>>>(D.n_own, d[0], ((out.k - 1) & 1) ? D.pB : D.pA, dst, D.K->sfac);
+    DDA_LAUNCHED();
+    DDA_CK(cudaStreamSynchronize(st));
+    *status = (dda_status_t)out.status;
+    *it = out.iters;
+    *checks_out = out.checks;
+    return DDA_OK;
+}
+
 }  // namespace
 
 extern "C" dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double* const* F, const double* const* d0,
@@ -2102,7 +2391,10 @@ extern "C" dda_status_t dda_pcg_solve_dist(dda_comm_t c, const double* const* F,
         // v6 (loopback default): one persistent kernel for every partition; DDA_DIST_VERSION=5 / 4 / 3
         // select the per-iteration launches (v5: peer-load halo, v4: halo copies, v3)
         bool ran = false;
-        if (c->loopback && !(dve && (dve[0] == '3' || dve[0] == '4' || dve[0] == '5')))
+        if (c->ipc && !(dve && (dve[0] == '3' || dve[0] == '4'))) {   // the IPC transport: v7, this process's rank
+            DDA_TRY(dist_ipc_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, &checks, st));
+            ran = true;
+        } else if (c->loopback && !(dve && (dve[0] == '3' || dve[0] == '4' || dve[0] == '5')))
             DDA_TRY(dist_v6_solve(c, F, d0, d, tol, maxit, &status, &it, &zero, &bnorm, &checks, &ran, st,
                                   dve && dve[0] == '7'));
         if (ran) {
