@@ -322,6 +322,9 @@ def main():
     ap.add_argument("--cpu-iter-sample", type=int, default=8, help="oracle PCG iterations timed (cpu_baseline)")
     ap.add_argument("--ref-iter-sample", type=int, default=4, help="oracle PCG iterations timed per reference step")
     ap.add_argument("--clock-period", type=float, default=0.05, help="NVML clock sampling period (s)")
+    ap.add_argument("--dist-transport", default="ipc", choices=["ipc", "nccl"],
+                    help="N > 1: peers' buffers mapped with CUDA IPC handles, one persistent kernel per rank (v7; "
+                         "falls back to nccl if the mapping fails) or NCCL halo + allreduce per iteration (v4)")
     ap.add_argument("--force-dist", action="store_true",
                     help="run the partitioned (NCCL) path even at N = 1 (a check of the N > 1 code path)")
     args = ap.parse_args()
@@ -543,9 +546,30 @@ def run_dist(args, P, world, rank, local):
     t = {k: dev(getattr(P, k)) for k in ("bi", "bj", "pen", "e", "g")}
     t["kdiag"] = dev(P.kdiag[r0:r1])
     t["F"] = dev(P.F[6 * r0:6 * r1])
-    obj = [dda.Comm.unique_id() if rank == 0 else None]
-    dist.broadcast_object_list(obj, src=0)
-    comm = dda.Comm.nccl(world, rank, obj[0])
+    transport = args.dist_transport
+    comm = None
+    if transport == "ipc":
+        # v7 over CUDA IPC: build this rank's partition, exchange the handle blobs over the process group,
+        # map the peers (every later rebuild re-attaches into the mapped buffers)
+        try:
+            comm = dda.Comm.ipc(world, rank)
+            comm.build_matrix_dist(0, P.n, bounds, t["kdiag"], t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+            blobs = [None] * world
+            dist.all_gather_object(blobs, comm.ipc_export())
+            comm.ipc_import(blobs)
+            ok = torch.tensor([1], device="cuda")
+        except Exception as exc:   # noqa: BLE001 -- every rank must agree on the fallback
+            print(f"ipc transport unavailable ({exc}); falling back to nccl", file=sys.stderr)
+            ok = torch.tensor([0], device="cuda")
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+        if int(ok.item()) == 0:
+            if comm is not None:
+                comm.free()
+            comm, transport = None, "nccl"
+    if comm is None:
+        obj = [dda.Comm.unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        comm = dda.Comm.nccl(world, rank, obj[0])
     stream = torch.cuda.current_stream()
     hbm_peak, peak_src = measured_peaks()
 
@@ -579,11 +603,11 @@ def run_dist(args, P, world, rank, local):
     pcg = statistics.mean(e[1].elapsed_time(e[2]) for e in evs)
     K, iters, rel_res, status = res[-1]
     assert status == dda.OK and rel_res <= 1.01e-10, (status, rel_res)
-    # v4 (block-Jacobi): the scaled engine per rank, 300u + 496 algorithmic bytes per own row and
-    # iteration (phase A 300u + 152, phase B 344); u over the rank's own rows
+    # algorithmic bytes per own row and iteration: v4 (NCCL) 300u + 496 (phase A 300u + 152,
+    # phase B 344); v7 (IPC) the single-GPU scaled engine's 300u + 448; u over the rank's own rows
     info = comm.info(0, nparts=world)
     u = K.nnzb / max(n_own, 1)
-    local_bytes = n_own * (300.0 * u + 496.0) * iters
+    local_bytes = n_own * (300.0 * u + (448.0 if transport == "ipc" else 496.0)) * iters
     ach = local_bytes / (pcg * 1e-3) / 1e9
     tt = torch.tensor([ms, pcg, asm], device="cuda")
     dist.all_reduce(tt, op=dist.ReduceOp.MAX)
@@ -591,18 +615,22 @@ def run_dist(args, P, world, rank, local):
     # comm / compute split: one extra (untimed) solve with CUDA events between the steps of every
     # iteration (halo exchange, phase A, allreduce, phase B; DDA_DIST_PROFILE=1), max over ranks
     import ctypes as _C
-    os.environ["DDA_DIST_PROFILE"] = "1"
-    comm.pcg_solve([t["F"]], tol=1e-10, maxit=10000, precond=args.precond)
-    os.environ.pop("DDA_DIST_PROFILE")
-    prof = (_C.c_double * 4)()
-    fprof = dda.lib().dda__dist_profile
-    fprof.argtypes = [_C.c_void_p, _C.c_void_p]
-    fprof(comm._h, prof)
-    tp = torch.tensor(list(prof), device="cuda")
-    dist.all_reduce(tp, op=dist.ReduceOp.MAX)
-    split = {"halo_ms": float(tp[0]), "phaseA_ms": float(tp[1]), "allreduce_ms": float(tp[2]),
-             "phaseB_ms": float(tp[3]), "note": "per solve, summed over iterations, max over ranks; one profiled "
-                                                "(event-instrumented, untimed) solve"}
+    if transport == "nccl":
+        os.environ["DDA_DIST_PROFILE"] = "1"
+        comm.pcg_solve([t["F"]], tol=1e-10, maxit=10000, precond=args.precond)
+        os.environ.pop("DDA_DIST_PROFILE")
+        prof = (_C.c_double * 4)()
+        fprof = dda.lib().dda__dist_profile
+        fprof.argtypes = [_C.c_void_p, _C.c_void_p]
+        fprof(comm._h, prof)
+        tp = torch.tensor(list(prof), device="cuda")
+        dist.all_reduce(tp, op=dist.ReduceOp.MAX)
+        split = {"halo_ms": float(tp[0]), "phaseA_ms": float(tp[1]), "allreduce_ms": float(tp[2]),
+                 "phaseB_ms": float(tp[3]), "note": "per solve, summed over iterations, max over ranks; one "
+                                                    "profiled (event-instrumented, untimed) solve"}
+    else:
+        split = {"note": "v7 over CUDA IPC: one persistent kernel per rank, halo reads and the one-shot allreduce "
+                         "inside it; no per-phase host events"}
     # e2e: pinned host local inputs -> device, assemble, solve, d -> host (max over ranks)
     e2e = None
     if not args.no_e2e:
@@ -634,7 +662,11 @@ def run_dist(args, P, world, rank, local):
             "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": workload_name(args.blocks), "n_blocks": P.n, "dof": 6 * P.n, "springs": P.m,
                        "precond": args.precond, "tol": 1e-10, "start": "cold (d0 = 0)",
-                       "parallelism": f"block-row partition over {world} ranks (NCCL halo + allreduce)",
+                       "parallelism": (f"block-row partition over {world} ranks, one persistent kernel per rank, "
+                                       "peers' buffers mapped with CUDA IPC (halo reads and one-shot allreduce "
+                                       "over NVLink)" if transport == "ipc" else
+                                       f"block-row partition over {world} ranks (NCCL halo + allreduce)"),
+                       "transport": transport,
                        "rank0_rows": n_own, "rank0_halo": info["n_halo"],
                        "step": "dda_build_matrix_dist (select + renumber + assemble + plan, device) + "
                                "dda_pcg_solve_dist",

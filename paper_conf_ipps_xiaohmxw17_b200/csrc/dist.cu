@@ -1444,9 +1444,21 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     if (slot < 0 || slot >= (int)c->parts.size() || n_own < 1 || n_own > K->n) return DDA_ERR_ARG;
     cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
     DistPart& D = c->parts[slot];
-    if (D.K) {                                   // re-attach (e.g. a rebuilt matrix): release the old buffers
-        if (c->ipc_ready) return DDA_ERR_ARG;    // peers have mapped the exported ones
+    // re-attach (e.g. the matrix rebuilt for the next step): release the old buffers.  Under a mapped IPC
+    // transport the exported ones stay (peers hold their handles): the new partition must have the same
+    // sizes and exchange plan
+    double *keep_sendbuf = nullptr, *keep_rt = nullptr, *keep_pA = nullptr, *keep_pB = nullptr;
+    int* keep_send_idx = nullptr;
+    if (D.K) {
         cudaStreamSynchronize(st);
+        if (c->ipc_ready) {
+            if (n_own != D.n_own || K->n != D.n_local) return DDA_ERR_ARG;
+            for (int q = 0; q < P; ++q)
+                if (send_counts[q] != D.send_counts[q] || recv_counts[q] != D.recv_counts[q]) return DDA_ERR_ARG;
+            keep_sendbuf = D.sendbuf; keep_rt = D.rt; keep_pA = D.pA; keep_pB = D.pB; keep_send_idx = D.send_idx;
+            D.sendbuf = D.rt = D.pA = D.pB = nullptr;
+            D.send_idx = nullptr;
+        }
         free_part(D);
         D = DistPart();
     }
@@ -1497,8 +1509,11 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
     auto xalloc = [&](void** ptr, size_t bytes) -> cudaError_t {
         return c->ipc ? cudaMalloc(ptr, bytes) : dev_alloc(ptr, bytes, st);
     };
-    DDA_CK(xalloc(reinterpret_cast<void**>(&D.send_idx), (D.n_send + 1) * sizeof(int)));
-    DDA_CK(xalloc(reinterpret_cast<void**>(&D.sendbuf), (24 * (size_t)D.n_send + 1) * sizeof(double)));
+    if (keep_send_idx) { D.send_idx = keep_send_idx; D.sendbuf = keep_sendbuf; }
+    else {
+        DDA_CK(xalloc(reinterpret_cast<void**>(&D.send_idx), (D.n_send + 1) * sizeof(int)));
+        DDA_CK(xalloc(reinterpret_cast<void**>(&D.sendbuf), (24 * (size_t)D.n_send + 1) * sizeof(double)));
+    }
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.x), nl6 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.q), no6 * sizeof(double), st));
     DDA_CK(dev_alloc(reinterpret_cast<void**>(&D.r), no6 * sizeof(double), st));
@@ -1536,9 +1551,12 @@ extern "C" dda_status_t dda_dist_attach(dda_comm_t c, int32_t part, dda_matrix_t
         if (sizeof(S4) > ds) ds = sizeof(S4);
         DDA_CK(dev_alloc(&D.dst, ds, st));
     }
-    DDA_CK(xalloc(reinterpret_cast<void**>(&D.rt), nl6 * sizeof(double)));
-    DDA_CK(xalloc(reinterpret_cast<void**>(&D.pA), nl6 * sizeof(double)));
-    DDA_CK(xalloc(reinterpret_cast<void**>(&D.pB), nl6 * sizeof(double)));
+    if (keep_rt) { D.rt = keep_rt; D.pA = keep_pA; D.pB = keep_pB; }
+    else {
+        DDA_CK(xalloc(reinterpret_cast<void**>(&D.rt), nl6 * sizeof(double)));
+        DDA_CK(xalloc(reinterpret_cast<void**>(&D.pA), nl6 * sizeof(double)));
+        DDA_CK(xalloc(reinterpret_cast<void**>(&D.pB), nl6 * sizeof(double)));
+    }
     DDA_CK(cudaMemsetAsync(D.rt, 0, nl6 * sizeof(double), st));
     DDA_CK(cudaMemsetAsync(D.pA, 0, nl6 * sizeof(double), st));
     DDA_CK(cudaMemsetAsync(D.pB, 0, nl6 * sizeof(double), st));

@@ -6,7 +6,8 @@ exchanged over a gloo process group (the caller's channel), and the block-Jacobi
 persistent cooperative kernel per process, halo rows read in place from the peers' mapped arrays,
 every reduction a fixed-order one-shot sum through rank 0's mapped slot sets.  The processes'
 kernels share the GPU by time slicing, so this checks the protocol, not the speed.  Rank 0 gathers
-the solution; the test compares it with the oracle (reading Z17) and with the loopback solve.
+the solution; the test compares it with the oracle (reading Z17).  A warm start and a rebuilt partition
+(the next step's matrix, re-attached into the mapped buffers) are checked too.
 """
 import json
 import os
@@ -50,6 +51,10 @@ d = ds[0].cpu().numpy()
 # warm start from the solution (every rank's own rows): at most one iteration
 ds2, it2, rr2, st2 = comm.pcg_solve([F], d0s=[ds[0].clone()], tol=1e-10, precond="bj")
 out["warm"] = (it2, rr2, st2)
+# the next step's rebuilt partition re-attaches into the mapped buffers (same plan): same solve
+K = comm.build_matrix_dist(0, P.n, b, t["kdiag"][r0:r1].contiguous(), t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+ds3, it3, rr3, st3 = comm.pcg_solve([F], tol=1e-10, precond="bj")
+out["rebuilt_same"] = bool(it3 == it and torch.equal(ds3[0], ds[0]))
 parts = [None] * world
 dist.all_gather_object(parts, d.tolist())
 if rank == 0:
@@ -91,6 +96,7 @@ def test_ipc_processes_pcg(case_name, world, tmp_path):
     it, rr, st = res["cold"]
     assert st == 0 and rr <= 1.01e-10, res["cold"]
     assert res["warm"][2] == 0 and res["warm"][0] <= 1, res["warm"]
+    assert res["rebuilt_same"]
     P = make_slope(preset(case_name))
     O = oracle.assemble(P)
     do, ito, rro, sto = O.pcg(P.F, tol=1e-10, precond="bj")
