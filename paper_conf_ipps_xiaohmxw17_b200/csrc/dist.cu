@@ -988,6 +988,12 @@ __global__ void __launch_bounds__(DDA_THREADS) k_dp_final(int n, double* d, cons
 // reads.  Across GPUs the same code needs the partition table and the slot / counter words mapped over
 // NVLink (IPC handles) and system-scope fences; here they are one device's memory.  Every wait is
 // bounded (an error flag instead of a hang).
+// one arrival on the (possibly peer-mapped) counter with release semantics at system scope: cumulative
+// over this thread's earlier writes and everything ordered before them (the CTA barrier, the grid
+// barrier), cheaper than a full system fence followed by an atomic
+__device__ __forceinline__ void arrive_release_sys(unsigned* p) {
+    asm volatile("red.release.sys.global.add.u32 [%0], 1;" :: "l"(p) : "memory");
+}
 __device__ __forceinline__ int ld_acquire(const int* p) {   // system scope: the counter may be a peer's
     int v;
     asm volatile("ld.acquire.sys.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -1051,8 +1057,7 @@ __device__ __forceinline__ void rank_allsum(const RArgs& a, cg::grid_group& grid
         if (threadIdx.x == 0) {
 #pragma unroll
             for (int k = 0; k < NV; ++k) set[(size_t)a.rank * kSlotStride + k] = red[k][0];
-            __threadfence_system();          // the slot is read by other ranks (other processes / GPUs)
-            atomicAdd_system(a.arrive, 1u);
+            arrive_release_sys(a.arrive);    // the slot (and the rank's phase writes) before the arrival
         }
         cta_barrier();
     }
@@ -1170,8 +1175,7 @@ __global__ void k_ipc_coll(const double* in, int nv, double* out, char* sync, in
     int* err = reinterpret_cast<int*>(sync + 16);
     double* set = reinterpret_cast<double*>(sync + kSyncHdr) + (size_t)(epoch % kRankSets) * P * kSlotStride;
     for (int k = 0; k < nv; ++k) set[(size_t)rank * kSlotStride + k] = in[k];
-    __threadfence_system();
-    atomicAdd_system(arrive, 1u);
+    arrive_release_sys(arrive);
     const unsigned target = epoch * (unsigned)P;
     unsigned long long spins = 0;
     while ((int)(ld_acquire(reinterpret_cast<const int*>(arrive)) - (int)target) < 0) {
