@@ -581,6 +581,19 @@ def run_dist(args, P, world, rank, local):
         if ev: ev[2].record(stream)
         return K, it, rr, st
 
+    if transport == "ipc":   # a failed IPC solve (e.g. a bounded wait expired) falls back to NCCL on every rank
+        try:
+            _, _, _, st0 = step()
+            ok = torch.tensor([1 if st0 == dda.OK else 0], device="cuda")
+        except Exception as exc:   # noqa: BLE001
+            print(f"ipc solve failed ({exc}); falling back to nccl", file=sys.stderr)
+            ok = torch.tensor([0], device="cuda")
+        dist.all_reduce(ok, op=dist.ReduceOp.MIN)
+        if int(ok.item()) == 0:
+            comm.free()
+            obj = [dda.Comm.unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(obj, src=0)
+            comm, transport = dda.Comm.nccl(world, rank, obj[0]), "nccl"
     for _ in range(args.warmup):
         step()
     torch.cuda.synchronize()
