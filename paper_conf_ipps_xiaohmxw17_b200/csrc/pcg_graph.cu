@@ -1074,9 +1074,9 @@ struct XCg1 {   // r_{k+1} = r_k - alpha (s_k + beta q_{k-1}) (first pass: q_0 =
     __device__ __forceinline__ double2 operator()(int vec, int pair) const { return raw(vec, pair); }
 };
 
-template <int MINB>
-__global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_cg1(const GArgs a) {
-    cg::grid_group grid = cg::this_grid();
+template <int TPB, class Sync>
+__device__ __forceinline__ void sp_cg1_body(const GArgs& a, Sync& sync) {
+    constexpr int WPBT = TPB / 32;
     State* st = a.st;
     if (st->done) return;
     double rho = st->rho, alpha = 0.0, beta = 0.0, rr_last = st->rr;
@@ -1085,7 +1085,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_cg1(const GArgs a) {
     BsrView A = a.A;
     A.upper = a.su;
     const int lane = threadIdx.x & 31;
-    const int w0 = blockIdx.x * WPB + (threadIdx.x >> 5), W = gridDim.x * WPB;
+    const int w0 = blockIdx.x * WPBT + (threadIdx.x >> 5), W = gridDim.x * WPBT;
     const int n = A.n, ngrp = (n + 4) / 5;
     double* x = a.ca->d;
     double* Rb[2] = {a.r, a.z};
@@ -1106,7 +1106,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_cg1(const GArgs a) {
             }
         });
         double v[1] = {mu}, tot[1];
-        grid_allsum<1>(a, grid, 4, v, tot);
+        sync.template allsum<1>(4, v, tot);
         if (!(tot[0] > 0.0) || !isfinite(tot[0])) status = DDA_ERR_BREAKDOWN;
         alpha = rho / tot[0];
     }
@@ -1146,7 +1146,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_cg1(const GArgs a) {
             }
         });
         double bv[3] = {rz, mu, lb}, btot[3];
-        grid_allsum<3>(a, grid, cur ? 4 : 1, bv, btot);
+        sync.template allsum<3>(cur ? 4 : 1, bv, btot);
         const double rho1 = btot[0];
         iters = k + 1;
         if (a.hist && k < a.hist_cap && blockIdx.x == 0 && threadIdx.x == 0) {
@@ -1165,7 +1165,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_cg1(const GArgs a) {
                 rl += o * o;
             }
             double cv[1] = {rl}, ctot[1];
-            grid_allsum<1>(a, grid, 0, cv, ctot);
+            sync.template allsum<1>(0, cv, ctot);
             if (a.hist && k < a.hist_cap && blockIdx.x == 0 && threadIdx.x == 0) a.hist[2 * (size_t)k + 1] = ctot[0];
             checks += 1;
             rr_last = ctot[0];
@@ -1181,6 +1181,7 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_cg1(const GArgs a) {
         rho = rho1;
         if (k >= maxit) { status = DDA_ERR_NO_CONVERGENCE; break; }
     }
+    sync.finish();
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         st->k = k;
         st->iters = iters;
@@ -1193,6 +1194,70 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_cg1(const GArgs a) {
         st->pend = 0;   // x already holds x_{k}
         st->checks = checks;
     }
+}
+
+
+// the grid-wide form: cooperative grid, fixed-order sums of the CTA partials in global memory
+struct GridSyncCg1 {
+    const GArgs& a;
+    cg::grid_group grid;
+    __device__ __forceinline__ void finish() {}
+    template <int NV>
+    __device__ __forceinline__ void allsum(int slot, double (&v)[NV], double (&tot)[NV]) {
+        grid_allsum<NV>(a, grid, slot, v, tot);
+    }
+};
+
+template <int MINB>
+__global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_cg1(const GArgs a) {
+    GridSyncCg1 s{a, cg::this_grid()};
+    sp_cg1_body<DDA_THREADS>(a, s);
+}
+
+// Small systems (the paper's case-1 scale): ONE thread-block cluster runs the whole loop.  The
+// cluster barrier (barrier.cluster, hardware) replaces the grid barrier, and every reduction reads
+// the cluster's CTA partials from their shared memory through DSMEM (map_shared_rank) in rank order:
+// deterministic, no global partials, no grid-wide barrier.  Vectors written by other CTAs of the
+// cluster are read after barrier.cluster's release / acquire (cluster scope).
+constexpr int kClThreads = 512;   // 16 warps per CTA
+struct ClusterSyncCg1 {
+    cg::cluster_group cl;
+    // no CTA may exit while another can still read its shared memory through DSMEM
+    __device__ __forceinline__ void finish() { cl.sync(); }
+    template <int NV>
+    __device__ __forceinline__ void allsum(int slot, double (&v)[NV], double (&tot)[NV]) {
+        __shared__ double red[NV][kClThreads / 32];
+        __shared__ double cpart[8];
+        const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+#pragma unroll
+        for (int k = 0; k < NV; ++k) v[k] = warp_sum(v[k]);
+        if (lane == 0) {
+#pragma unroll
+            for (int k = 0; k < NV; ++k) red[k][wib] = v[k];
+        }
+        cta_barrier();
+        if (threadIdx.x == 0) {
+#pragma unroll
+            for (int k = 0; k < NV; ++k) {
+                double s = 0.0;
+                for (int w = 0; w < kClThreads / 32; ++w) s += red[k][w];
+                cpart[slot + k] = s;
+            }
+        }
+        cl.sync();
+        const int nr = (int)cl.num_blocks();
+#pragma unroll
+        for (int k = 0; k < NV; ++k) {
+            double s = 0.0;
+            for (int r = 0; r < nr; ++r) s += *cl.map_shared_rank(&cpart[slot + k], r);
+            tot[k] = s;
+        }
+    }
+};
+
+__global__ void __launch_bounds__(kClThreads, 1) k_sp_cg1_cl(const GArgs a) {
+    ClusterSyncCg1 s{cg::this_cluster()};
+    sp_cg1_body<kClThreads>(a, s);
 }
 
 __global__ void __launch_bounds__(DDA_THREADS, 3) k_sp_ssor(const GArgs a) {
@@ -1337,6 +1402,28 @@ unsigned long long* g_trace = nullptr;   // k_sp_loop timeline (internal hook dd
 int g_trace_iters = 0;
 
 constexpr int kCg1Rows = 60000;   // k_sp_cg1 below this many block rows (see pcg_graph_solve)
+constexpr int kClMaxRows = 65536; // k_sp_cg1_cl (one cluster, opt-in) up to this many block rows
+constexpr int kClCtas = 16;       // the cluster: 16 CTAs of kClThreads (non-portable size)
+bool cluster_size_ok() {
+    static int ok = -1;
+    if (ok < 0) {
+        cudaFuncSetAttribute(k_sp_cg1_cl, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(kClCtas);
+        cfg.blockDim = dim3(kClThreads);
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeClusterDimension;
+        at[0].val.clusterDim.x = kClCtas;
+        at[0].val.clusterDim.y = 1;
+        at[0].val.clusterDim.z = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        int nclusters = 0;
+        ok = (cudaOccupancyMaxActiveClusters(&nclusters, k_sp_cg1_cl, &cfg) == cudaSuccess && nclusters >= 1) ? 1 : 0;
+        cudaGetLastError();
+    }
+    return ok == 1;
+}
 
 // Per-handle cached graph engine
 struct PcgGraph {
@@ -1347,6 +1434,7 @@ struct PcgGraph {
     cudaGraphConditionalHandle h = 0;
     int G_spmv = 0, G_vec = 0, g_ilu = 0;
     int G_persist = 0;   // scaled engine, persistent loop: cooperative grid (0: graph loop)
+    bool cluster = false;   // the persistent loop is k_sp_cg1_cl in one thread-block cluster
     int body_iters = 2;
 };
 
@@ -1398,6 +1486,10 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     // crossover).  DDA_SCALED_CG1 = 0 / 1 forces either (tests, A/B).
     const int cg1_env = env_int("DDA_SCALED_CG1", -1);
     const bool cg1 = scaled && pc == DDA_PC_BJ && (cg1_env >= 0 ? cg1_env != 0 : K->n < kCg1Rows);
+    // the single-reduction loop in ONE thread-block cluster (k_sp_cg1_cl): opt-in (DDA_SCALED_CLUSTER=1,
+    // up to kClMaxRows), measured slower than the grid form at every size
+    const bool cl = cg1 && g_scaled_loop != 0 && K->n <= kClMaxRows && env_int("DDA_SCALED_CLUSTER", 0) == 1 &&
+                    cluster_size_ok();
     const void* persist_kernel = pc == DDA_PC_SSOR_AI ? reinterpret_cast<const void*>(k_sp_ssor)
                                                       : cg1 ? reinterpret_cast<const void*>(k_sp_cg1<3>)
                                                       : reinterpret_cast<const void*>(k_sp_loop<3>);
@@ -1416,7 +1508,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
             persist = false;
         }
     }
-    const int key = (scaled ? (persist ? 200 : 100) + (int)pc : (int)pc) + (cg1 ? 1000 : 0);
+    const int key = (scaled ? (persist ? 200 : 100) + (int)pc : (int)pc) + (cg1 ? 1000 : 0) + (cl ? 2000 : 0);
     PcgGraph*& G = reinterpret_cast<PcgGraph*&>(K->graph_engine);
     if (G && G->pc != key) {
         pcg_graph_free(G);
@@ -1438,7 +1530,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, persist_kernel, DDA_THREADS, 0);
             if (per_sm > 3) per_sm = 3;
             if (per_sm < 1) per_sm = 1;   // (checked above)
-            g_persist = device_sms() * per_sm;
+            g_persist = cl ? kClCtas : device_sms() * per_sm;
             // small (L2-resident) systems are barrier-latency bound: no more CTAs than ten-row groups
             // need (DDA_PERSIST_CTAS overrides, tuning aid)
             const int cap = env_int("DDA_PERSIST_CTAS", need_rows > 0 ? need_rows : 1);
@@ -1454,6 +1546,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         G->G_spmv = g_spmv;
         G->G_vec = g_vec;
         G->G_persist = g_persist;
+        G->cluster = cl;
         double* ws = K->ws;
         GArgs& a = G->a;
         a.A = view_of(K);
@@ -1575,9 +1668,24 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         a.trace_iters = g_trace_iters;
         a.hist = K->hist;
         a.hist_cap = K->hist_cap;
-        void* kargs[] = {reinterpret_cast<void*>(&a)};
-        DDA_CK(cudaLaunchCooperativeKernel(persist_kernel, dim3(G->G_persist),
-                                           dim3(DDA_THREADS), kargs, 0, st));
+        if (G->cluster) {   // one cluster of kClCtas CTAs (co-scheduled by the hardware)
+            cudaLaunchConfig_t cfg = {};
+            cfg.gridDim = dim3(kClCtas);
+            cfg.blockDim = dim3(kClThreads);
+            cfg.stream = st;
+            cudaLaunchAttribute at[1];
+            at[0].id = cudaLaunchAttributeClusterDimension;
+            at[0].val.clusterDim.x = kClCtas;
+            at[0].val.clusterDim.y = 1;
+            at[0].val.clusterDim.z = 1;
+            cfg.attrs = at;
+            cfg.numAttrs = 1;
+            DDA_CK(cudaLaunchKernelEx(&cfg, k_sp_cg1_cl, a));
+        } else {
+            void* kargs[] = {reinterpret_cast<void*>(&a)};
+            DDA_CK(cudaLaunchCooperativeKernel(persist_kernel, dim3(G->G_persist),
+                                               dim3(DDA_THREADS), kargs, 0, st));
+        }
         DDA_LAUNCHED();
     } else {
         DDA_CK(cudaGraphLaunch(G->exec, st));

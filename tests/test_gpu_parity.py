@@ -270,7 +270,8 @@ def _set_engine(dda, engine, loop=-1):
     g(loop)
 
 
-@pytest.fixture(params=["auto", "graph", "persistent", "scaled", "scaled_2phase", "scaled_cg1", "scaled_graph"])
+@pytest.fixture(params=["auto", "graph", "persistent", "scaled", "scaled_2phase", "scaled_cg1", "scaled_cluster",
+                        "scaled_graph"])
 def engine(request, dda, monkeypatch):
     """PCG engine: the CUDA-graph while loop, the persistent cooperative kernel, or the
     block-scaled matrix S K S^T (block-Jacobi only; other preconditioners fall back to
@@ -278,10 +279,12 @@ def engine(request, dda, monkeypatch):
     or the single-reduction k_sp_cg1 by size; '_2phase' / '_cg1' force one) or by the
     CUDA-graph while loop ('scaled_graph') — internal hooks; 'auto' picks by size and
     preconditioner."""
-    if request.param in ("scaled_2phase", "scaled_cg1"):
-        monkeypatch.setenv("DDA_SCALED_CG1", "1" if request.param == "scaled_cg1" else "0")
+    if request.param in ("scaled_2phase", "scaled_cg1", "scaled_cluster"):
+        monkeypatch.setenv("DDA_SCALED_CG1", "0" if request.param == "scaled_2phase" else "1")
+        monkeypatch.setenv("DDA_SCALED_CLUSTER", "1" if request.param == "scaled_cluster" else "0")
     _set_engine(dda, *{"auto": (-1, -1), "graph": (0, -1), "persistent": (1, -1), "scaled": (2, 1),
-                       "scaled_2phase": (2, 1), "scaled_cg1": (2, 1), "scaled_graph": (2, 0)}[request.param])
+                       "scaled_2phase": (2, 1), "scaled_cg1": (2, 1), "scaled_cluster": (2, 1),
+                       "scaled_graph": (2, 0)}[request.param])
     yield request.param
     _set_engine(dda, -1, -1)
 
