@@ -534,3 +534,36 @@ def test_scaled_ssor_omega0_is_bj(dda, name):
     assert stb == sts == dda.OK and itb == its, (itb, its)
     db, ds = db.cpu().numpy(), ds.cpu().numpy()
     assert np.linalg.norm(ds - db) <= 1e-12 * np.linalg.norm(db)
+
+
+def test_new_entry_points_reject_bad_arguments(dda):
+    """Argument checks of the round-2 entry points (dda.h): dda_pcg_set_history with a buffer / capacity
+    mismatch, dda_solve_host_batch with a system missing its arrays, and the IPC import of blobs that
+    are not a consistent set (wrong size, wrong rank order) or on a communicator without a partition."""
+    import ctypes as C
+    L = dda.lib()
+    P, O = case("tiny")
+    K = dda.build_from_problem(P)
+    assert L.dda_pcg_set_history(K.handle, None, 5) == dda.ERR_ARG
+    assert L.dda_pcg_set_history(None, None, 0) == dda.ERR_ARG
+    assert L.dda_pcg_set_history(K.handle, None, 0) == dda.OK
+    bad = (dda.HostSystem * 1)()
+    bad[0].n_blocks = P.n
+    assert L.dda_solve_host_batch(1, bad, 1e-10, 100, 0, 1.0, None) == dda.ERR_ARG
+    assert L.dda_solve_host_batch(-1, None, 1e-10, 100, 0, 1.0, None) == dda.ERR_ARG
+    assert L.dda_solve_host_batch(0, None, 1e-10, 100, 0, 1.0, None) == dda.OK
+    # IPC: import before a partition exists, then blobs of the wrong size / order
+    c = dda.Comm.ipc(2, 0)
+    n = C.c_int64()
+    assert L.dda_comm_ipc_export(c._h, None, C.byref(n)) == dda.OK and n.value > 0
+    buf = C.create_string_buffer(2 * n.value)
+    assert L.dda_comm_ipc_import(c._h, buf, n.value) == dda.ERR_ARG         # no partition attached
+    t = dda.problem_to_device(P)
+    b = dda.row_bounds(P.n, 2)
+    c.build_matrix_dist(0, P.n, b, t["kdiag"][: int(b[1])].contiguous(), t["bi"], t["bj"], t["pen"], t["e"], t["g"])
+    blob = c.ipc_export()
+    assert L.dda_comm_ipc_import(c._h, C.create_string_buffer(blob * 2, 2 * len(blob)), len(blob) - 8) == dda.ERR_ARG
+    assert L.dda_comm_ipc_import(c._h, C.create_string_buffer(blob * 2, 2 * len(blob)), len(blob)) == dda.ERR_ARG   # rank 0 twice
+    c.free()
+    with pytest.raises(Exception):
+        dda.Comm.ipc(2, 5)
