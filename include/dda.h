@@ -265,11 +265,14 @@ dda_status_t dda_solve_host_batch(int32_t nsys, dda_host_system *sys, double tol
  * statuses and reported TRUE residual as dda_pcg_solve; DDA_PC_BJ or
  * DDA_PC_NONE (SSOR-AI and ILU(0) are single-GPU only).  Block-Jacobi runs the
  * scaled engine per partition (PCG on S K S^T, reading Z25; S of the halo rows is
- * exchanged once per solve); per iteration: halo exchanges of r~ and p, the fused
- * p-update + SpMV over own rows, allreduces of p^T q and of (|r~|^2, the stopping
- * bound), and of |L r~|^2 when the exact stopping test is due.  The CG scalars
- * stay on the device; the host reads the loop state once per DDA_DIST_CHUNK (8)
- * iterations.  DDA_DIST_SCALED=0 selects the unscaled loop.  Synchronising.
+ * exchanged once per solve).  The loop depends on the transport: NCCL runs v4
+ * (per iteration one halo of p overlapped with the interior rows and one 6-double
+ * allreduce); LOOPBACK runs v6 (every partition in ONE persistent cooperative
+ * kernel, halo rows read from their owners, fixed-order sums); IPC runs v7 (one
+ * persistent kernel per rank, see dda_comm_init_ipc).  DDA_DIST_VERSION = 7 / 5 /
+ * 4 / 3 selects the loopback per-rank kernels, the peer-load per-iteration
+ * launches, the halo-copy launches or the round-1 loop; DDA_DIST_SCALED=0 the
+ * unscaled loop (also the unpreconditioned solve).  Synchronising.
  * dda_spmv_dist: y = K x over own rows (x, y device [6 n_own] per partition).
  */
 typedef struct dda_comm *dda_comm_t;
