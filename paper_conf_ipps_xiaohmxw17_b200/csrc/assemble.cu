@@ -287,7 +287,7 @@ void dda::matrix_free_impl(dda_matrix_t K, cudaStream_t* sync) {
     void* ptrs[] = {K->row_ptr, K->col_idx, K->low_ptr, K->low_row, K->low_to_up, K->urow, K->diag, K->upper,
                     K->perm, K->seg, K->dperm, K->dstart, K->orient, K->dinv, K->ws, K->scratch,
                     K->ilu_up, K->ilu_inv, K->ilu_flags, K->ilu_order, K->full_ptr, K->full_col, K->full_val,
-                    K->lfac, K->sfac, K->bj_w, K->sc_upper, K->rperm, K->rinv, K->rtmp, K->tma_tiles};
+                    K->lfac, K->sfac, K->bj_w, K->sc_upper, K->rperm, K->rinv, K->rtmp, K->tma_tiles, K->lr_off, K->lr_buf};
     for (void* p : ptrs)
         if (p) dev_free(p);
     cudaSetDevice(prev);

@@ -179,6 +179,10 @@ struct dda_matrix {
     int32_t* rperm = nullptr;
     int32_t* rinv = nullptr;
     double* rtmp = nullptr;         // [3][6n] permuted vector scratch
+    // push-form phase A of the persistent BJ loop (pcg_graph.cu, phase_a_lr): structure-only map
+    int32_t* lr_off = nullptr;      // [nnzb] entry of upper block u in lr_buf, 16 B units
+    void* lr_buf = nullptr;         // 48 nnzb + 128 ceil(n/10) + 128 bytes of entries, then counters
+    size_t lr_bytes = 0;            // bytes of entries (the counters follow)
 };
 
 // contact records of dda_detect_contacts (contact.cu) and the open-close state (openclose.cu)

@@ -79,6 +79,12 @@ struct GArgs {           // constant for a (matrix, preconditioner): baked into 
     int trace_iters;
     double* hist;        // residual history [hist_cap][2] (dda_pcg_set_history), null = off
     int hist_cap;
+    // k_sp_loop push form (phase_a_lr): entries, their offsets per upper block, per-step counters
+    double2* lr;
+    const int* lr_off;
+    unsigned* lr_cnt;
+    int lr_discard;
+    int lr_sync;
 };
 
 __device__ __forceinline__ unsigned long long gtimer() {
@@ -809,8 +815,296 @@ __device__ __forceinline__ void grid_allsum(const GArgs& a, cg::grid_group& grid
     cta_barrier();
 }
 
-template <int MINB>
+// ---- phase A with the transposed products pushed, not pulled ("low-res" in L2)
+//
+// The paper's two-stage SpMV applies every stored block once in both directions and
+// parks the transposed product V_ij^T x_i in a low-res array that a second stage sums per row.
+// k_sp_loop's pull form instead re-reads each V_ki through low_to_up from L2 (0.86 GB per iteration
+// at 1M) and gathers the lower neighbours' r~ / p_old, which puts phase A at the L2 sector cap
+// (DESIGN.md §10).  Here one sweep does both stages, ten block rows per warp step:
+//   produce (step s):  p_i (own rows), the forward products V_ij p_j, and the 48 B push
+//                      lr[slot(ij)] = V_ij^T p_i for every upper block, in the same registers;
+//   consume (step s-1): q_j = p_j + (its forward sum, kept in registers) + sum over its lower
+//                      blocks of the pushed entries, in lower-CSR order (deterministic).
+// A row's lower blocks all belong to rows with a smaller index, so to steps <= its own; one step of
+// lag plus an ordering of the pushes before the reads replaces a grid barrier: per-group ready flags
+// (release by the producing warp, acquire per pushing group by the consumer; default), per-step
+// arrival counters, or entries tagged with the iteration parity in their last mantissa bit (the
+// data is its own flag; results then differ from the untagged form by <= 1 ulp per entry).  The
+// entries are laid out by CONSUMER group, each ten-row group's run 128 B aligned
+// (base(g) = roundup128(48 lo(10g) + 128 g)), and the consuming warp may discard its lines from L2
+// after reading them (discard.global.L2; not with tags) so they never reach HBM.
+// Measured at 1M (profiles/r02_push_form.md): correct, but slower than the pull form
+// (373-399 vs 304 us per iteration; 327 with no ordering at all): the producer holds p_i, the
+// pending group and two blocks in flight in 128 registers, so 16 warps per SM instead of 24, and
+// the 16 B entry accesses give back most of the L2 sectors the transposed re-reads cost.  Opt-in.
+struct LrArgs {
+    double2* lr;           // pushed entries (16 B units)
+    const int* lr_off;     // [nnzb] entry of upper block u, in 16 B units
+    unsigned* cnt;         // [ngrp] per-group ready flags (epoch), or [nsteps] per-step counters; zeroed per launch
+    int discard;           // discard consumed lines from L2
+    int sync;              // 0 per-group flags, 1 per-step counters, 2 none (timing diagnostic only: wrong results)
+};
+
+__device__ __forceinline__ void red_release_add(unsigned* p, unsigned v) {
+    asm volatile("red.release.gpu.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned ld_acquire_u(const unsigned* p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void l2_discard(const void* p) {
+    asm volatile("discard.global.L2 [%0], 128;" ::"l"(p) : "memory");
+}
+__device__ __forceinline__ double tag_lsb(double v, int t) {
+    return __longlong_as_double((__double_as_longlong(v) & ~1ll) | (long long)t);
+}
+__device__ __forceinline__ void st_relaxed2(double2* p, double x, double y) {
+    asm volatile("st.relaxed.gpu.global.v2.f64 [%0], {%1, %2};" ::"l"(p), "d"(x), "d"(y) : "memory");
+}
+__device__ __forceinline__ double2 ld_relaxed2(const double2* p) {
+    double2 v;
+    asm volatile("ld.relaxed.gpu.global.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ long long lr_base16(int lo_first, int g) {   // group g's first entry, 16 B units
+    return ((48ll * lo_first + 128ll * g + 127) >> 7) << 3;
+}
+
+// Forward products and pushes of row i (group lanes; lane C owns column pair C of every block):
+// y (pair C after the 3-lane reduce-scatter) = sum_j V_ij p_j, and lr entry of block ij, pair C,
+// = sum_r V_ij[r][2C..2C+1] p_i[r] (the lane holds column pair C of all six rows).  Two blocks in
+// flight per lane, the block list decoded one block ahead (as spmv_row_c5).
+template <bool DEEP, class XLoad>
+__device__ __forceinline__ void lr_row_produce(const BsrView& A, const LrArgs& L, int i, bool ok, const RowBounds& rb,
+                                               const XLoad& xload, int lane, const double (&p6)[6], double& y0,
+                                               double& y1, int tag) {
+    const unsigned full = 0xffffffffu;
+    const int h = cgrp_of(lane);
+    const int C = ccol_of(lane);
+    const int nb = (ok && lane < 30) ? rb.nu : 0;
+    const int nbmax = __reduce_max_sync(full, nb);
+    double acc[6] = {0.0, 0.0, 0.0, 0.0, 0.0, 0.0};
+    auto decode = [&](int b, int& vec, int& off) {
+        const bool v = b < nb;
+        vec = v ? __ldg(A.col_idx + rb.up0 + b) : 0;
+        off = v ? __ldg(L.lr_off + rb.up0 + b) : 0;
+    };
+    struct D {
+        double4 c0, c1, c2;
+        double2 x;
+    };
+    auto load = [&](int b, int vec) {
+        D d;
+        const bool v = b < nb;
+        const double* blk = A.upper + (size_t)kBlk * (rb.up0 + (v ? b : 0));
+        d.x = v ? xload.raw(vec, C) : make_double2(0.0, 0.0);
+        d.c0 = ld_chunk_if(blk + 4 * C, v);
+        d.c1 = ld_chunk_if(blk + 4 * (3 + C), v);
+        d.c2 = ld_chunk_if(blk + 4 * (6 + C), v);
+        return d;
+    };
+    int v1, o1, o0;
+    decode(0, v1, o0);
+    D d0 = load(0, v1);
+    decode(1, v1, o1);
+    for (int b = 0; b < nbmax; ++b) {
+        int v2, o2;
+        decode(b + 2, v2, o2);
+        D d1;
+        if (DEEP) d1 = load(b + 1, v1);   // two blocks in flight (else the next block loads after use)
+        const double4 cs[3] = {d0.c0, d0.c1, d0.c2};
+        const double2 xv = d0.x;
+        double e0 = 0.0, e1 = 0.0;
+#pragma unroll
+        for (int k = 0; k < 3; ++k) {
+            const double4 c = cs[k];
+            acc[2 * k] = fma(c.x, xv.x, fma(c.y, xv.y, acc[2 * k]));
+            acc[2 * k + 1] = fma(c.z, xv.x, fma(c.w, xv.y, acc[2 * k + 1]));
+            e0 = fma(c.z, p6[2 * k + 1], fma(c.x, p6[2 * k], e0));
+            e1 = fma(c.w, p6[2 * k + 1], fma(c.y, p6[2 * k], e1));
+        }
+        if (b < nb) {
+            if (tag >= 0)   // last mantissa bit = iteration parity (the entry is its own ready flag)
+                st_relaxed2(L.lr + (size_t)o0 + C, tag_lsb(e0, tag), tag_lsb(e1, tag));
+            else
+                L.lr[(size_t)o0 + C] = make_double2(e0, e1);
+        }
+        if (!DEEP) d1 = load(b + 1, v1);
+        d0 = d1;
+        v1 = v2;
+        o0 = o1;
+        o1 = o2;
+    }
+    const int c1 = C == 2 ? 0 : C + 1, c2 = C == 0 ? 2 : C - 1;
+    const int s1 = lane < 30 ? 3 * h + c1 : lane, s2 = lane < 30 ? 3 * h + c2 : lane;
+    const double2 w1 = pick_pair(acc, c2);
+    const double r1x = __shfl_sync(full, w1.x, s1), r1y = __shfl_sync(full, w1.y, s1);
+    const double2 w2 = pick_pair(acc, c1);
+    const double r2x = __shfl_sync(full, w2.x, s2), r2y = __shfl_sync(full, w2.y, s2);
+    const double2 own = pick_pair(acc, C);
+    y0 = (own.x + r1x) + r2x;
+    y1 = (own.y + r1y) + r2y;
+}
+
+// Phase A of k_sp_loop in the push form; returns this thread's partial of sigma = p.q.  `target` is
+// the per-step counter value that means "every warp has produced this step in this iteration".
+template <bool DEEP>
+__device__ __forceinline__ double phase_a_lr(const GArgs& a, const LrArgs& L, const BsrView& A, const XFusedW& xf,
+                                             const double* pold, double* pnew, double* x, double ap, int w0, int W,
+                                             int lane, unsigned epoch) {
+    const unsigned target = epoch * (unsigned)W;   // per-step counters: every warp produced the step
+    const unsigned full = 0xffffffffu;
+    const int h = cgrp_of(lane), C = ccol_of(lane);
+    const bool lane_ok = lane < 30;
+    const int n = A.n, ngrp = (n + 9) / 10, nsteps = (ngrp + W - 1) / W;
+    double acc = 0.0;
+    bool have = false;                      // a produced group waiting for its lower pushes
+    int pg = 0, plo = 0, pnl = 0;
+    double py0 = 0.0, py1 = 0.0, pp0 = 0.0, pp1 = 0.0;
+    // consume, first half: wait for the pushes into the pending group's rows (sync 0 / 1), then issue
+    // the loads of up to three of each row's entries, which stay in flight while the next group is
+    // produced; sync 3 tags every pushed double with the iteration parity in its last mantissa bit
+    // and the reader re-loads until the tag matches (the data is its own ready flag)
+    const unsigned par = epoch & 1u;
+    double2 lv[3];
+    long long cb16 = 0;
+    auto consume_begin = [&](int s) {
+        const int j = 10 * pg + h;
+        const bool ok = lane_ok && j < n;
+        if (L.sync == 1 && lane == 0) {
+            unsigned spins = 0;
+            while ((int)(ld_acquire_u(L.cnt + s) - target) < 0) {
+                __nanosleep(32);
+                if (++spins > (1u << 26)) __trap();   // a lost arrival: fail loudly, never hang the GPU
+            }
+        } else if (L.sync == 0 && ok) {
+            // the groups that pushed into this row (other than this warp's own, ordered by __syncwarp)
+            for (int e = C; e < pnl; e += 3) {
+                const int pgrp = __ldg(A.low_row + plo + e) / 10;
+                if (pgrp == pg) continue;
+                unsigned spins = 0;
+                while ((int)(ld_acquire_u(L.cnt + pgrp) - epoch) < 0) {
+                    __nanosleep(32);
+                    if (++spins > (1u << 26)) __trap();
+                }
+            }
+        }
+        __syncwarp();
+        const int lo_first = __shfl_sync(full, plo, 0);   // lane 0 holds row 10 pg (always < n)
+        cb16 = lr_base16(lo_first, pg);
+        const double2* src = L.lr + cb16 + 3ll * (plo - lo_first) + C;
+        const int nl = ok ? pnl : 0;
+#pragma unroll
+        for (int t = 0; t < 3; ++t)
+            lv[t] = t < nl ? (L.sync == 3 ? ld_relaxed2(src + 3 * t) : __ldcg(src + 3 * t)) : make_double2(0.0, 0.0);
+    };
+    auto consume_end = [&]() {
+        const int j = 10 * pg + h;
+        const bool ok = lane_ok && j < n;
+        const int lo_first = __shfl_sync(full, plo, 0);
+        const int lo_end = __reduce_max_sync(full, ok ? plo + pnl : 0);
+        const double2* src = L.lr + cb16 + 3ll * (plo - lo_first) + C;
+        const int nl = ok ? pnl : 0;
+        double y0 = py0, y1 = py1;
+        for (int e = 0; e < nl; ++e) {
+            double2 v = e < 3 ? (e == 0 ? lv[0] : (e == 1 ? lv[1] : lv[2]))
+                              : (L.sync == 3 ? ld_relaxed2(src + 3 * e) : __ldcg(src + 3 * e));
+            if (L.sync == 3) {
+                unsigned spins = 0;
+                while (((unsigned)__double_as_longlong(v.x) & 1u) != par || ((unsigned)__double_as_longlong(v.y) & 1u) != par) {
+                    if (++spins > (1u << 26)) __trap();
+                    v = ld_relaxed2(src + 3 * e);
+                }
+            }
+            y0 += v.x;
+            y1 += v.y;
+        }
+        if (ok) {
+            const size_t o = 6 * (size_t)j + 2 * C;
+            *reinterpret_cast<double2*>(a.q + o) = make_double2(y0, y1);
+            acc += pp0 * y0 + pp1 * y1;
+        }
+        if (L.discard && L.sync != 3) {
+            __syncwarp();
+            const int nlines = (int)((48ll * (lo_end - lo_first) + 127) >> 7);
+            const char* base = reinterpret_cast<const char*>(L.lr + cb16);
+            for (int l = lane; l < nlines; l += 32) l2_discard(base + 128 * (size_t)l);
+        }
+    };
+    RowBounds nxt = row_bounds<SPMV_OFFDIAG>(A, 10 * w0 + h, lane_ok);
+    for (int s = 0; s < nsteps; ++s) {
+        const int g = w0 + s * W;
+        const int i = 10 * g + h;
+        const bool ok = lane_ok && i < n;
+        const RowBounds cur = nxt;
+        nxt = row_bounds<SPMV_OFFDIAG>(A, i + 10 * W, lane_ok);
+        // own p_i pair (x = r~ + beta p_old, as the gathers form it) and x += alpha_prev p_old
+        double2 pv = make_double2(0.0, 0.0);
+        if (ok) {
+            const size_t o = 6 * (size_t)i + 2 * C;
+            const double2 po = ld_cg2(pold + o);
+            const double2 rr = ld_cg2(a.r + o);
+            pv = make_double2(fma(xf.beta, po.x, rr.x), fma(xf.beta, po.y, rr.y));
+            const double2 xo = ld_cg2(x + o);
+            *reinterpret_cast<double2*>(x + o) = make_double2(xo.x + ap * po.x, xo.y + ap * po.y);
+            *reinterpret_cast<double2*>(pnew + o) = pv;
+        }
+        double p6[6];
+        {
+            const int b0 = lane_ok ? 3 * h : lane;
+#pragma unroll
+            for (int c = 0; c < 3; ++c) {
+                p6[2 * c] = __shfl_sync(full, pv.x, lane_ok ? b0 + c : lane);
+                p6[2 * c + 1] = __shfl_sync(full, pv.y, lane_ok ? b0 + c : lane);
+            }
+        }
+        if (have) consume_begin(s - 1);
+        double y0, y1;
+        lr_row_produce<DEEP>(A, L, i, ok, cur, xf, lane, p6, y0, y1, L.sync == 3 ? (int)par : -1);
+        __syncwarp();
+        if (lane == 0) {
+            if (L.sync == 1)
+                red_release_add(L.cnt + s, 1u);
+            else if (L.sync == 0 && g < ngrp)
+                st_release(reinterpret_cast<int*>(L.cnt + g), (int)epoch);
+        }
+        if (have) consume_end();
+        have = g < ngrp;
+        pg = g;
+        plo = cur.lo0;
+        pnl = cur.nl;
+        py0 = y0 + pv.x;
+        py1 = y1 + pv.y;
+        pp0 = pv.x;
+        pp1 = pv.y;
+    }
+    if (have) {
+        consume_begin(nsteps - 1);
+        consume_end();
+    }
+    return acc;
+}
+
+// lr_off[u] for every upper block u = (i, j): the position of u in row j's lower list (lower CSR
+// index t), inside consumer group j / 10's 128 B-aligned run
+__global__ void k_lr_off(int64_t nnzb, const int32_t* __restrict__ low_ptr, const int32_t* __restrict__ low_to_up,
+                         const int32_t* __restrict__ col_idx, int32_t* __restrict__ lr_off) {
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < nnzb; t += (int64_t)gridDim.x * blockDim.x) {
+        const int u = __ldg(low_to_up + t);
+        const int j = __ldg(col_idx + u);
+        const int g = j / 10;
+        const int lo_first = __ldg(low_ptr + 10 * g);
+        lr_off[u] = (int32_t)(lr_base16(lo_first, g) + 3 * (t - lo_first));
+    }
+}
+
+// LR: 0 = phase A in the pull form (for_rows_c), 1 = push form (phase_a_lr) with one block in flight
+// per lane, 2 = with two (the opt-in variant: 128 registers, 2 CTAs/SM)
+template <int MINB, int LR>
 __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_loop(const GArgs a) {
+    const LrArgs L{a.lr, a.lr_off, a.lr_cnt, a.lr_discard, a.lr_sync};
     cg::grid_group grid = cg::this_grid();
     State* st = a.st;
     unsigned long long* tr_k = (a.trace && blockIdx.x == 0 && threadIdx.x == 0)
@@ -852,7 +1146,10 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_loop(const GArgs a) {
                 acc += pv.x * y0 + pv.y * y1;
             }
         };
-        for_rows_c<SPMV_OFFDIAG, 5>(A, w0, W, xf, lane, rowA);
+        if (LR)
+            acc = phase_a_lr<LR == 2>(a, L, A, xf, pold, pnew, x, ap, w0, W, lane, (unsigned)(k + 1));
+        else
+            for_rows_c<SPMV_OFFDIAG, 5>(A, w0, W, xf, lane, rowA);
         if (tr) tr[1] = gtimer();
         double sv[1] = {acc}, stot[1];
         grid_allsum<1>(a, grid, 0, sv, stot);
@@ -1462,6 +1759,24 @@ dda_status_t scaled_setup(dda_matrix* K, cudaStream_t st) {
     return DDA_OK;
 }
 
+// The push-form phase A's entry map and buffers (structure only: built once per matrix)
+dda_status_t lr_setup(dda_matrix* K, cudaStream_t st) {
+    if (K->lr_off || K->nnzb == 0) return DDA_OK;
+    const int64_t ngrp = (K->n + 9) / 10;
+    const size_t ebytes = (size_t)(48 * K->nnzb + 128 * ngrp + 256);
+    if ((int64_t)(ebytes / 16) > INT32_MAX) return DDA_ERR_ARG;   // 16 B offsets are int32
+    const size_t cbytes = sizeof(unsigned) * (size_t)(ngrp + 1);
+    DDA_CK(dev_alloc(&K->lr_buf, ebytes + cbytes, st));
+    DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->lr_off), sizeof(int32_t) * (size_t)K->nnzb, st));
+    K->lr_bytes = ebytes;
+    int g = (int)((K->nnzb + 255) / 256);
+    const int cap = device_sms() * 8;
+    if (g > cap) g = cap;
+    k_lr_off<<<g, 256, 0, st>>>(K->nnzb, K->low_ptr, K->low_to_up, K->col_idx, K->lr_off);
+    DDA_LAUNCHED();
+    return DDA_OK;
+}
+
 dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, double* d, double tol,
                              int32_t maxit, dda_precond_t pc, double omega, int32_t* iters, double* rel_res,
                              cudaStream_t st, bool scaled) {
@@ -1490,9 +1805,14 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     // up to kClMaxRows), measured slower than the grid form at every size
     const bool cl = cg1 && g_scaled_loop != 0 && K->n <= kClMaxRows && env_int("DDA_SCALED_CLUSTER", 0) == 1 &&
                     cluster_size_ok();
+    // the two-phase loop's phase A in the pull form (default) or the push form (phase_a_lr, opt-in
+    // DDA_SP_LR=1: measured slower); DDA_LR_SYNC selects its ordering (0 ready flags,
+    // 1 step counters, 3 parity-tagged entries), DDA_LR_DISCARD=0 keeps consumed entries in L2
+    const bool lr = scaled && pc == DDA_PC_BJ && !cg1 && K->nnzb > 0 && env_int("DDA_SP_LR", 0) != 0;
     const void* persist_kernel = pc == DDA_PC_SSOR_AI ? reinterpret_cast<const void*>(k_sp_ssor)
-                                                      : cg1 ? reinterpret_cast<const void*>(k_sp_cg1<3>)
-                                                      : reinterpret_cast<const void*>(k_sp_loop<3>);
+                                 : cg1                ? reinterpret_cast<const void*>(k_sp_cg1<3>)
+                                 : lr                 ? reinterpret_cast<const void*>(k_sp_loop<2, 2>)
+                                                      : reinterpret_cast<const void*>(k_sp_loop<3, 0>);
     if (persist) {
         // The persistent kernels need every CTA co-resident (cooperative launch).  If not even one CTA
         // per SM fits (e.g. a smaller shared-memory carve-out forced by the caller's context), fall
@@ -1508,7 +1828,12 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
             persist = false;
         }
     }
-    const int key = (scaled ? (persist ? 200 : 100) + (int)pc : (int)pc) + (cg1 ? 1000 : 0) + (cl ? 2000 : 0);
+    const int key = (scaled ? (persist ? 200 : 100) + (int)pc : (int)pc) + (cg1 ? 1000 : 0) + (cl ? 2000 : 0) +
+                    (persist && lr ? 4000 : 0);
+    if (persist && lr) {
+        dda_status_t s = lr_setup(K, st);
+        if (s != DDA_OK) return s;
+    }
     PcgGraph*& G = reinterpret_cast<PcgGraph*&>(K->graph_engine);
     if (G && G->pc != key) {
         pcg_graph_free(G);
@@ -1574,6 +1899,11 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         a.sfac = K->sfac;
         a.bj_w = K->bj_w;
         a.dinv_fmax = reinterpret_cast<const unsigned long long*>(reinterpret_cast<char*>(K->scratch) + 192);
+        if (persist && lr) {
+            a.lr = reinterpret_cast<double2*>(K->lr_buf);
+            a.lr_off = K->lr_off;
+            a.lr_cnt = reinterpret_cast<unsigned*>(reinterpret_cast<char*>(K->lr_buf) + K->lr_bytes);
+        }
         G->g_ilu = ilu_grid();
         DDA_CK(cudaMemsetAsync(a.st, 0, sizeof(State), st));       // ticket = 0
 
@@ -1664,6 +1994,8 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     }
     // ---- the device-side loop (its kernel launches are counted below from the iteration count)
     if (G->G_persist) {
+        a.lr_discard = env_int("DDA_LR_DISCARD", 1) != 0;
+        a.lr_sync = env_int("DDA_LR_SYNC", 0);
         a.trace = g_trace;
         a.trace_iters = g_trace_iters;
         a.hist = K->hist;
@@ -1682,6 +2014,14 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
             cfg.numAttrs = 1;
             DDA_CK(cudaLaunchKernelEx(&cfg, k_sp_cg1_cl, a));
         } else {
+            if (a.lr_cnt) {   // the push form's ready flags / step counters start at zero in every launch
+                const int ngrp = (K->n + 9) / 10, W = G->G_persist * WPB;
+                const int nc = a.lr_sync == 1 ? (ngrp + W - 1) / W : ngrp;
+                DDA_CK(cudaMemsetAsync(a.lr_cnt, 0, sizeof(unsigned) * (size_t)nc, st));
+                // tag mode: every entry starts with tag 0, the parity of no iteration of this launch
+                // before the first (iteration k writes tag (k + 1) & 1)
+                if (a.lr_sync == 3) DDA_CK(cudaMemsetAsync(a.lr, 0, K->lr_bytes, st));
+            }
             void* kargs[] = {reinterpret_cast<void*>(&a)};
             DDA_CK(cudaLaunchCooperativeKernel(persist_kernel, dim3(G->G_persist),
                                                dim3(DDA_THREADS), kargs, 0, st));

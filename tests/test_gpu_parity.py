@@ -567,3 +567,34 @@ def test_new_entry_points_reject_bad_arguments(dda):
     c.free()
     with pytest.raises(Exception):
         dda.Comm.ipc(2, 5)
+
+
+@pytest.mark.parametrize("sync,discard", [("0", "1"), ("0", "0"), ("1", "1"), ("3", "0")],
+                         ids=["flags", "flags_keep", "step_counters", "parity_tags"])
+@pytest.mark.parametrize("name", ["tiny", "ragged_1k", "paper"])
+def test_push_form_phase_a(dda, name, sync, discard, monkeypatch):
+    """The opt-in push form of k_sp_loop's phase A (phase_a_lr: each upper block applied once in both
+    directions, V_ij^T p_i pushed to an L2-resident entry the row j sums; the paper's up-res / low-res
+    scheme, in one sweep) under each ordering of pushes before reads: oracle parity
+    (reading Z17), bitwise repeatability, and agreement with the pull form."""
+    P, O = case(name)
+    monkeypatch.setenv("DDA_SCALED_CG1", "0")
+    out = {}
+    try:
+        _set_engine(dda, 2, 1)
+        monkeypatch.setenv("DDA_SP_LR", "0")
+        out["pull"] = _pcg_parity(dda, P, O, "bj")
+        monkeypatch.setenv("DDA_SP_LR", "1")
+        monkeypatch.setenv("DDA_LR_SYNC", sync)
+        monkeypatch.setenv("DDA_LR_DISCARD", discard)
+        out["push"] = _pcg_parity(dda, P, O, "bj")
+        K = dda.build_from_problem(P)
+        F = torch.from_numpy(P.F).cuda()
+        a = K.pcg_solve(F)[0].cpu().numpy()
+        b = K.pcg_solve(F)[0].cpu().numpy()
+    finally:
+        _set_engine(dda, -1, -1)
+    assert np.array_equal(a, b)
+    (dl, itl), (dp, itp) = out["pull"], out["push"]
+    assert abs(itl - itp) <= 1, (itl, itp)
+    assert np.linalg.norm(dp - dl) <= 1e-9 * np.linalg.norm(dl)

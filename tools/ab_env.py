@@ -32,6 +32,6 @@ for r in range(reps + 1):
         if r:
             res[i].append(a.elapsed_time(b))
 print(json.dumps({"n": K.n, "sets": sets, "median_ms": [statistics.median(res[i]) for i in res],
-                  "us_per_iter": [1000 * statistics.median(res[i]) / its[i][0] for i in res],
+                  "us_per_iter": [1000 * statistics.median(res[i]) / max(its[i][0], 1) for i in res],
                   "iters_rel_status": [its[i] for i in res], "max_rel_diff_vs_first": [diff[i] for i in res],
                   "all": [res[i] for i in res]}), flush=True)
