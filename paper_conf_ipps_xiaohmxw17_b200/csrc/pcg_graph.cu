@@ -31,6 +31,8 @@ namespace dda {
 namespace {
 
 constexpr int WPB = DDA_THREADS / 32;
+// largest power of two <= DDA_THREADS (the CTA tree sums; the library is built with 256)
+constexpr int kTreeP2 = DDA_THREADS >= 512 ? 512 : DDA_THREADS >= 256 ? 256 : DDA_THREADS >= 128 ? 128 : 64;
 
 struct CallArgs {
     const double* F;
@@ -144,7 +146,14 @@ __device__ __forceinline__ bool grid_reduce_last(const GArgs& a, double (&v)[NV]
         red[k][threadIdx.x] = s;
     }
     cta_barrier_na();
-    for (int h = DDA_THREADS / 2; h > 0; h >>= 1) {      // fixed-shape tree
+    if (kTreeP2 < DDA_THREADS) {                          // fold a non-power-of-two CTA first
+        if ((int)threadIdx.x < DDA_THREADS - kTreeP2) {
+#pragma unroll
+            for (int k = 0; k < NV; ++k) red[k][threadIdx.x] += red[k][threadIdx.x + kTreeP2];
+        }
+        cta_barrier_na();
+    }
+    for (int h = kTreeP2 / 2; h > 0; h >>= 1) {           // fixed-shape tree
         if (threadIdx.x < h) {
 #pragma unroll
             for (int k = 0; k < NV; ++k) red[k][threadIdx.x] += red[k][threadIdx.x + h];
@@ -803,7 +812,14 @@ __device__ __forceinline__ void grid_allsum(const GArgs& a, cg::grid_group& grid
         red[k][threadIdx.x] = s;
     }
     cta_barrier();
-    for (int h = DDA_THREADS / 2; h > 0; h >>= 1) {
+    if (kTreeP2 < DDA_THREADS) {
+        if ((int)threadIdx.x < DDA_THREADS - kTreeP2) {
+#pragma unroll
+            for (int k = 0; k < NV; ++k) red[k][threadIdx.x] += red[k][threadIdx.x + kTreeP2];
+        }
+        cta_barrier();
+    }
+    for (int h = kTreeP2 / 2; h > 0; h >>= 1) {
         if (threadIdx.x < h) {
 #pragma unroll
             for (int k = 0; k < NV; ++k) red[k][threadIdx.x] += red[k][threadIdx.x + h];
@@ -1698,6 +1714,10 @@ int g_scaled_loop = -1;
 unsigned long long* g_trace = nullptr;   // k_sp_loop timeline (internal hook dda__set_loop_trace)
 int g_trace_iters = 0;
 
+#ifndef DDA_SPLOOP_MINB
+#define DDA_SPLOOP_MINB 3
+#endif
+constexpr int kSpLoopMinb = DDA_SPLOOP_MINB;   // CTAs per SM of the persistent loops (tuning build flag)
 constexpr int kCg1Rows = 60000;   // k_sp_cg1 below this many block rows (see pcg_graph_solve)
 constexpr int kClMaxRows = 65536; // k_sp_cg1_cl (one cluster, opt-in) up to this many block rows
 constexpr int kClCtas = 16;       // the cluster: 16 CTAs of kClThreads (non-portable size)
@@ -1812,7 +1832,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
     const void* persist_kernel = pc == DDA_PC_SSOR_AI ? reinterpret_cast<const void*>(k_sp_ssor)
                                  : cg1                ? reinterpret_cast<const void*>(k_sp_cg1<3>)
                                  : lr                 ? reinterpret_cast<const void*>(k_sp_loop<2, 2>)
-                                                      : reinterpret_cast<const void*>(k_sp_loop<3, 0>);
+                                                      : reinterpret_cast<const void*>(k_sp_loop<kSpLoopMinb, 0>);
     if (persist) {
         // The persistent kernels need every CTA co-resident (cooperative launch).  If not even one CTA
         // per SM fits (e.g. a smaller shared-memory carve-out forced by the caller's context), fall
@@ -1853,7 +1873,7 @@ dda_status_t pcg_graph_solve(dda_matrix* K, const double* F, const double* d0, d
         if (persist) {   // every CTA must be co-resident (cooperative launch)
             int per_sm = 0;
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, persist_kernel, DDA_THREADS, 0);
-            if (per_sm > 3) per_sm = 3;
+            if (per_sm > kSpLoopMinb) per_sm = kSpLoopMinb;
             if (per_sm < 1) per_sm = 1;   // (checked above)
             g_persist = cl ? kClCtas : device_sms() * per_sm;
             // small (L2-resident) systems are barrier-latency bound: no more CTAs than ten-row groups
