@@ -1786,8 +1786,16 @@ dda_status_t lr_setup(dda_matrix* K, cudaStream_t st) {
     const size_t ebytes = (size_t)(48 * K->nnzb + 128 * ngrp + 256);
     if ((int64_t)(ebytes / 16) > INT32_MAX) return DDA_ERR_ARG;   // 16 B offsets are int32
     const size_t cbytes = sizeof(unsigned) * (size_t)(ngrp + 1);
-    DDA_CK(dev_alloc(&K->lr_buf, ebytes + cbytes, st));
-    DDA_CK(dev_alloc(reinterpret_cast<void**>(&K->lr_off), sizeof(int32_t) * (size_t)K->nnzb, st));
+    void* buf = nullptr;
+    void* off = nullptr;
+    DDA_CK(dev_alloc(&buf, ebytes + cbytes, st));
+    cudaError_t e = dev_alloc(&off, sizeof(int32_t) * (size_t)K->nnzb, st);
+    if (e != cudaSuccess) {   // publish both or neither (lr_off set means the map is built)
+        dev_free_on(buf, st);
+        return cuda_fail(e);
+    }
+    K->lr_buf = buf;
+    K->lr_off = reinterpret_cast<int32_t*>(off);
     K->lr_bytes = ebytes;
     int g = (int)((K->nnzb + 255) / 256);
     const int cap = device_sms() * 8;
