@@ -478,18 +478,20 @@ __device__ __noinline__ void init_decide(const GArgs& a, const double (&tot)[3])
     }
 }
 
-// q = K x with x = d0 (prelude, D0 = true) or x = d (true residual; skipped when d = 0 by reading Z2)
+// q = K x with x = d0 (prelude, D0 = true) or x = d (true residual; skipped when d = 0 by reading Z2),
+// with the standalone SpMV's column-pair map (v5, 3 CTAs/SM): the 9-lane group map at 6 CTAs/SM took
+// twice as long (0.47 vs 0.24 ms at 1M under ncu)
 template <bool D0>
-__global__ void __launch_bounds__(DDA_THREADS, 6) k_g_spmv_x(const GArgs a) {
+__global__ void __launch_bounds__(DDA_THREADS, 3) k_g_spmv_x(const GArgs a) {
     if (!D0 && a.st->zero_d) return;
     const int lane = threadIdx.x & 31;
     const XPlain xf{D0 ? a.ca->d0 : a.ca->d};
-    for_rows<SPMV_FULL>(a.A, blockIdx.x * WPB + (threadIdx.x >> 5), gridDim.x * WPB, xf, lane,
-                        [&](int i, bool ok, double y0, double y1) {
-                            if (ok && is_out_lane(lane))
-                                *reinterpret_cast<double2*>(a.q + 6 * (size_t)i + 2 * (q_of(lane) / 3)) =
-                                    make_double2(y0, y1);
-                        });
+    for_rows_c<SPMV_FULL, 5>(a.A, blockIdx.x * WPB + (threadIdx.x >> 5), gridDim.x * WPB, xf, lane,
+                             [&](int i, bool ok, double y0, double y1) {
+                                 if (ok)
+                                     *reinterpret_cast<double2*>(a.q + 6 * (size_t)i + 2 * ccol_of(lane)) =
+                                         make_double2(y0, y1);
+                             });
 }
 
 // ||F - q||^2 (or d = 0 when F = 0); last CTA writes rel_res, iterations and status
