@@ -20,7 +20,6 @@
 #include <cooperative_groups.h>
 
 #include <cmath>
-#include <type_traits>
 #include <cstdlib>
 
 #include "ilu_dev.cuh"
@@ -478,9 +477,7 @@ __device__ __noinline__ void init_decide(const GArgs& a, const double (&tot)[3])
     }
 }
 
-// q = K x with x = d0 (prelude, D0 = true) or x = d (true residual; skipped when d = 0 by reading Z2),
-// with the standalone SpMV's column-pair map (v5, 3 CTAs/SM): the 9-lane group map at 6 CTAs/SM took
-// twice as long (0.47 vs 0.24 ms at 1M under ncu)
+// q = K x with x = d0 (prelude, D0 = true) or x = d (true residual; skipped when d = 0 by reading Z2)
 template <bool D0>
 __global__ void __launch_bounds__(DDA_THREADS, 3) k_g_spmv_x(const GArgs a) {
     if (!D0 && a.st->zero_d) return;
@@ -1179,39 +1176,19 @@ __global__ void __launch_bounds__(DDA_THREADS, MINB) k_sp_loop(const GArgs a) {
         alpha = rho / sigma;
         // phase B: r~ -= alpha q; rho' = |r~|^2 and the lower bound sum_i w_i |r~_i|^2 of |L r~|^2
         double rz = 0.0, lb = 0.0;
-        // phase B streams r~, q and w: PB five-row groups in flight per warp (every load issued before any
-        // store, which the compiler cannot reorder itself: r~ is stored), summed pairwise in the order of
-        // a two-group loop, so the result does not depend on PB
-        auto phase_b = [&](auto pbc) {
-            constexpr int PB = decltype(pbc)::value;
-            for (int grp = w0; grp < ngrp; grp += PB * W) {
-                Row5 R[PB];
-                double rr[PB], qq[PB], ww[PB];
-#pragma unroll
-                for (int u = 0; u < PB; ++u) {
-                    R[u] = row5(grp + u * W, lane, n);
-                    rr[u] = 0.0, qq[u] = 0.0, ww[u] = 0.0;
-                    if (R[u].valid) {
-                        rr[u] = ld_cg(a.r + R[u].idx);
-                        qq[u] = ld_cg(a.q + R[u].idx);
-                        ww[u] = __ldg(a.bj_w + R[u].i);
-                    }
-                }
-#pragma unroll
-                for (int u = 0; u < PB; ++u) {
-                    rr[u] = R[u].valid ? rr[u] - alpha * qq[u] : 0.0;
-                    if (R[u].valid) a.r[R[u].idx] = rr[u];
-                }
-#pragma unroll
-                for (int u = 0; u < PB; u += 2) {
-                    if (u == 0 || grp + u * W < ngrp) {
-                        rz += rr[u] * rr[u] + rr[u + 1] * rr[u + 1];
-                        lb += ww[u] * (rr[u] * rr[u]) + ww[u + 1] * (rr[u + 1] * rr[u + 1]);
-                    }
-                }
-            }
-        };
-        phase_b(std::integral_constant<int, 4>{});   // (8 measured the same as 4)
+        for (int grp = w0; grp < ngrp; grp += 2 * W) {
+            const Row5 RA = row5(grp, lane, n);
+            const Row5 RB = row5(grp + W, lane, n);
+            double ra = 0, qa = 0, rb = 0, qb = 0, wa = 0, wb = 0;
+            if (RA.valid) { ra = ld_cg(a.r + RA.idx); qa = ld_cg(a.q + RA.idx); wa = __ldg(a.bj_w + RA.i); }
+            if (RB.valid) { rb = ld_cg(a.r + RB.idx); qb = ld_cg(a.q + RB.idx); wb = __ldg(a.bj_w + RB.i); }
+            const double rva = RA.valid ? ra - alpha * qa : 0.0;
+            const double rvb = RB.valid ? rb - alpha * qb : 0.0;
+            if (RA.valid) a.r[RA.idx] = rva;
+            if (RB.valid) a.r[RB.idx] = rvb;
+            rz += rva * rva + rvb * rvb;
+            lb += wa * (rva * rva) + wb * (rvb * rvb);
+        }
         if (tr) tr[3] = gtimer();
         double bv[2] = {rz, lb}, btot[2];
         grid_allsum<2>(a, grid, 1, bv, btot);
