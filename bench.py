@@ -519,7 +519,7 @@ def main():
                      "bound": "hbm", "achieved": ach, "peak": hbm_peak, "unit": "GB/s", "frac": ach / hbm_peak,
                      "traffic": traffic_for(n, "pcg_" + str(engine)), "peak_source": peak_src,
                      "algorithmic_bytes_per_launch": pcg_bytes, "l2": l2_roofline(n, iters, pcg_ms)},
-        "spmv": {"kernel": "k_spmv<FULL,6>", "ms": spmv_ms, "traffic": traffic_for(n, "spmv"), "gbs": spmv_gbs, "frac_hbm": spmv_gbs / hbm_peak,
+        "spmv": {"kernel": "k_spmv3<FULL,3,5> (column-pair map, two blocks in flight per lane, 3 CTAs/SM)", "ms": spmv_ms, "traffic": traffic_for(n, "spmv"), "gbs": spmv_gbs, "frac_hbm": spmv_gbs / hbm_peak,
                  "gflops": n * (72 + 144 * u) / (spmv_ms * 1e-3) / 1e9, "bytes": spmv_bytes,
                  "timing": "back to back (hot), inputs > L2"},
         "e2e": e2e, "cpu_baseline": cpu, "gpu_launches": int(launches),
