@@ -80,8 +80,11 @@ def l2_roofline(n_blocks: int, iters: int, pcg_ms: float):
         return None
     tbps = e["l2_bytes_per_iter"] * iters / (pcg_ms * 1e-3) / 1e12
     cap = e["lts_cap_bytes_per_cycle"] * e["sm_clock_hz"] / 1e12
-    return {"l2_bytes_per_iter": e["l2_bytes_per_iter"], "achieved_tbps": tbps, "cap_tbps": cap,
-            "frac": tbps / cap, "source": e["source"]}
+    out = {"l2_bytes_per_iter": e["l2_bytes_per_iter"], "achieved_tbps": tbps, "cap_tbps": cap,
+           "frac": tbps / cap, "source": e["source"]}
+    if "note" in e:
+        out["note"] = e["note"]
+    return out
 
 
 def bytes_per_row_spmv(u: float) -> float:
